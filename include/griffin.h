@@ -1,0 +1,213 @@
+/*
+ * griffin.h — C ABI of the B200-native Griffin-GPU conjunctive query path.
+ *
+ * The path (Liu, Wang, Swanson, "Griffin", PPoPP'18; /root/reference/PAPER.md,
+ * cited P:<line>):
+ *   block-parallel Elias-Fano decode (§3.1.1, Alg. 1)
+ *   -> SvS list intersection, merge-path partitioned (§3.1.2) or
+ *      skip-pointer galloping for skewed lengths
+ *   -> BM25 scoring of the survivors (§2.1.3)
+ *   -> top-k selection (§3.1.3)
+ * with docID-range sharding across GPUs (not in the paper).
+ *
+ * Conventions (all entry points):
+ *  - No exceptions cross this boundary; every call returns a griffin_status.
+ *    On failure no output is written and griffin_last_error() returns a
+ *    thread-local message.
+ *  - "host" pointers are ordinary CPU memory, borrowed for the duration of the
+ *    call; the library keeps no input pointer after returning.
+ *  - "device" pointers are CUDA global memory on the index's device; calls that
+ *    take them are asynchronous on the given stream (cudaStream_t passed as
+ *    void*; NULL = the legacy default stream).
+ *  - One call at a time per index handle (calls are serialised by a mutex).
+ *  - docIDs are uint32 in [0, num_docs), num_docs < 2^32 - 1; 0xFFFFFFFF is
+ *    the "no result" sentinel.
+ *  - Results are ordered by score descending, ties by docID ascending
+ *    (SURVEY A16); slots [count, k) hold docID 0xFFFFFFFF and score -inf.
+ *  - Scores are fp32 BM25 with k1/b from griffin_build_opts,
+ *    idf_t = ln(1 + (N - df_t + 0.5)/(df_t + 0.5)) and
+ *    w = idf_t * (tf*(k1+1)) / (tf + k1*((1-b) + b*dl/avgdl)), each term's w
+ *    accumulated in (global df asc, termID asc) order.
+ *
+ * This header is the only interface between the product and its callers; it is
+ * not shared with the test oracle (oracle/), which has its own.
+ */
+#ifndef GRIFFIN_H_
+#define GRIFFIN_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GRIFFIN_MAX_TERMS 16   /* distinct terms per query */
+#define GRIFFIN_MAX_K 4096     /* largest k accepted */
+#define GRIFFIN_MAX_SHARDS 8
+
+typedef struct griffin_index griffin_index; /* opaque; owns device memory + stream */
+
+typedef enum {
+  GRIFFIN_OK = 0,
+  GRIFFIN_ERR_INVALID_ARG = 1, /* bad sizes, term >= V, k == 0 or > GRIFFIN_MAX_K, ... */
+  GRIFFIN_ERR_UNSORTED = 2,    /* a list not strictly increasing or a docID >= N */
+  GRIFFIN_ERR_OOM = 3,         /* device allocation failed / workspace too small */
+  GRIFFIN_ERR_CUDA = 4,        /* CUDA runtime error (message in griffin_last_error) */
+  GRIFFIN_ERR_NCCL = 5,        /* reserved: collective failure reported by a caller */
+  GRIFFIN_ERR_UNSUPPORTED = 6  /* no CUDA device / not sm_100 */
+} griffin_status;
+
+/* Corpus in CSR form (host pointers).  Term t's postings are
+ * docids[list_offsets[t] .. list_offsets[t+1]) with matching tfs; docIDs strictly
+ * increasing and < num_docs; tfs >= 1 (the per-posting "document frequency" of
+ * P:357-361 / P:1009-1010 read as term frequency); tfs > 65535 are
+ * clamped to 65535.  doc_lengths[num_docs] are the BM25 document lengths
+ * (SURVEY A13); their sum must be > 0. */
+typedef struct {
+  uint32_t num_docs;
+  uint32_t num_terms;
+  const uint64_t *list_offsets; /* [num_terms + 1] */
+  const uint32_t *docids;
+  const uint32_t *tfs;
+  const uint32_t *doc_lengths;  /* [num_docs] */
+} griffin_corpus;
+
+typedef struct {
+  uint32_t block_size;   /* EF block length B: 64..512, multiple of 32; 0 -> 128 */
+  double bm25_k1;        /* BM25 k1 (paper silent); <= 0 -> 1.2 */
+  double bm25_b;         /* BM25 b; < 0 -> 0.75 */
+  uint32_t gallop_ratio; /* T: a round gallops iff |S| > T*|R|; 0 -> block_size */
+  int32_t device;        /* CUDA device ordinal to build on; < 0 -> current device */
+  uint32_t shard_index;  /* docID-range shard g of num_shards */
+  uint32_t num_shards;   /* 0 or 1 -> unsharded */
+} griffin_build_opts;
+
+typedef struct {
+  uint32_t shard_index, num_shards;
+  uint32_t doc_base, doc_end;     /* this shard owns docIDs [doc_base, doc_end) */
+  uint32_t block_size, num_terms;
+  uint64_t num_postings;          /* postings stored in this shard */
+  uint64_t num_blocks;
+  uint64_t payload_bytes;         /* EF low+high streams incl. 16-B block padding */
+  uint64_t skip_bytes;            /* per-block first[] + meta[] */
+  uint64_t tf_bytes;              /* packed tf streams */
+  uint64_t device_bytes;          /* everything the index holds on the device */
+} griffin_stats;
+
+/* Intersection mode for griffin_debug_intersect / griffin_set_mode. */
+typedef enum { GRIFFIN_MODE_AUTO = 0, GRIFFIN_MODE_MERGE = 1, GRIFFIN_MODE_GALLOP = 2 } griffin_mode;
+
+/* Per-stage device timings and algorithmic counters accumulated while
+ * profiling is on (griffin_set_profiling).  Times are CUDA-event milliseconds on
+ * the launching stream. */
+typedef struct {
+  double ms_plan, ms_intersect, ms_compact, ms_topk, ms_merge;
+  uint64_t launches_intersect, launches_total;
+  uint64_t alg_bytes;        /* algorithmic bytes read+written by the intersect kernels */
+  uint64_t payload_bytes;    /* compressed EF bytes of the blocks the method had to read */
+  uint64_t decoded_postings; /* postings of those blocks */
+  uint64_t survivors;        /* (docID, score) pairs emitted by intersection rounds */
+} griffin_profile;
+
+/* ---- index ------------------------------------------------------------------
+ * griffin_index_build ("compression ... occurs once ... offline";
+ * P:537-552 EF; P:609-610 fixed-length partitioned EF; Fig. 2 P:216-220 skip
+ * pointers).  Validates the corpus on the host, computes global BM25 statistics
+ * in double (rounded once to f32), keeps this shard's docID range, and
+ * Elias-Fano encodes every list into blocks of B postings ON THE DEVICE
+ * (size pass -> scan -> write pass).  On success *out owns all device memory. */
+griffin_status griffin_index_build(const griffin_corpus *corpus, const griffin_build_opts *opts,
+                                   griffin_index **out);
+void griffin_index_destroy(griffin_index *ix);
+griffin_status griffin_index_stats(const griffin_index *ix, griffin_stats *out);
+
+/* ---- queries (host buffers; synchronous) --------------------------------------
+ * A conjunctive query returns the docs containing every term (P:228-231,
+ * P:269-271), BM25-scored, top k.  Duplicate terms are deduplicated; a term with
+ * an empty list gives count 0.  Output arrays: out_docids[k], out_scores[k]
+ * (GLOBAL docIDs; for a sharded index, this shard's top-k only). */
+griffin_status griffin_query(griffin_index *ix, const uint32_t *terms, uint32_t nterms,
+                             uint32_t k, uint32_t *out_docids, float *out_scores,
+                             uint32_t *out_count);
+
+/* Batch of nq queries: query q is terms[query_offsets[q] .. query_offsets[q+1]).
+ * Outputs [nq*k] docIDs/scores (row q at q*k) and [nq] counts.  The whole batch
+ * runs as one launch per SvS round on the device. */
+griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_t *query_offsets,
+                                   const uint32_t *terms, uint32_t k, uint32_t *out_docids,
+                                   float *out_scores, uint32_t *out_counts);
+
+/* ---- queries (device buffers; asynchronous on `stream`) ------------------------
+ * Same computation with every input and output in device memory.  max_terms is
+ * a host-side bound on terms per query (<= GRIFFIN_MAX_TERMS).  Outputs are the
+ * unique 64-bit keys (f32 score bits << 32) | (0xFFFFFFFF - global docID),
+ * sorted descending ([nq*k], 0 past count) and counts [nq].  Workspace must be
+ * reserved first (griffin_reserve); overflow or a bad term is reported by
+ * griffin_sync_status. */
+griffin_status griffin_reserve(griffin_index *ix, uint32_t nq, const uint32_t *query_offsets,
+                               const uint32_t *terms, uint32_t k);
+griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq,
+                                          const uint32_t *d_query_offsets, const uint32_t *d_terms,
+                                          uint32_t max_terms, uint32_t k, uint64_t *d_out_keys,
+                                          uint32_t *d_out_counts, void *stream);
+/* Synchronise the index's work and return (then clear) any device-side error. */
+griffin_status griffin_sync_status(griffin_index *ix);
+
+/* Shard merge: given G per-shard sorted key runs
+ * d_keys[g][nq*k] and counts d_counts[g][nq] (laid out contiguously, g-major, as
+ * an all-gather produces them), write the global top-k keys and counts.  Exact:
+ * keys are unique, so a global top-k key is in its shard's top-k. */
+griffin_status griffin_merge_topk_device(griffin_index *ix, uint32_t num_runs, uint32_t nq,
+                                         uint32_t k, const uint64_t *d_keys,
+                                         const uint32_t *d_counts, uint64_t *d_out_keys,
+                                         uint32_t *d_out_counts, void *stream);
+/* keys -> (docID, score) rows, sentinel-filled past count. */
+griffin_status griffin_keys_to_results_device(griffin_index *ix, uint32_t nq, uint32_t k,
+                                              const uint64_t *d_keys, const uint32_t *d_counts,
+                                              uint32_t *d_docids, float *d_scores, void *stream);
+
+/* ---- configuration / instrumentation ---------------------------------------- */
+griffin_status griffin_set_mode(griffin_index *ix, int mode); /* griffin_mode; default AUTO */
+griffin_status griffin_set_profiling(griffin_index *ix, int on);
+griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out); /* syncs */
+griffin_status griffin_reset_profile(griffin_index *ix);
+const char *griffin_last_error(void);
+
+/* docID range owned by shard g of G over num_docs docs: [g*ceil(N/G), min(N,(g+1)*ceil(N/G))).
+ * Pure host function (no device needed). */
+griffin_status griffin_shard_range(uint32_t num_docs, uint32_t num_shards, uint32_t shard,
+                                   uint32_t *doc_base, uint32_t *doc_end);
+
+/* Merge-path split of the diagonal d over sorted arrays a[na], b[nb] (host
+ * reference of the device search; Fig. 6, rule "advance in A iff
+ * A[i] <= B[j]", P:690-691 / SURVEY A8) with the matched-pair fix-up of SURVEY
+ * A9 applied when fixup != 0.  Pure host function. */
+griffin_status griffin_merge_path_split(const uint32_t *a, uint32_t na, const uint32_t *b,
+                                        uint32_t nb, uint32_t diag, int fixup, uint32_t *i_out,
+                                        uint32_t *j_out);
+
+/* ---- test-only parity hooks (same conventions) ---------------------------------
+ * Logical EF streams of block `blk` of term t in this shard (low stream of
+ * n*b bits, high stream of L bits, LSB-first u32 words). */
+griffin_status griffin_debug_block_streams(griffin_index *ix, uint32_t term, uint64_t blk,
+                                           uint32_t *first, uint32_t *n, uint32_t *b,
+                                           uint32_t *low, uint64_t low_cap, uint64_t *low_bits,
+                                           uint32_t *high, uint64_t high_cap, uint64_t *high_bits);
+/* Warp-parallel decode (Alg. 1) of term t's whole list in this shard -> GLOBAL docIDs. */
+griffin_status griffin_debug_decode_list(griffin_index *ix, uint32_t term, uint32_t *out,
+                                         uint64_t cap, uint64_t *n);
+/* Decode-only bandwidth kernel over every block of the shard (decode sweep):
+ * returns the device time in ms and writes the XOR of all decoded docIDs (so the
+ * work cannot be elided) to *checksum. */
+griffin_status griffin_debug_decode_all(griffin_index *ix, int iters, double *ms,
+                                        uint64_t *checksum, uint64_t *postings, uint64_t *bytes);
+/* Full docID set of the conjunctive query (GLOBAL docIDs), mode = griffin_mode. */
+griffin_status griffin_debug_intersect(griffin_index *ix, const uint32_t *terms, uint32_t nterms,
+                                       int mode, uint32_t *out_docids, uint64_t cap,
+                                       uint64_t *count);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GRIFFIN_H_ */

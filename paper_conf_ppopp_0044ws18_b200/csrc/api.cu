@@ -1,0 +1,579 @@
+// api.cu — the C ABI of include/griffin.h: host-side validation, global BM25
+// statistics, docID-range sharding, workspace management and the synchronous
+// host-buffer entry points.  Every step of the query path itself runs in the
+// kernels of encode.cu / query.cu; nothing here computes query results.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+namespace griffin {
+
+static thread_local std::string g_err;
+void set_error(const std::string &msg) { g_err = msg; }
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+static griffin_status invalid(const std::string &m) {
+  set_error(m);
+  return GRIFFIN_ERR_INVALID_ARG;
+}
+
+static griffin_status ensure_pinned(griffin_index *ix, size_t bytes) {
+  Workspace &w = ix->ws;
+  if (w.h_pinned_bytes >= bytes) return GRIFFIN_OK;
+  if (w.h_pinned) cudaFreeHost(w.h_pinned);
+  w.h_pinned = nullptr;
+  w.h_pinned_bytes = 0;
+  size_t nb = bytes + bytes / 4 + 4096;
+  GRIFFIN_CUDA_TRY(cudaMallocHost(&w.h_pinned, nb));
+  w.h_pinned_bytes = nb;
+  return GRIFFIN_OK;
+}
+
+// Host validation of one batch's query terms + workspace reservation.
+static griffin_status reserve_for(griffin_index *ix, uint32_t nq, const uint32_t *qoffs,
+                                  const uint32_t *terms, uint32_t k, uint32_t *max_terms) {
+  if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
+  uint64_t caps = 0, units = 0;
+  uint32_t mt = 1;
+  for (uint32_t q = 0; q < nq; ++q) {
+    if (qoffs[q + 1] < qoffs[q]) return invalid("query_offsets must be non-decreasing");
+    const uint32_t n = qoffs[q + 1] - qoffs[q];
+    if (n == 0) return invalid("a query has no terms");
+    std::vector<uint32_t> ts(terms + qoffs[q], terms + qoffs[q + 1]);
+    for (uint32_t t : ts)
+      if (t >= ix->V) return invalid("query term >= num_terms");
+    std::sort(ts.begin(), ts.end());
+    ts.erase(std::unique(ts.begin(), ts.end()), ts.end());
+    if (ts.size() > (size_t)GRIFFIN_MAX_TERMS) return invalid("more than GRIFFIN_MAX_TERMS distinct terms");
+    mt = std::max<uint32_t>(mt, (uint32_t)ts.size());
+    uint64_t c, u;
+    host_query_bounds(ix, terms + qoffs[q], n, &c, &u);
+    caps += c;
+    units += u;
+  }
+  if (max_terms) *max_terms = mt;
+  return reserve_ws(ix, nq, units, caps);
+}
+
+static griffin_status read_status(griffin_index *ix) {
+  int status = 0;
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(&status, ix->ws.scal.as<unsigned long long>() + kScalStatus,
+                                   sizeof(int), cudaMemcpyDeviceToHost, ix->stream));
+  GRIFFIN_CUDA_TRY(cudaStreamSynchronize(ix->stream));
+  if (status) {
+    GRIFFIN_CUDA_TRY(cudaMemsetAsync(ix->ws.scal.as<unsigned long long>() + kScalStatus, 0, 8,
+                                     ix->stream));
+    GRIFFIN_CUDA_TRY(cudaStreamSynchronize(ix->stream));
+    if (status & kStatusOverflow) {
+      set_error("query workspace overflow (reserve more with griffin_reserve)");
+      return GRIFFIN_ERR_OOM;
+    }
+    set_error("invalid query term(s) detected on the device");
+    return GRIFFIN_ERR_INVALID_ARG;
+  }
+  return GRIFFIN_OK;
+}
+
+}  // namespace griffin
+
+using namespace griffin;
+
+extern "C" {
+
+const char *griffin_last_error(void) { return g_err.c_str(); }
+
+griffin_status griffin_shard_range(uint32_t num_docs, uint32_t num_shards, uint32_t shard,
+                                   uint32_t *doc_base, uint32_t *doc_end) {
+  if (num_shards == 0 || num_shards > GRIFFIN_MAX_SHARDS || shard >= num_shards || !doc_base ||
+      !doc_end)
+    return invalid("bad shard arguments");
+  const uint64_t per = ((uint64_t)num_docs + num_shards - 1) / num_shards;
+  *doc_base = (uint32_t)std::min<uint64_t>((uint64_t)shard * per, num_docs);
+  *doc_end = (uint32_t)std::min<uint64_t>((uint64_t)(shard + 1) * per, num_docs);
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_merge_path_split(const uint32_t *a, uint32_t na, const uint32_t *b,
+                                        uint32_t nb, uint32_t diag, int fixup, uint32_t *i_out,
+                                        uint32_t *j_out) {
+  if ((!a && na) || (!b && nb) || diag > na + nb || !i_out || !j_out)
+    return invalid("bad merge-path arguments");
+  merge_path_split([&](uint32_t i) { return a[i]; }, na, [&](uint32_t j) { return b[j]; }, nb,
+                   diag, fixup != 0, i_out, j_out);
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_opts *o,
+                                   griffin_index **out) {
+  if (!c || !out) return invalid("null corpus/out");
+  *out = nullptr;
+  griffin_build_opts opts{};
+  if (o) opts = *o;
+  const uint32_t B = opts.block_size ? opts.block_size : 128;
+  if (B < 64 || B > 512 || (B % 32)) return invalid("block_size must be 64..512 and a multiple of 32");
+  const double k1 = opts.bm25_k1 > 0 ? opts.bm25_k1 : 1.2;
+  const double bb = opts.bm25_b >= 0 ? opts.bm25_b : 0.75;
+  const uint32_t G = opts.num_shards ? opts.num_shards : 1;
+  if (G > GRIFFIN_MAX_SHARDS || opts.shard_index >= G) return invalid("bad shard index / count");
+  const uint32_t N = c->num_docs, V = c->num_terms;
+  if (N == 0 || N >= 0xFFFFFFFFu) return invalid("num_docs must be in [1, 2^32-2]");
+  if (!c->list_offsets || !c->doc_lengths) return invalid("null corpus arrays");
+  if (c->list_offsets[0] != 0) return invalid("list_offsets[0] must be 0");
+  for (uint32_t t = 0; t < V; ++t)
+    if (c->list_offsets[t + 1] < c->list_offsets[t]) return invalid("list_offsets not monotone");
+  const uint64_t P = c->list_offsets[V];
+  if (P && (!c->docids || !c->tfs)) return invalid("null docids/tfs");
+  for (uint32_t t = 0; t < V; ++t) {
+    const uint64_t a = c->list_offsets[t], e = c->list_offsets[t + 1];
+    if (e - a > 0xFFFFFFFFull) return invalid("list longer than 2^32-1");
+    for (uint64_t p = a; p < e; ++p) {
+      if (c->docids[p] >= N || (p > a && c->docids[p] <= c->docids[p - 1])) {
+        set_error("list " + std::to_string(t) + " not strictly increasing or docID >= num_docs");
+        return GRIFFIN_ERR_UNSORTED;
+      }
+      if (c->tfs[p] == 0) return invalid("tf must be >= 1");
+    }
+  }
+  uint64_t sum_dl = 0;
+  for (uint32_t d = 0; d < N; ++d) sum_dl += c->doc_lengths[d];
+  if (sum_dl == 0) return invalid("sum of doc_lengths must be > 0");
+
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    set_error("no CUDA device");
+    return GRIFFIN_ERR_UNSUPPORTED;
+  }
+  int dev = opts.device;
+  if (dev < 0) cudaGetDevice(&dev);
+  if (dev >= ndev) return invalid("device ordinal out of range");
+  cudaDeviceProp prop;
+  GRIFFIN_CUDA_TRY(cudaGetDeviceProperties(&prop, dev));
+  if (prop.major != 10 || prop.minor != 0) {
+    set_error("this build targets sm_100a (B200); device is sm_" + std::to_string(prop.major) +
+              std::to_string(prop.minor));
+    return GRIFFIN_ERR_UNSUPPORTED;
+  }
+  DeviceGuard guard(dev);
+
+  griffin_index *ix = new griffin_index();
+  ix->device = dev;
+  ix->B = B;
+  ix->T = opts.gallop_ratio ? opts.gallop_ratio : B;
+  ix->D = std::max<uint32_t>(2, 1024 / B);
+  ix->k1 = k1;
+  ix->bm25_b = bb;
+  ix->N = N;
+  ix->V = V;
+  ix->shard = opts.shard_index;
+  ix->nshards = G;
+  griffin_shard_range(N, G, opts.shard_index, &ix->doc_base, &ix->doc_end);
+  ix->k1p1 = (float)(k1 + 1.0);
+  if (cudaStreamCreateWithFlags(&ix->stream, cudaStreamNonBlocking) != cudaSuccess) {
+    delete ix;
+    set_error("cudaStreamCreate failed");
+    return GRIFFIN_ERR_CUDA;
+  }
+  // global statistics (double, rounded once)
+  const double avgdl = (double)sum_dl / (double)N;
+  ix->h_terms.assign(V, TermInfo{});
+  for (uint32_t t = 0; t < V; ++t) {
+    const double df = (double)(c->list_offsets[t + 1] - c->list_offsets[t]);
+    ix->h_terms[t].df_global = (uint32_t)(c->list_offsets[t + 1] - c->list_offsets[t]);
+    ix->h_terms[t].idf = (float)std::log1p(((double)N - df + 0.5) / (df + 0.5));
+  }
+  const uint32_t nd = ix->doc_end - ix->doc_base;
+  std::vector<float> norm(std::max<uint32_t>(nd, 1));
+  for (uint32_t d = 0; d < nd; ++d)
+    norm[d] = (float)(k1 * ((1.0 - bb) + bb * ((double)c->doc_lengths[ix->doc_base + d] / avgdl)));
+  // this shard's slice of every list, local docIDs
+  std::vector<uint64_t> post_off(V + 1, 0);
+  std::vector<uint64_t> lo(V), hi(V);
+  for (uint32_t t = 0; t < V; ++t) {
+    const uint32_t *a = c->docids + c->list_offsets[t], *e = c->docids + c->list_offsets[t + 1];
+    lo[t] = (G == 1) ? c->list_offsets[t] : (std::lower_bound(a, e, ix->doc_base) - c->docids);
+    hi[t] = (G == 1) ? c->list_offsets[t + 1] : (std::lower_bound(a, e, ix->doc_end) - c->docids);
+    post_off[t + 1] = post_off[t] + (hi[t] - lo[t]);
+  }
+  const uint64_t Ps = post_off[V];
+  std::vector<uint32_t> ldoc(std::max<uint64_t>(Ps, 1)), ltf(std::max<uint64_t>(Ps, 1));
+  for (uint32_t t = 0; t < V; ++t) {
+    uint64_t o = post_off[t];
+    for (uint64_t p = lo[t]; p < hi[t]; ++p, ++o) {
+      ldoc[o] = c->docids[p] - ix->doc_base;
+      ltf[o] = std::min<uint32_t>(c->tfs[p], 65535u);
+    }
+  }
+  griffin_status s = encode_index(ix, ldoc.data(), ltf.data(), post_off);
+  if (s == GRIFFIN_OK) {
+    cudaError_t e = cudaMalloc(&ix->d_norm, norm.size() * 4);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(ix->d_norm, norm.data(), norm.size() * 4, cudaMemcpyHostToDevice,
+                          ix->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(ix->stream);
+    if (e != cudaSuccess) {
+      set_error(std::string("norm upload: ") + cudaGetErrorString(e));
+      s = GRIFFIN_ERR_CUDA;
+    }
+  }
+  if (s != GRIFFIN_OK) {
+    griffin_index_destroy(ix);
+    return s;
+  }
+  *out = ix;
+  return GRIFFIN_OK;
+}
+
+void griffin_index_destroy(griffin_index *ix) {
+  if (!ix) return;
+  {
+    DeviceGuard guard(ix->device);
+    if (ix->stream) cudaStreamSynchronize(ix->stream);
+    cudaFree(ix->d_terms);
+    cudaFree(ix->d_first);
+    cudaFree(ix->d_meta);
+    cudaFree(ix->d_payload);
+    cudaFree(ix->d_tfw);
+    cudaFree(ix->d_norm);
+    Workspace &w = ix->ws;
+    for (DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel, &w.qmode,
+                      &w.unit_base, &w.unit_off, &w.unit_cnt, &w.rbuf0, &w.rbuf1, &w.bump, &w.scal,
+                      &w.keys, &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms})
+      b->release();
+    if (w.h_pinned) cudaFreeHost(w.h_pinned);
+    for (cudaEvent_t e : ix->ev_pool) cudaEventDestroy(e);
+    if (ix->stream) cudaStreamDestroy(ix->stream);
+  }
+  delete ix;
+}
+
+griffin_status griffin_index_stats(const griffin_index *ix, griffin_stats *out) {
+  if (!ix || !out) return invalid("null argument");
+  std::memset(out, 0, sizeof(*out));
+  out->shard_index = ix->shard;
+  out->num_shards = ix->nshards;
+  out->doc_base = ix->doc_base;
+  out->doc_end = ix->doc_end;
+  out->block_size = ix->B;
+  out->num_terms = ix->V;
+  out->num_postings = ix->postings;
+  out->num_blocks = ix->nblocks;
+  out->payload_bytes = ix->payload16 * 16;
+  out->skip_bytes = ix->nblocks * 12;
+  out->tf_bytes = ix->tf_words * 4;
+  out->device_bytes = out->payload_bytes + out->skip_bytes + out->tf_bytes +
+                      (uint64_t)ix->V * sizeof(TermInfo) + (uint64_t)(ix->doc_end - ix->doc_base) * 4;
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_t *qoffs,
+                                   const uint32_t *terms, uint32_t k, uint32_t *out_docids,
+                                   float *out_scores, uint32_t *out_counts) {
+  if (!ix) return invalid("null index");
+  if (nq == 0) return GRIFFIN_OK;
+  if (!qoffs || !terms || !out_docids || !out_scores || !out_counts) return invalid("null argument");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  uint32_t max_terms = 1;
+  griffin_status s = reserve_for(ix, nq, qoffs, terms, k, &max_terms);
+  if (s) return s;
+  Workspace &w = ix->ws;
+  const uint64_t nt = qoffs[nq];
+  const size_t nk = (size_t)nq * k;
+  GRIFFIN_CUDA_TRY(w.qoffs.reserve(((size_t)nq + 1) * 4));
+  GRIFFIN_CUDA_TRY(w.qterms.reserve(std::max<uint64_t>(nt, 1) * 4));
+  GRIFFIN_CUDA_TRY(w.keys.reserve(nk * 8));
+  GRIFFIN_CUDA_TRY(w.counts.reserve((size_t)nq * 4));
+  GRIFFIN_CUDA_TRY(w.docids.reserve(nk * 4));
+  GRIFFIN_CUDA_TRY(w.scores.reserve(nk * 4));
+  // pinned staging: [qoffs | terms | docids | scores | counts]
+  const size_t b_in = ((size_t)nq + 1 + nt) * 4, b_out = nk * 8 + (size_t)nq * 4;
+  if ((s = ensure_pinned(ix, b_in + b_out))) return s;
+  uint8_t *hp = static_cast<uint8_t *>(w.h_pinned);
+  std::memcpy(hp, qoffs, ((size_t)nq + 1) * 4);
+  std::memcpy(hp + ((size_t)nq + 1) * 4, terms, nt * 4);
+  cudaStream_t st = ix->stream;
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qoffs.p, hp, ((size_t)nq + 1) * 4, cudaMemcpyHostToDevice, st));
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qterms.p, hp + ((size_t)nq + 1) * 4, nt * 4,
+                                   cudaMemcpyHostToDevice, st));
+  s = run_batch(ix, nq, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), max_terms, k,
+                w.keys.as<uint64_t>(), w.counts.as<uint32_t>(), st, true, ix->mode);
+  if (s) return s;
+  if ((s = launch_keys_to_results(ix, nq, k, w.keys.as<uint64_t>(), w.counts.as<uint32_t>(),
+                                  w.docids.as<uint32_t>(), w.scores.as<float>(), st)))
+    return s;
+  uint8_t *ho = hp + b_in;
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho, w.docids.p, nk * 4, cudaMemcpyDeviceToHost, st));
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho + nk * 4, w.scores.p, nk * 4, cudaMemcpyDeviceToHost, st));
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho + nk * 8, w.counts.p, (size_t)nq * 4, cudaMemcpyDeviceToHost, st));
+  if ((s = read_status(ix))) return s;  // synchronises
+  std::memcpy(out_docids, ho, nk * 4);
+  std::memcpy(out_scores, ho + nk * 4, nk * 4);
+  std::memcpy(out_counts, ho + nk * 8, (size_t)nq * 4);
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_query(griffin_index *ix, const uint32_t *terms, uint32_t nterms, uint32_t k,
+                             uint32_t *out_docids, float *out_scores, uint32_t *out_count) {
+  if (nterms == 0) return invalid("nterms must be > 0");
+  const uint32_t offs[2] = {0, nterms};
+  return griffin_query_batch(ix, 1, offs, terms, k, out_docids, out_scores, out_count);
+}
+
+griffin_status griffin_reserve(griffin_index *ix, uint32_t nq, const uint32_t *qoffs,
+                               const uint32_t *terms, uint32_t k) {
+  if (!ix || (nq && (!qoffs || !terms))) return invalid("null argument");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  return reserve_for(ix, nq, qoffs, terms, k, nullptr);
+}
+
+griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs,
+                                          const uint32_t *d_terms, uint32_t max_terms, uint32_t k,
+                                          uint64_t *d_out_keys, uint32_t *d_out_counts,
+                                          void *stream) {
+  if (!ix) return invalid("null index");
+  if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
+  if (max_terms == 0 || max_terms > GRIFFIN_MAX_TERMS) return invalid("max_terms out of range");
+  if (nq == 0) return GRIFFIN_OK;
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  return run_batch(ix, nq, d_qoffs, d_terms, max_terms, k, d_out_keys, d_out_counts,
+                   static_cast<cudaStream_t>(stream), true, ix->mode);
+}
+
+griffin_status griffin_sync_status(griffin_index *ix) {
+  if (!ix) return invalid("null index");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  GRIFFIN_CUDA_TRY(cudaDeviceSynchronize());
+  if (!ix->ws.scal.p) return GRIFFIN_OK;
+  return read_status(ix);
+}
+
+griffin_status griffin_merge_topk_device(griffin_index *ix, uint32_t num_runs, uint32_t nq,
+                                         uint32_t k, const uint64_t *d_keys,
+                                         const uint32_t *d_counts, uint64_t *d_out_keys,
+                                         uint32_t *d_out_counts, void *stream) {
+  if (!ix) return invalid("null index");
+  if (num_runs == 0 || num_runs > 32) return invalid("num_runs must be in [1, 32]");
+  if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  return launch_merge_topk(ix, num_runs, nq, k, d_keys, d_counts, d_out_keys, d_out_counts,
+                           static_cast<cudaStream_t>(stream));
+}
+
+griffin_status griffin_keys_to_results_device(griffin_index *ix, uint32_t nq, uint32_t k,
+                                              const uint64_t *d_keys, const uint32_t *d_counts,
+                                              uint32_t *d_docids, float *d_scores, void *stream) {
+  if (!ix) return invalid("null index");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  return launch_keys_to_results(ix, nq, k, d_keys, d_counts, d_docids, d_scores,
+                                static_cast<cudaStream_t>(stream));
+}
+
+griffin_status griffin_set_mode(griffin_index *ix, int mode) {
+  if (!ix || mode < 0 || mode > 2) return invalid("mode must be 0 (auto), 1 (merge) or 2 (gallop)");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  ix->mode = mode;
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_set_profiling(griffin_index *ix, int on) {
+  if (!ix) return invalid("null index");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  ix->profiling = on != 0;
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_reset_profile(griffin_index *ix) {
+  if (!ix) return invalid("null index");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  GRIFFIN_CUDA_TRY(cudaDeviceSynchronize());
+  ix->prof = griffin_profile{};
+  ix->pending.clear();
+  ix->ev_next = 0;
+  ix->launch_count = 0;
+  if (ix->ws.scal.p) GRIFFIN_CUDA_TRY(cudaMemset(ix->ws.scal.p, 0, 4 * 8));
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
+  if (!ix || !out) return invalid("null argument");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  GRIFFIN_CUDA_TRY(cudaDeviceSynchronize());
+  for (auto &p : ix->pending) {
+    float ms = 0.f;
+    GRIFFIN_CUDA_TRY(cudaEventElapsedTime(&ms, p.second.first, p.second.second));
+    double *slot[5] = {&ix->prof.ms_plan, &ix->prof.ms_intersect, &ix->prof.ms_compact,
+                       &ix->prof.ms_topk, &ix->prof.ms_merge};
+    *slot[p.first] += ms;
+    if (p.first == 1) ix->prof.launches_intersect += 1;
+  }
+  ix->pending.clear();
+  ix->ev_next = 0;
+  *out = ix->prof;
+  out->launches_total = ix->launch_count;
+  if (ix->ws.scal.p) {
+    unsigned long long c[4];
+    GRIFFIN_CUDA_TRY(cudaMemcpy(c, ix->ws.scal.p, sizeof(c), cudaMemcpyDeviceToHost));
+    out->alg_bytes = c[0];
+    out->payload_bytes = c[1];
+    out->decoded_postings = c[2];
+    out->survivors = c[3];
+  }
+  return GRIFFIN_OK;
+}
+
+// ---- debug hooks ------------------------------------------------------------------
+
+griffin_status griffin_debug_block_streams(griffin_index *ix, uint32_t term, uint64_t blk,
+                                           uint32_t *first, uint32_t *n, uint32_t *b,
+                                           uint32_t *low, uint64_t low_cap, uint64_t *low_bits,
+                                           uint32_t *high, uint64_t high_cap, uint64_t *high_bits) {
+  if (!ix || term >= ix->V) return invalid("bad term");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  const TermInfo &t = ix->h_terms[term];
+  if (blk >= t.nblocks) return invalid("bad block");
+  const uint64_t gb = (uint64_t)t.block0 + blk;
+  uint2 m;
+  uint32_t f;
+  GRIFFIN_CUDA_TRY(cudaMemcpy(&m, ix->d_meta + gb, 8, cudaMemcpyDeviceToHost));
+  GRIFFIN_CUDA_TRY(cudaMemcpy(&f, ix->d_first + gb, 4, cudaMemcpyDeviceToHost));
+  const uint32_t bb = meta_b(m.y), nn = meta_n(m.y), hw = meta_hw(m.y);
+  const uint32_t lw = low_words(nn, bb);
+  std::vector<uint32_t> words((size_t)(lw + hw + 3) / 4 * 4);
+  GRIFFIN_CUDA_TRY(cudaMemcpy(words.data(), ix->d_payload + m.x, words.size() * 4,
+                              cudaMemcpyDeviceToHost));
+  // logical high-stream length: position of the n-th one + 1
+  uint64_t L = 0, ones = 0;
+  for (uint64_t p = 0; p < (uint64_t)hw * 32 && ones < nn; ++p)
+    if ((words[lw + p / 32] >> (p % 32)) & 1u) {
+      ++ones;
+      L = p + 1;
+    }
+  const uint64_t lb = (uint64_t)nn * bb;
+  if ((lb + 31) / 32 > low_cap || (L + 31) / 32 > high_cap) return invalid("capacity too small");
+  *first = f + ix->doc_base;
+  *n = nn;
+  *b = bb;
+  *low_bits = lb;
+  *high_bits = L;
+  for (uint64_t i = 0; i < (lb + 31) / 32; ++i) {
+    uint32_t v = words[i];
+    if (i == lb / 32 && (lb % 32)) v &= (1u << (lb % 32)) - 1u;
+    low[i] = v;
+  }
+  for (uint64_t i = 0; i < (L + 31) / 32; ++i) {
+    uint32_t v = words[lw + i];
+    if (i == L / 32 && (L % 32)) v &= (1u << (L % 32)) - 1u;
+    high[i] = v;
+  }
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_debug_decode_list(griffin_index *ix, uint32_t term, uint32_t *out,
+                                         uint64_t cap, uint64_t *n) {
+  if (!ix || term >= ix->V || !n) return invalid("bad arguments");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  const TermInfo &t = ix->h_terms[term];
+  *n = t.df_local;
+  if (t.df_local > cap) return invalid("capacity too small");
+  if (!t.df_local) return GRIFFIN_OK;
+  uint32_t *d = nullptr;
+  GRIFFIN_CUDA_TRY(cudaMalloc(&d, (size_t)t.nblocks * ix->B * 4));
+  griffin_status s = launch_decode_list(ix, term, d, ix->stream);
+  if (!s) {
+    cudaError_t e = cudaMemcpyAsync(out, d, (size_t)t.df_local * 4, cudaMemcpyDeviceToHost, ix->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(ix->stream);
+    if (e != cudaSuccess) {
+      set_error(cudaGetErrorString(e));
+      s = GRIFFIN_ERR_CUDA;
+    }
+  }
+  cudaFree(d);
+  return s;
+}
+
+griffin_status griffin_debug_decode_all(griffin_index *ix, int iters, double *ms,
+                                        uint64_t *checksum, uint64_t *postings, uint64_t *bytes) {
+  if (!ix || iters <= 0) return invalid("bad arguments");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  unsigned long long *acc = nullptr;
+  GRIFFIN_CUDA_TRY(cudaMalloc(&acc, 3 * 8));
+  GRIFFIN_CUDA_TRY(cudaMemsetAsync(acc, 0, 24, ix->stream));
+  griffin_status s = launch_decode_all(ix, acc, ix->stream);  // warm-up
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  GRIFFIN_CUDA_TRY(cudaMemsetAsync(acc, 0, 24, ix->stream));
+  cudaEventRecord(a, ix->stream);
+  for (int i = 0; i < iters && !s; ++i) s = launch_decode_all(ix, acc, ix->stream);
+  cudaEventRecord(b, ix->stream);
+  unsigned long long h[3] = {0, 0, 0};
+  cudaMemcpyAsync(h, acc, 24, cudaMemcpyDeviceToHost, ix->stream);
+  cudaError_t e = cudaStreamSynchronize(ix->stream);
+  float t = 0;
+  cudaEventElapsedTime(&t, a, b);
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(acc);
+  if (e != cudaSuccess) {
+    set_error(cudaGetErrorString(e));
+    return GRIFFIN_ERR_CUDA;
+  }
+  if (s) return s;
+  if (ms) *ms = t / iters;
+  if (checksum) *checksum = h[0];
+  if (postings) *postings = h[1] / iters;
+  if (bytes) *bytes = h[2] / iters;
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_debug_intersect(griffin_index *ix, const uint32_t *terms, uint32_t nterms,
+                                       int mode, uint32_t *out_docids, uint64_t cap,
+                                       uint64_t *count) {
+  if (!ix || !terms || nterms == 0 || !count) return invalid("bad arguments");
+  if (mode < 0 || mode > 2) return invalid("bad mode");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  const uint32_t offs[2] = {0, nterms};
+  uint32_t max_terms = 1;
+  griffin_status s = reserve_for(ix, 1, offs, terms, 1, &max_terms);
+  if (s) return s;
+  Workspace &w = ix->ws;
+  GRIFFIN_CUDA_TRY(w.qoffs.reserve(8));
+  GRIFFIN_CUDA_TRY(w.qterms.reserve((size_t)nterms * 4));
+  cudaStream_t st = ix->stream;
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qoffs.p, offs, 8, cudaMemcpyHostToDevice, st));
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qterms.p, terms, (size_t)nterms * 4, cudaMemcpyHostToDevice, st));
+  s = run_batch(ix, 1, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), max_terms, 1, nullptr,
+                nullptr, st, false, mode);
+  if (s) return s;
+  if ((s = read_status(ix))) return s;
+  return copy_final_docids(ix, out_docids, cap, count);
+}
+
+}  // extern "C"

@@ -1,0 +1,172 @@
+// internal.h — host-side definition of griffin_index and launcher prototypes.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/griffin.h"
+#include "griffin_dev.cuh"
+
+namespace griffin {
+
+void set_error(const std::string &msg);
+
+#define GRIFFIN_CUDA_TRY(expr)                                                          \
+  do {                                                                                   \
+    cudaError_t _e = (expr);                                                             \
+    if (_e != cudaSuccess) {                                                             \
+      ::griffin::set_error(std::string(#expr) + ": " + cudaGetErrorString(_e));          \
+      return _e == cudaErrorMemoryAllocation ? GRIFFIN_ERR_OOM : GRIFFIN_ERR_CUDA;        \
+    }                                                                                    \
+  } while (0)
+
+// Device status bits (set by kernels, read by griffin_sync_status).
+enum : int { kStatusBadTerm = 1, kStatusOverflow = 2, kStatusTooManyTerms = 4 };
+
+// Query modes per (query, round).
+enum : uint32_t { kModeNone = 0, kModeMerge = 1, kModeGallop = 2, kModeAll = 3 };
+
+// Grow-only device buffer.
+struct DevBuf {
+  void *p = nullptr;
+  size_t bytes = 0;
+  cudaError_t reserve(size_t want) {
+    if (want <= bytes) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+    size_t nb = want + want / 4 + 256;
+    cudaError_t e = cudaMalloc(&p, nb);
+    if (e == cudaSuccess) bytes = nb;
+    return e;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+  }
+  template <class T> T *as() const { return static_cast<T *>(p); }
+};
+
+// Query workspace (all grow-only; sized by griffin_reserve / the host API).
+struct Workspace {
+  DevBuf plan_terms, plan_m, cap, cap_off, rcount, rsel, qmode, unit_base;  // per query
+  DevBuf unit_off, unit_cnt;                                                // per unit
+  DevBuf rbuf0, rbuf1, bump;                                                // per survivor
+  DevBuf scal;       // scalars: counters, status, bump ctr, unit ctr
+  DevBuf keys, counts, docids, scores, qoffs, qterms;  // host-API staging on device
+  size_t nq_cap = 0, unit_cap = 0, entry_cap = 0;
+  // pinned host staging
+  void *h_pinned = nullptr;
+  size_t h_pinned_bytes = 0;
+};
+
+// Offsets of the scalar block (u64 slots).
+enum : int {
+  kScalCounters = 0,  // 4 x u64: alg bytes, payload bytes, decoded postings, survivors
+  kScalBump = 4,      // u64 bump counter
+  kScalUnitCtr = 5,   // u32 unit ticket counter (in a u64 slot)
+  kScalStatus = 6,    // int status
+  kScalTotals = 7,    // u64 x2: sum cap, sum units (written by plan kernels)
+  kScalCount = 10
+};
+
+struct RoundArgs {
+  uint32_t nq, round, D, T;
+  int forced_mode;
+  const uint32_t *plan_terms;
+  const uint32_t *plan_m;
+  const uint32_t *cap;
+  const uint64_t *cap_off;
+  uint32_t *rcount;
+  uint8_t *rsel;
+  uint32_t *qmode;
+  uint64_t *unit_base;
+  uint64_t *unit_off;
+  uint32_t *unit_cnt;
+  uint64_t unit_cap;
+  const uint2 *rprev;
+  uint2 *rnext;
+  uint2 *bump;
+  uint64_t entry_cap;
+  unsigned long long *scal;
+};
+
+}  // namespace griffin
+
+struct griffin_index {
+  std::mutex mu;
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  // options
+  uint32_t B = 128, T = 128, D = 8;
+  double k1 = 1.2, bm25_b = 0.75;
+  uint32_t shard = 0, nshards = 1, doc_base = 0, doc_end = 0, N = 0, V = 0;
+  float k1p1 = 0.f;
+  // device index
+  griffin::TermInfo *d_terms = nullptr;
+  uint32_t *d_first = nullptr;
+  uint2 *d_meta = nullptr;
+  uint4 *d_payload = nullptr;
+  uint32_t *d_tfw = nullptr;
+  float *d_norm = nullptr;
+  uint64_t nblocks = 0, payload16 = 0, tf_words = 0, postings = 0;
+  std::vector<griffin::TermInfo> h_terms;
+  // query state
+  griffin::Workspace ws;
+  int mode = 0;
+  bool profiling = false;
+  griffin_profile prof{};
+  std::vector<cudaEvent_t> ev_pool;
+  std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending;  // stage, events
+  size_t ev_next = 0;
+  uint64_t launch_count = 0;  // kernels launched by this handle (always on)
+
+  griffin::DevIndex dev() const {
+    griffin::DevIndex d;
+    d.terms = d_terms;
+    d.first = d_first;
+    d.meta = d_meta;
+    d.payload = d_payload;
+    d.tfw = d_tfw;
+    d.norm = d_norm;
+    d.num_terms = V;
+    d.doc_base = doc_base;
+    d.n_docs = doc_end - doc_base;
+    d.B = B;
+    d.log2B = 0;
+    d.k1p1 = k1p1;
+    return d;
+  }
+};
+
+namespace griffin {
+
+// encode.cu
+griffin_status encode_index(griffin_index *ix, const uint32_t *h_docids_local,
+                            const uint32_t *h_tfs, const std::vector<uint64_t> &post_off);
+// query.cu
+griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs,
+                         const uint32_t *d_terms, uint32_t max_terms, uint32_t k,
+                         uint64_t *d_keys, uint32_t *d_counts, cudaStream_t st, bool final_topk,
+                         int forced_mode);
+griffin_status reserve_ws(griffin_index *ix, uint32_t nq, uint64_t units, uint64_t entries);
+griffin_status launch_merge_topk(griffin_index *ix, uint32_t G, uint32_t nq, uint32_t k,
+                                 const uint64_t *d_keys, const uint32_t *d_counts,
+                                 uint64_t *d_out_keys, uint32_t *d_out_counts, cudaStream_t st);
+griffin_status launch_keys_to_results(griffin_index *ix, uint32_t nq, uint32_t k,
+                                      const uint64_t *d_keys, const uint32_t *d_counts,
+                                      uint32_t *d_docids, float *d_scores, cudaStream_t st);
+griffin_status launch_decode_list(griffin_index *ix, uint32_t term, uint32_t *d_out,
+                                  cudaStream_t st);
+griffin_status launch_decode_all(griffin_index *ix, unsigned long long *d_acc, cudaStream_t st);
+// copies the final survivor docIDs (global) of query 0 after run_batch(final_topk=false)
+griffin_status copy_final_docids(griffin_index *ix, uint32_t *h_out, uint64_t cap, uint64_t *count);
+// per-query bounds used to size the workspace (same rule as the device plan kernel)
+void host_query_bounds(const griffin_index *ix, const uint32_t *terms, uint32_t nterms,
+                       uint64_t *cap, uint64_t *units);
+
+}  // namespace griffin

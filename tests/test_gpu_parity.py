@@ -1,0 +1,301 @@
+"""Parity of the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar (BASELINE.json north_star): docID sets and top-k ordering bit-exact with ties
+by docID; BM25 scores within 1e-5 relative — in practice bit-identical, which is
+what these tests require (same f32 op order on both sides)."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ppopp_0044ws18_b200 as g
+from helpers import corpus_from_lists, random_corpus, random_queries
+from synth import QueryLog, make_pair_workload, make_workload
+
+pytestmark = pytest.mark.gpu
+
+
+def _bits(a):
+    return np.asarray(a, np.float32).view(np.uint32)
+
+
+def assert_topk_equal(gd, gs, gc, od, os_, oc, rel=1e-5):
+    assert np.array_equal(np.asarray(gc), np.asarray(oc)), "counts differ"
+    assert np.array_equal(gd, od), "docIDs / order differ"
+    fin = np.isfinite(os_)
+    assert np.array_equal(np.isfinite(gs), fin)
+    assert np.all(np.abs(gs[fin] - os_[fin]) <= rel * np.abs(os_[fin]))
+    # the f32 op order is identical on both sides: expect identical bits
+    assert np.array_equal(_bits(gs), _bits(os_)), "scores not bit-identical"
+
+
+@pytest.fixture(scope="module")
+def tiny():
+    c, ql, cfg = make_workload("tiny")
+    return c, ql, oracle.OracleIndex(c, block_size=128)
+
+
+@pytest.fixture(scope="module")
+def tiny_gpu(tiny):
+    return g.GriffinIndex(tiny[0], block_size=128)
+
+
+# ---------------------------------------------------------------- codec
+
+@pytest.mark.parametrize("B", [64, 128, 256, 512])
+def test_encoder_logical_streams_match_oracle(B):
+    c, ql, _ = make_workload("tiny")
+    ox = oracle.OracleIndex(c, block_size=B)
+    gx = g.GriffinIndex(c, block_size=B)
+    rng = np.random.default_rng(B)
+    terms = list(range(0, 12)) + rng.integers(0, c.num_terms, 40).tolist()
+    for t in terms:
+        nb = ox.num_blocks(t)
+        for blk in range(nb):
+            o = ox.block_streams(t, blk)
+            gg = gx.griffin_debug_block_streams(t, blk)
+            assert o[0] == gg[0] and o[1] == gg[1] and o[2] == gg[2]
+            assert o[4] == gg[4] and np.array_equal(o[3], gg[3])
+            assert o[6] == gg[6] and np.array_equal(o[5], gg[5])
+
+
+@pytest.mark.parametrize("B", [64, 96, 128, 256, 512])
+def test_decode_list_roundtrip(B):
+    c, ql, _ = make_workload("tiny")
+    gx = g.GriffinIndex(c, block_size=B)
+    for t in range(c.num_terms):
+        assert np.array_equal(gx.griffin_debug_decode_list(t), c.list(t)), t
+
+
+def test_decode_edge_lists():
+    N = 5_000_000
+    lists = [np.array([0]), np.array([N - 1]), np.array([0, N - 1]), np.arange(1000, 1000 + 777),
+             np.arange(0, N, 4999), np.array([3, 4, 5, 1 << 20, (1 << 20) + 1])]
+    c = corpus_from_lists(N, lists, doc_lengths=np.full(N, 7, np.uint32))
+    for B in (64, 512):
+        gx = g.GriffinIndex(c, block_size=B)
+        for t in range(len(lists)):
+            assert np.array_equal(gx.griffin_debug_decode_list(t), c.list(t))
+
+
+def test_decode_all_checksum(tiny, tiny_gpu):
+    c = tiny[0]
+    r = tiny_gpu.griffin_debug_decode_all(iters=2)
+    assert r["postings"] == c.num_postings
+    assert r["checksum"] == int(np.bitwise_xor.reduce(c.docids.astype(np.uint64)))
+
+
+# ---------------------------------------------------------------- intersection
+
+@pytest.mark.parametrize("mode", [g.MODE_AUTO, g.MODE_MERGE, g.MODE_GALLOP])
+def test_intersect_sets_match_oracle(tiny, tiny_gpu, mode):
+    c, ql, ox = tiny
+    for q in range(ql.num_queries):
+        terms = ql.query(q)
+        want = ox.intersect(terms)
+        got = tiny_gpu.griffin_debug_intersect(terms, mode)
+        assert np.array_equal(got, want), (q, terms, len(got), len(want))
+
+
+@pytest.mark.parametrize("mode", [g.MODE_MERGE, g.MODE_GALLOP])
+def test_intersect_random_small_corpora(mode):
+    rng = np.random.default_rng(11 + mode)
+    for trial in range(6):
+        c = random_corpus(rng, num_docs=int(rng.integers(500, 60_000)), num_terms=8, max_df=20_000)
+        ox = oracle.OracleIndex(c, block_size=128)
+        gx = g.GriffinIndex(c, block_size=int(rng.choice([64, 128, 256])))
+        for _ in range(12):
+            terms = rng.integers(0, c.num_terms, size=int(rng.integers(1, 6)))
+            assert np.array_equal(gx.griffin_debug_intersect(terms, mode), ox.intersect(terms))
+
+
+def test_ratio_pairs_all_modes_agree():
+    """Skewed pairs (G6): merge, gallop and auto give the oracle's set."""
+    c, ql = make_pair_workload(3_000_000, 200_000, [1, 3, 16, 100, 300, 1000, 5000], seed=77)
+    ox = oracle.OracleIndex(c)
+    gx = g.GriffinIndex(c)
+    for q in range(ql.num_queries):
+        want = ox.intersect(ql.query(q))
+        for mode in (g.MODE_AUTO, g.MODE_MERGE, g.MODE_GALLOP):
+            assert np.array_equal(gx.griffin_debug_intersect(ql.query(q), mode), want)
+
+
+# ---------------------------------------------------------------- end to end
+
+@pytest.mark.parametrize("k", [1, 10, 1000])
+def test_query_batch_bit_exact(tiny, tiny_gpu, k):
+    c, ql, ox = tiny
+    od, os_, oc = ox.query_batch(ql, k)
+    gd, gs, gc = tiny_gpu.griffin_query_batch(ql.offsets, ql.terms, k)
+    assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+@pytest.mark.parametrize("mode", [g.MODE_MERGE, g.MODE_GALLOP])
+def test_query_batch_forced_modes(tiny, mode):
+    c, ql, ox = tiny
+    gx = g.GriffinIndex(c, block_size=128)
+    gx.griffin_set_mode(mode)
+    od, os_, oc = ox.query_batch(ql, 10)
+    gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 10)
+    assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+def test_c1_single_query():
+    c, ql, cfg = make_workload("c1")
+    ox = oracle.OracleIndex(c, block_size=128)
+    gx = g.GriffinIndex(c, block_size=128)
+    od, os_, oc = ox.query(ql.query(0), 10)
+    gd, gs, gc = gx.griffin_query(ql.query(0), 10)
+    assert oc > 0
+    assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+def test_large_result_radix_select_path():
+    """> 4096 survivors per query exercises the radix-select top-k."""
+    rng = np.random.default_rng(21)
+    N = 200_000
+    lists = [np.sort(rng.choice(N, size=n, replace=False)) for n in (120_000, 150_000, 90_000, 5)]
+    tfs = [rng.integers(1, 30, size=len(l)) for l in lists]
+    c = corpus_from_lists(N, lists, tfs, rng.integers(1, 3000, size=N))
+    ox = oracle.OracleIndex(c)
+    gx = g.GriffinIndex(c)
+    qs = [[0, 1], [0, 1, 2], [2], [0], [3, 0]]
+    ql = QueryLog(offsets=np.cumsum([0] + [len(q) for q in qs]).astype(np.uint32),
+                  terms=np.concatenate(qs).astype(np.uint32))
+    for k in (10, 4096):
+        od, os_, oc = ox.query_batch(ql, k)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+def test_edge_queries():
+    c = corpus_from_lists(1000, [[1, 2, 3, 999], [], [2, 3, 4, 999], [0]],
+                          [[1, 2, 3, 4], [], [5, 6, 7, 8], [9]], np.arange(1, 1001))
+    ox = oracle.OracleIndex(c)
+    gx = g.GriffinIndex(c)
+    for terms in ([0, 0, 2], [2, 0], [0, 1], [1], [3], [3, 0], [0]):
+        od, os_, oc = ox.query(terms, 5)
+        gd, gs, gc = gx.griffin_query(terms, 5)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+    for bad in ([7], []):
+        with pytest.raises(g.GriffinError):
+            gx.griffin_query(bad, 5)
+    with pytest.raises(g.GriffinError):
+        gx.griffin_query([0], 4097)
+
+
+def test_random_batches_bit_exact():
+    rng = np.random.default_rng(123)
+    for trial in range(4):
+        c = random_corpus(rng, num_docs=int(rng.integers(1000, 100_000)), num_terms=12,
+                          max_df=40_000)
+        ox = oracle.OracleIndex(c)
+        gx = g.GriffinIndex(c, block_size=int(rng.choice([64, 128, 256, 512])),
+                            gallop_ratio=int(rng.choice([0, 4, 1000])))
+        ql = random_queries(rng, c.num_terms, 50)
+        k = int(rng.choice([5, 100, 2000]))
+        od, os_, oc = ox.query_batch(ql, k)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+def test_device_api_matches_host_api(tiny, tiny_gpu):
+    import torch
+    c, ql, ox = tiny
+    k = 10
+    nq = ql.num_queries
+    tiny_gpu.griffin_reserve(ql.offsets, ql.terms, k)
+    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
+    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
+    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(nq, dtype=torch.int32, device="cuda")
+    dd = torch.zeros(nq * k, dtype=torch.int32, device="cuda")
+    ds = torch.zeros(nq * k, dtype=torch.float32, device="cuda")
+    s = torch.cuda.current_stream()
+    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    tiny_gpu.griffin_query_batch_device(d_off, d_t, mt, k, keys, cnt, s)
+    tiny_gpu.griffin_keys_to_results_device(nq, k, keys, cnt, dd, ds, s)
+    torch.cuda.synchronize()
+    tiny_gpu.griffin_sync_status()
+    od, os_, oc = ox.query_batch(ql, k)
+    gd = dd.cpu().numpy().view(np.uint32).reshape(nq, k)
+    gs = ds.cpu().numpy().reshape(nq, k)
+    assert_topk_equal(gd, gs, cnt.cpu().numpy().view(np.uint32), od, os_, oc)
+
+
+@pytest.mark.parametrize("G", [2, 3, 8])
+def test_docid_sharding_merge_equals_unsharded(tiny, G):
+    """G docID-range shards on one device (same code path as one shard per GPU,
+    minus NCCL): per-shard top-k keys merged by the device k-way merge equal the
+    unsharded oracle bit for bit (SURVEY §8(e) exactness argument)."""
+    import torch
+    c, ql, ox = tiny
+    k = 20
+    nq = ql.num_queries
+    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
+    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
+    keys = torch.zeros(G, nq * k, dtype=torch.int64, device="cuda")
+    cnts = torch.zeros(G, nq, dtype=torch.int32, device="cuda")
+    shards = []
+    for s in range(G):
+        sx = g.GriffinIndex(c, shard_index=s, num_shards=G)
+        sx.griffin_reserve(ql.offsets, ql.terms, k)
+        sx.griffin_query_batch_device(d_off, d_t, mt, k, keys[s], cnts[s],
+                                      torch.cuda.current_stream())
+        shards.append(sx)
+    torch.cuda.synchronize()
+    out_k = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
+    out_c = torch.zeros(nq, dtype=torch.int32, device="cuda")
+    shards[0].griffin_merge_topk_device(G, nq, k, keys, cnts, out_k, out_c)
+    dd = torch.zeros(nq * k, dtype=torch.int32, device="cuda")
+    ds = torch.zeros(nq * k, dtype=torch.float32, device="cuda")
+    shards[0].griffin_keys_to_results_device(nq, k, out_k, out_c, dd, ds)
+    torch.cuda.synchronize()
+    od, os_, oc = ox.query_batch(ql, k)
+    assert_topk_equal(dd.cpu().numpy().view(np.uint32).reshape(nq, k),
+                      ds.cpu().numpy().reshape(nq, k), out_c.cpu().numpy().view(np.uint32),
+                      od, os_, oc)
+
+
+# ---------------------------------------------------------------- full size (bench config)
+
+@pytest.mark.slow
+def test_c2_full_size_sampled():
+    """BASELINE configs[1] at full size, in the launch configuration bench.py
+    times (one batch of all 1000 queries, device API): a sample of queries is
+    checked one by one against the oracle; the rest via invariants."""
+    import torch
+    c, ql, cfg = make_workload("c2")
+    gx = g.GriffinIndex(c, block_size=128)
+    k = cfg["k"]
+    nq = ql.num_queries
+    gx.griffin_reserve(ql.offsets, ql.terms, k)
+    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
+    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
+    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(nq, dtype=torch.int32, device="cuda")
+    gx.griffin_query_batch_device(d_off, d_t, mt, k, keys, cnt, torch.cuda.current_stream())
+    dd = torch.zeros(nq * k, dtype=torch.int32, device="cuda")
+    ds = torch.zeros(nq * k, dtype=torch.float32, device="cuda")
+    gx.griffin_keys_to_results_device(nq, k, keys, cnt, dd, ds)
+    torch.cuda.synchronize()
+    gx.griffin_sync_status()
+    gd = dd.cpu().numpy().view(np.uint32).reshape(nq, k)
+    gs = ds.cpu().numpy().reshape(nq, k)
+    gc = cnt.cpu().numpy().view(np.uint32)
+    # invariants for every query: sorted by (score desc, docID asc); every docID
+    # is in all of the query's lists
+    for q in range(nq):
+        n = gc[q]
+        for i in range(1, n):
+            assert gs[q, i] < gs[q, i - 1] or (gs[q, i] == gs[q, i - 1] and gd[q, i] > gd[q, i - 1])
+        for t in set(ql.query(q).tolist()):
+            lst = c.list(t)
+            pos = np.searchsorted(lst, gd[q, :n])
+            assert np.all(lst[np.minimum(pos, len(lst) - 1)] == gd[q, :n])
+    ox = oracle.OracleIndex(c, block_size=128)
+    sample = np.random.default_rng(0).choice(nq, size=25, replace=False)
+    for q in sample:
+        od, os_, oc = ox.query(ql.query(q), k)
+        assert_topk_equal(gd[q], gs[q], gc[q], od, os_, oc)
