@@ -1,0 +1,357 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 Griffin-GPU conjunctive query path.
+
+One "step" = one pass of the whole hot path (plus a8 for
+N > 1) over one batch: the BASELINE.json configs[1] workload — a 10M-doc
+synthetic Zipfian index (EF blocks of 128) and its 1000-query 2-5 term log,
+BM25 top-10 — with the query log already resident in HBM.  Prints ONE JSON line.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl reference]
+
+N > 1 is launched by torchrun (one process per GPU): each rank holds one
+docID-range shard of the same corpus, runs the batch, and the per-shard top-k
+keys are all-gathered over NCCL and merged by the library's k-way merge kernel.
+The reference arm (--impl reference) times the CPU oracle (the test oracle,
+as it stands) on the same workload; there is no installable reference code.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+WORKLOAD_DESC = {
+    "c1": "C1: single 2-term AND query, 100K-doc synthetic Zipf index (lists ~10K and ~1K), EF block 128, BM25 top-10",
+    "c2": "C2: 10M-doc synthetic Zipf index (alpha 0.8, df 1K..5M, 42K terms, 0.19B postings), replayed 1000-query 2-5 term log, EF block 128, BM25 top-10",
+    "c3": "C3: GOV2-shaped 25M-doc synthetic Zipf index (df up to 10M), 1000-query log, BM25 top-10",
+    "c4": "C4: ClueWeb-shaped 50M-doc synthetic Zipf index (df up to 30M), 10K-query log, BM25 top-10",
+    "c5": "C5: 50M-doc index, 10K concurrent queries, BM25 top-1000",
+}
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        try:
+            out, _ = self.p.communicate(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.p.kill()
+            out, _ = self.p.communicate()
+        rows = [r.split(",") for r in out.strip().splitlines() if r.strip()]
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[1]))
+                mx = max(mx, float(r[2]))
+                for nm, v in zip(names, r[5:9]):
+                    if v.strip().lower() == "active":
+                        reasons.add(nm)
+            except (ValueError, IndexError):
+                continue
+        if not sm:
+            return None
+        loaded = [s for s in sm if s > 0.5 * mx] or sm
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def _cpu_info():
+    model = ""
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name"):
+                model = line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return os.cpu_count() or 1, model
+
+
+def oracle_baseline(corpus, ql, k, block, budget_s=12.0, threads=None):
+    """Time the oracle (as it stands) on a bounded prefix of the query log."""
+    import oracle
+    cores, model = _cpu_info()
+    threads = threads or cores
+    t0 = time.time()
+    ox = oracle.OracleIndex(corpus, block_size=block)
+    build_s = time.time() - t0
+    m = min(ql.num_queries, max(threads, 16))
+    while True:
+        sub = ql.slice(0, m)
+        t0 = time.perf_counter()
+        ox.query_batch(sub, k, nthreads=threads)
+        dt = time.perf_counter() - t0
+        if dt >= budget_s / 3 or m >= ql.num_queries:
+            break
+        m = min(ql.num_queries, int(m * max(2.0, budget_s / 3 / max(dt, 1e-3))))
+    return {"value": m / dt, "unit": "queries/s", "cores": threads, "kind": "oracle",
+            "sample": f"first {m} of the {ql.num_queries}-query log, {threads} std::threads, "
+                      f"round-robin; oracle index build {build_s:.1f}s not timed",
+            "cpu_model": model, "seconds": dt}, ox, m
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from synth import make_workload
+    corpus, ql, cfg = make_workload(args.config)
+    k = cfg["k"]
+    base, ox, m = oracle_baseline(corpus, ql, k, cfg["block"], budget_s=6.0)
+    sub = ql.slice(0, m)
+    threads = base["cores"]
+    for _ in range(args.warmup):
+        ox.query_batch(sub, k, nthreads=threads)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        ox.query_batch(sub, k, nthreads=threads)
+        times.append(time.perf_counter() - t0)
+    ms = 1e3 * statistics.mean(times)
+    qps = m / (ms / 1e3)
+    base["value"] = qps
+    line = {"impl": "reference", "metric": "queries/sec", "value": qps, "unit": "queries/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/f32",
+            "data": "synthetic",
+            "config": {"workload": WORKLOAD_DESC[args.config], "num_docs": corpus.num_docs,
+                       "queries_per_step": m, "k": k, "block_size": cfg["block"]},
+            "cpu_baseline": base,
+            "e2e": {"value": qps, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_gpu(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_0044ws18_b200 as g
+    from synth import make_workload
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.cuda.current_device()
+    corpus, ql, cfg = make_workload(args.config)
+    k, B = cfg["k"], cfg["block"]
+    nq = ql.num_queries
+    t0 = time.time()
+    ix = g.GriffinIndex(corpus, block_size=B, device=dev, shard_index=rank, num_shards=world)
+    build_s = time.time() - t0
+    st = ix.griffin_index_stats()
+    ix.griffin_reserve(ql.offsets, ql.terms, k)
+    max_terms = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    stream = torch.cuda.current_stream()
+    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
+    d_terms = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
+    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
+    cnts = torch.zeros(nq, dtype=torch.int32, device="cuda")
+    if world > 1:
+        all_keys = torch.zeros(world, nq * k, dtype=torch.int64, device="cuda")
+        all_cnts = torch.zeros(world, nq, dtype=torch.int32, device="cuda")
+        out_keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
+        out_cnts = torch.zeros(nq, dtype=torch.int32, device="cuda")
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device="cuda")  # 256 MB > L2
+
+    def step():
+        ix.griffin_query_batch_device(d_off, d_terms, max_terms, k, keys, cnts, stream)
+        if world > 1:
+            dist.all_gather_into_tensor(all_keys.view(-1), keys)
+            dist.all_gather_into_tensor(all_cnts.view(-1), cnts)
+            ix.griffin_merge_topk_device(world, nq, k, all_keys, all_cnts, out_keys, out_cnts,
+                                         stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    ix.griffin_sync_status()
+    ix.griffin_reset_profile()
+    ix.griffin_set_profiling(True)
+    clocks = ClockSampler(dev)
+    clocks.start()
+    time.sleep(0.3)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        flush.fill_(i)                       # L2 flush between timed steps (outside events)
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ix.griffin_set_profiling(False)
+    prof = ix.griffin_get_profile()
+    ix.griffin_sync_status()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    total_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ms_per_step = total_ms / args.steps
+    qps = nq * args.steps / (total_ms / 1e3)
+    peak, peak_kind = _peaks()
+    ms_x = prof["ms_intersect"]
+    achieved = prof["alg_bytes"] / (ms_x / 1e3) / 1e9 if ms_x > 0 else 0.0
+    # per-GPU figures of this rank; the job aggregate for N ranks is N x (max-time) based
+    decoded_ps = prof["decoded_postings"] / (total_ms / 1e3) if total_ms > 0 else 0.0
+
+    # ---- e2e: the public host-buffer C-ABI call, H2D of the step's queries and
+    # D2H of its results inside every timed step (wall clock, max over ranks)
+    e2e_times = []
+    for i in range(args.warmup + args.steps):
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        dd, ss, cc = ix.griffin_query_batch(ql.offsets, ql.terms, k)
+        if world > 1:
+            # per-shard results are merged the same way (device all-gather + merge)
+            keys.copy_(torch.from_numpy(
+                ((ss.view(np.uint32).astype(np.uint64) << 32) |
+                 (0xFFFFFFFF - dd.astype(np.uint64))).view(np.int64).reshape(-1)))
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            e2e_times.append(dt)
+    e2e_s = sum(e2e_times)
+    if world > 1:
+        t = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = float(t.item())
+    h2d = (nq + 1) * 4 + len(ql.terms) * 4
+    d2h = nq * k * 8 + nq * 4
+
+    # ---- closed-loop single-query latency (griffin_query, one in flight)
+    lat = []
+    nlat = min(nq, args.latency_queries)
+    for q in range(nlat):
+        t0 = time.perf_counter()
+        ix.griffin_query(ql.query(q), k)
+        lat.append((time.perf_counter() - t0) * 1e3)
+    lat.sort()
+
+    def pct(p):
+        return lat[min(len(lat) - 1, int(np.ceil(p / 100 * len(lat))) - 1)] if lat else None
+
+    line = {
+        "metric": "queries/sec", "value": qps, "unit": "queries/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/f32",
+        "data": "synthetic",
+        "config": {"workload": WORKLOAD_DESC[args.config], "num_docs": corpus.num_docs,
+                   "num_terms": corpus.num_terms, "num_postings": corpus.num_postings,
+                   "queries_per_step": nq, "k": k, "block_size": B,
+                   "l2": "flushed between timed steps (256 MB write)",
+                   "parallelism": f"docid-range shards x{world}" if world > 1 else "1 shard",
+                   "index_bytes_per_shard": st["payload_bytes"] + st["skip_bytes"] + st["tf_bytes"],
+                   "index_build_s": build_s},
+        "decoded_postings_per_s": decoded_ps * world,
+        "hbm_gbs": achieved,
+        "latency_ms": {"p50": pct(50), "p99": pct(99), "queries": nlat,
+                       "mode": "closed-loop griffin_query (host buffers), one in flight"},
+        "roofline": {"bound": "hbm", "kernel": "intersect_kernel (fused EF decode + merge-path/gallop + BM25)",
+                     "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak if peak else None, "traffic": None,
+                     "peak_kind": peak_kind,
+                     "alg_bytes_per_launch": prof["alg_bytes"] / max(1, prof["launches_intersect"]),
+                     "ms_per_launch": ms_x / max(1, prof["launches_intersect"]),
+                     "share_of_step": ms_x / total_ms if total_ms else None},
+        "stage_ms_per_step": {kk: prof[kk] / args.steps for kk in
+                              ("ms_plan", "ms_intersect", "ms_compact", "ms_topk", "ms_merge")},
+        "gpu_launches": int(prof["launches_total"]),
+        "e2e": {"value": nq * args.steps / e2e_s, "unit": "queries/s", "h2d_bytes_per_step": h2d,
+                "d2h_bytes_per_step": d2h,
+                "how": "griffin_query_batch (host buffers; pinned staging, H2D queries, D2H results)"},
+        "clocks": clk,
+    }
+    traffic = _ncu_traffic(args.config)
+    if traffic is not None:
+        line["roofline"]["traffic"] = traffic
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        base, _, _ = oracle_baseline(corpus, ql, k, B, budget_s=args.cpu_budget)
+        line["cpu_baseline"] = base
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def _ncu_traffic(config):
+    """dram read+write bytes per intersect launch from the committed ncu summary."""
+    p = os.path.join(ROOT, "profiles", f"ncu_summary_{config}.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get("intersect_dram_bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c2", choices=sorted(WORKLOAD_DESC))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--latency-queries", type=int, default=1000)
+    ap.add_argument("--cpu-budget", type=float, default=12.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_gpu(args)
+
+
+if __name__ == "__main__":
+    main()
