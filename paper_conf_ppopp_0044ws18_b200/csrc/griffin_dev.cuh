@@ -84,55 +84,132 @@ __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v) {
   return v;
 }
 
+// ---- shared memory / async-proxy primitives (sm_90+; TMA bulk copies) -----------
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+// order this thread's earlier generic-proxy smem accesses before later async-proxy writes
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+// 1-D TMA bulk copy global -> shared (16-B aligned, size multiple of 16)
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+          "r"(smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(phase)
+      : "memory");
+}
+
+// ---- select-in-word (the shared-memory look-up table of) --------------
+// lut[v*8 + r] = bit position of the r-th one of byte v.  Built once per CTA.
+__device__ __forceinline__ void build_select_lut(uint8_t *lut) {
+  for (uint32_t v = threadIdx.x; v < 256; v += blockDim.x) {
+    uint32_t r = 0;
+    for (uint32_t bit = 0; bit < 8; ++bit)
+      if ((v >> bit) & 1u) lut[v * 8 + r++] = (uint8_t)bit;
+    for (; r < 8; ++r) lut[v * 8 + r] = 0;
+  }
+}
+// position of the r-th (0-based) one of x; requires r < popc(x)
+__device__ __forceinline__ uint32_t select_in_word(uint32_t x, uint32_t r, const uint8_t *lut) {
+  const uint32_t c1 = __popc(x & 0xFFu), c2 = __popc(x & 0xFFFFu), c3 = __popc(x & 0xFFFFFFu);
+  uint32_t sh = 0, base = 0;
+  if (r >= c1) { sh = 8; base = c1; }
+  if (r >= c2) { sh = 16; base = c2; }
+  if (r >= c3) { sh = 24; base = c3; }
+  return sh + lut[((x >> sh) & 0xFFu) * 8u + (r - base)];
+}
+
 // ---- Elias-Fano block decode (Para-EF, §3.1.1 / Alg. 1) -------------
-// One warp decodes one block of n <= B postings into dst[0..n) (shared memory),
-// as absolute local docIDs x_i = first + ((h_i << b) | low_i).
-//  * scheduling phase (Alg. 1 l.2-8): the high stream is consumed one 32-bit
-//    word per warp step; lane l owns bit l of the word, its rank among the word's
-//    ones is popc(word & lanemask_lt) and the running count of ones before the
-//    word is the warp-uniform prefix `base` (the prefix sum of l.3).  A lane whose
-//    bit is set is element k = base + rank and writes its high part h_k = p - k
-//    (the number of zeros before the k-th one).
-//  * decompress phase (l.9-10): lane-strided elements funnel-shift their b low
-//    bits out of the staged low stream and OR them in.
-// `scratch` is per-warp shared memory of >= payload words + 4 u32, 16-B aligned.
-__device__ __forceinline__ uint32_t warp_decode_block(const DevIndex &ix, uint64_t blk,
-                                                      uint32_t *__restrict__ dst,
-                                                      uint32_t *__restrict__ scratch,
-                                                      uint32_t *payload_bytes = nullptr) {
+// One warp decodes one block of n <= B postings, already staged in shared memory
+// (low stream: lw words, then high stream: hw words), into dst[0..n) as absolute
+// local docIDs x_k = first + ((h_k << b) | low_k).
+//  * Alg. 1 l.2-3: lane w popcounts high word w; a warp shuffle scan gives the
+//    inclusive prefix counts (the "synchronization point").
+//  * Alg. 1 l.4-8 (scheduling): instead of scattering word ids element by
+//    element, lane l owns the E = ceil(n/32) consecutive elements k0 = l*E ...;
+//    it binary-searches the prefix counts for the word holding element k0 and
+//    selects the bit with the byte LUT.
+//  * Alg. 1 l.9-10: the following E-1 ones are the next set bits (clear-lowest +
+//    find-first-set); h_k = p_k - k (the zeros before the k-th one);
+//    the b low bits are funnel-shifted out of the staged low stream.
+// `cnt` is per-warp smem scratch of >= 64 u32.
+__device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ stg, uint32_t first,
+                                                   uint32_t y, uint32_t *__restrict__ dst,
+                                                   uint32_t *__restrict__ cnt,
+                                                   const uint8_t *__restrict__ lut) {
   const uint32_t lane = lane_id();
-  const uint2 m = ix.meta[blk];
-  const uint32_t first = ix.first[blk];
-  const uint32_t b = meta_b(m.y), n = meta_n(m.y), hw = meta_hw(m.y);
+  const uint32_t b = meta_b(y), n = meta_n(y), hw = meta_hw(y);
   const uint32_t lw = low_words(n, b);
-  const uint32_t n16 = (lw + hw + 3u) >> 2;
-  const uint4 *src = ix.payload + m.x;
-  uint4 *s4 = reinterpret_cast<uint4 *>(scratch);
-  for (uint32_t i = lane; i < n16; i += 32) s4[i] = ldg_nc_v4(src + i);
-  if (lane == 0) s4[n16] = make_uint4(0, 0, 0, 0);
-  __syncwarp();
-  // scheduling phase: scatter high parts
-  const uint32_t *hs = scratch + lw;
-  const uint32_t lt = lanemask_lt();
-  uint32_t base = 0;
-  for (uint32_t w = 0; base < n; ++w) {
-    const uint32_t word = hs[w];
-    const uint32_t k = base + __popc(word & lt);
-    if ((word >> lane) & 1u) dst[k] = (w << 5) + lane - k;
-    base += __popc(word);
+  const uint32_t *hs = stg + lw;
+  const uint32_t w0 = lane < hw ? hs[lane] : 0u;
+  const uint32_t i0 = warp_incl_scan(__popc(w0));
+  cnt[lane] = i0;
+  if (hw > 32) {
+    const uint32_t w1 = lane + 32 < hw ? hs[lane + 32] : 0u;
+    cnt[lane + 32] = __shfl_sync(0xffffffffu, i0, 31) + warp_incl_scan(__popc(w1));
   }
   __syncwarp();
-  // decompress phase: low bits
-  const uint32_t mask = b ? (0xFFFFFFFFu >> (32u - b)) : 0u;
-  for (uint32_t e = lane; e < n; e += 32) {
-    const uint32_t bit = e * b;
-    const uint32_t wi = bit >> 5;
-    const uint32_t lo = __funnelshift_r(scratch[wi], scratch[wi + 1], bit & 31u) & mask;
-    dst[e] = first + ((dst[e] << b) | lo);
+  const uint32_t E = (n + 31u) >> 5;
+  const uint32_t k0 = lane * E;
+  if (k0 < n) {
+    const uint32_t ne = min(E, n - k0);
+    // word holding element k0: smallest w with cnt[w] > k0
+    uint32_t lo = 0, hi = hw - 1;
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (cnt[mid] > k0) hi = mid; else lo = mid + 1;
+    }
+    uint32_t w = lo;
+    uint32_t cur = hs[w];
+    const uint32_t pos = select_in_word(cur, k0 - (w ? cnt[w - 1] : 0u), lut);
+    cur &= 0xFFFFFFFEu << pos;  // ones after element k0 in this word
+    uint32_t p = (w << 5) + pos;
+    const uint32_t mask = b ? (0xFFFFFFFFu >> (32u - b)) : 0u;
+    uint32_t bp = k0 * b;
+    for (uint32_t j = 0; j < ne; ++j) {
+      if (j) {
+        while (cur == 0u) cur = hs[++w];
+        p = (w << 5) + (__ffs(cur) - 1u);
+        cur &= cur - 1u;
+      }
+      const uint32_t h = p - (k0 + j);
+      const uint32_t wi = bp >> 5;
+      const uint32_t lo_bits = __funnelshift_r(stg[wi], stg[wi + 1], bp) & mask;
+      dst[k0 + j] = first + ((h << b) | lo_bits);
+      bp += b;
+    }
   }
   __syncwarp();
-  if (payload_bytes) *payload_bytes = n16 * 16u;
-  return n;
+}
+
+// payload size of a block in 16-B units
+__host__ __device__ inline uint32_t block_size16(uint32_t y) {
+  return (low_words(meta_n(y), meta_b(y)) + meta_hw(y) + 3u) >> 2;
+}
+// staging words per block (upper bound for any b <= 31, plus read slack)
+__host__ __device__ inline uint32_t stage_words_per_block(uint32_t B) {
+  return ((B * 34u) / 32u + 8u + 3u) & ~3u;
 }
 
 // ---- tf and BM25 ---------------------------------------------------------------

@@ -54,8 +54,8 @@ struct DevBuf {
 // Query workspace (all grow-only; sized by griffin_reserve / the host API).
 struct Workspace {
   DevBuf plan_terms, plan_m, cap, cap_off, rcount, rsel, qmode, unit_base;  // per query
-  DevBuf unit_off, unit_cnt;                                                // per unit
-  DevBuf rbuf0, rbuf1, bump;                                                // per survivor
+  DevBuf unit_off, unit_cnt, unit_dst;                                      // per unit
+  DevBuf rbuf0, rbuf1, bump, cand;                                          // per survivor
   DevBuf scal;       // scalars: counters, status, bump ctr, unit ctr
   DevBuf keys, counts, docids, scores, qoffs, qterms;  // host-API staging on device
   size_t nq_cap = 0, unit_cap = 0, entry_cap = 0;

@@ -169,33 +169,83 @@ struct Acc {
   unsigned long long alg = 0, pay = 0, post = 0, surv = 0;
 };
 
-struct WarpSmem {
-  uint32_t *scratch;  // EF payload staging (16-B aligned)
-  uint32_t *tile;     // decoded values, (D+2)*B
-  uint32_t *match;    // per R-tile element: S posting position or kNone, (D+1)*B
-};
-
-__host__ __device__ inline uint32_t scratch_words(uint32_t B) {
-  return ((B * 34u) / 32u + 24u + 3u) & ~3u;
+// Per-warp shared memory carve-up (u32 words):
+//   [mbar 4][cnt 64][aux B+32][stg SW][tile (D+2)*B]
+// stg holds TMA-staged EF payloads; after decoding, the merge path reuses it for
+// the per-R-element match array.  The gallop path carves tile into
+// tileR | kidx | match | tileS[G blocks].
+__host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D) {
+  return (D + 2) * stage_words_per_block(B);
 }
 __host__ __device__ inline uint32_t warp_smem_words(uint32_t B, uint32_t D) {
-  return scratch_words(B) + (((D + 2) * B + (D + 1) * B + 3u) & ~3u);
+  return 4 + 64 + (B + 32) + stage_words(B, D) + (D + 2) * B;
+}
+constexpr uint32_t kLutBytes = 2048;
+
+struct WarpSmem {
+  uint64_t *mbar;
+  uint32_t *cnt, *aux, *stg, *tile;
+  const uint8_t *lut;
+  uint32_t phase;
+};
+
+__device__ __forceinline__ WarpSmem carve_warp_smem(uint4 *smem4, uint32_t B, uint32_t D) {
+  uint8_t *base = reinterpret_cast<uint8_t *>(smem4);
+  WarpSmem w;
+  w.lut = base;
+  uint32_t *wb = reinterpret_cast<uint32_t *>(base + kLutBytes) +
+                 (threadIdx.x >> 5) * warp_smem_words(B, D);
+  w.mbar = reinterpret_cast<uint64_t *>(wb);
+  w.cnt = wb + 4;
+  w.aux = w.cnt + 64;
+  w.stg = w.aux + B + 32;
+  w.tile = w.stg + stage_words(B, D);
+  w.phase = 0;
+  return w;
 }
 
-// Load R "block" k into dst.  Compressed R: EF decode; intermediate R: copy the
-// docIDs of chunk k (B entries).  Returns the element count.
-template <bool RC>
-__device__ __forceinline__ uint32_t load_r_block(const DevIndex &ix, const TermInfo &tR,
-                                                 const uint2 *Rq, uint32_t nR, uint32_t k,
-                                                 uint32_t *dst, uint32_t *scratch,
-                                                 uint32_t *pay = nullptr) {
-  if (RC) return warp_decode_block(ix, (uint64_t)tR.block0 + k, dst, scratch, pay);
+// CTA prologue: LUT + one mbarrier per warp.
+__device__ __forceinline__ void cta_smem_init(uint4 *smem4, const WarpSmem &w) {
+  build_select_lut(reinterpret_cast<uint8_t *>(smem4));
+  if (lane_id() == 0) {
+    mbar_init(w.mbar, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+}
+
+// Stage the payloads of the blocks whose (meta, staging offset in 16-B units)
+// are held by lanes [0, nb) as one or more TMA bulk copies, then wait.
+// `contig` = the blocks are consecutive in the payload (one copy suffices).
+__device__ __forceinline__ void stage_blocks(const DevIndex &ix, WarpSmem &w, uint32_t nb,
+                                             uint2 m, uint32_t soff16, uint32_t sz16,
+                                             bool contig) {
   const uint32_t lane = lane_id();
-  const uint32_t s = k * ix.B;
-  const uint32_t n = min(ix.B, nR - s);
+  const uint32_t tot16 = __reduce_add_sync(0xffffffffu, lane < nb ? sz16 : 0u);
+  if (tot16 == 0) return;
+  const uint32_t m0x = __shfl_sync(0xffffffffu, m.x, 0);
+  if (lane == 0) {
+    fence_proxy_async();
+    mbar_expect_tx(w.mbar, tot16 * 16u);
+  }
+  if (contig) {
+    if (lane == 0) bulk_g2s(w.stg, ix.payload + m0x, tot16 * 16u, w.mbar);
+  } else if (lane < nb && sz16) {
+    fence_proxy_async();
+    bulk_g2s(w.stg + soff16 * 4u, ix.payload + m.x, sz16 * 16u, w.mbar);
+  }
+  mbar_wait(w.mbar, w.phase);
+  w.phase ^= 1u;
+}
+
+// Load R "block" k of an intermediate (chunk of B entries) into dst.
+__device__ __forceinline__ uint32_t load_r_chunk(const uint2 *Rq, uint32_t nR, uint32_t B,
+                                                 uint32_t k, uint32_t *dst) {
+  const uint32_t lane = lane_id();
+  const uint32_t s = k * B;
+  const uint32_t n = min(B, nR - s);
   for (uint32_t i = lane; i < n; i += 32) dst[i] = Rq[s + i].x;
   __syncwarp();
-  if (pay) *pay = n * 8u;
   return n;
 }
 
@@ -258,31 +308,70 @@ __device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, co
   }
 }
 
+// Coarse merge path over the block heads: lanes 0-15 find the crossing of
+// diagonal d0, lanes 16-31 of d1, with a 16-ary search (each step probes 16
+// points of the diagonal and narrows the range to one interval).
+template <class HR, class HS>
+__device__ __forceinline__ void warp_mp_search2(HR hR, uint32_t nbR, HS hS, uint32_t nbS,
+                                                uint32_t d0, uint32_t d1, uint32_t *i0,
+                                                uint32_t *i1) {
+  const uint32_t lane = lane_id(), half = lane >> 4, hl = lane & 15u;
+  const uint32_t d = half ? d1 : d0;
+  // answer: smallest i in [lo, hi] with pred(i) = hR(i) > hS(d-i-1); pred(hi) := true
+  uint32_t lo = d > nbS ? d - nbS : 0u;
+  uint32_t hi = d < nbR ? d : nbR;
+  for (;;) {
+    const bool done = lo >= hi;
+    if (__all_sync(0xffffffffu, done)) break;
+    const uint32_t span = hi - lo;
+    // probes cand(p) = lo + ceil((p+1)*span/16) - 1, p = 0..15; cand(15) = hi-1
+    auto cand = [&](uint32_t p) -> uint32_t {
+      return lo + (uint32_t)(((uint64_t)(p + 1) * span + 15u) / 16u) - 1u;
+    };
+    bool pred = true;
+    if (!done) {
+      const uint32_t c = cand(hl);
+      pred = hR(c) > hS(d - c - 1);
+    }
+    const uint32_t hb = (__ballot_sync(0xffffffffu, pred) >> (half * 16u)) & 0xFFFFu;
+    if (!done) {
+      if (hb == 0) {
+        lo = hi;
+      } else {
+        const uint32_t ps = __ffs(hb) - 1u;
+        const uint32_t nhi = cand(ps);
+        const uint32_t nlo = ps ? cand(ps - 1) + 1u : lo;
+        hi = nhi;
+        lo = nlo;
+      }
+    }
+  }
+  *i0 = __shfl_sync(0xffffffffu, lo, 0);
+  *i1 = __shfl_sync(0xffffffffu, lo, 16);
+}
+
 template <bool RC>
-__global__ void __launch_bounds__(kIntersectThreads) intersect_kernel(DevIndex ix, RoundArgs a) {
+__global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevIndex ix, RoundArgs a) {
   extern __shared__ uint4 smem4[];
-  const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
+  const uint32_t lane = lane_id();
   const uint32_t B = ix.B, D = a.D;
-  uint32_t *wbase = reinterpret_cast<uint32_t *>(smem4) + wid * warp_smem_words(B, D);
-  WarpSmem sm;
-  sm.scratch = wbase;
-  sm.tile = wbase + scratch_words(B);
-  sm.match = sm.tile + (D + 2) * B;
+  WarpSmem sm = carve_warp_smem(smem4, B, D);
+  cta_smem_init(smem4, sm);
   const uint64_t *ubase = a.unit_base;
   const uint64_t total = ubase[a.nq];
+  const uint32_t G = min(D - 1u, 31u);   // gallop: S blocks staged per group
   Acc acc;
   for (;;) {
     unsigned long long u = 0;
     if (lane == 0) u = atomicAdd(a.scal + kScalUnitCtr, 1ull);
     u = __shfl_sync(0xffffffffu, u, 0);
     if (u >= total) break;
-    // query of this unit: last q with ubase[q] <= u
-    uint32_t lo = 0, hi = a.nq;
-    while (hi - lo > 1) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if (ubase[mid] <= u) lo = mid; else hi = mid;
+    uint32_t qlo = 0, qhi = a.nq;
+    while (qhi - qlo > 1) {
+      const uint32_t mid = (qlo + qhi) >> 1;
+      if (ubase[mid] <= u) qlo = mid; else qhi = mid;
     }
-    const uint32_t q = lo;
+    const uint32_t q = qlo;
     const uint32_t lu = (uint32_t)(u - ubase[q]);
     const uint32_t mode = a.qmode[q];
     const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
@@ -292,12 +381,17 @@ __global__ void __launch_bounds__(kIntersectThreads) intersect_kernel(DevIndex i
     const uint32_t nbR = RC ? tR.nblocks : (nR + B - 1) / B;
 
     if (RC && mode == kModeAll) {  // single-term query: the whole list is the result
-      uint32_t pay = 0;
-      const uint32_t n = warp_decode_block(ix, (uint64_t)tR.block0 + lu, sm.tile, sm.scratch, &pay);
+      const uint64_t gb = (uint64_t)tR.block0 + lu;
+      const uint2 m = ix.meta[gb];
+      const uint32_t f = ix.first[gb];
+      const uint32_t sz = block_size16(m.y);
+      stage_blocks(ix, sm, 1, m, 0, sz, true);
+      warp_decode_staged(sm.stg, f, m.y, sm.tile, sm.cnt, sm.lut);
+      const uint32_t n = meta_n(m.y);
       if (lane == 0) {
-        acc.pay += pay;
+        acc.pay += sz * 16u;
         acc.post += n;
-        acc.alg += pay + 8u;
+        acc.alg += sz * 16u + 8u;
       }
       emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, 0, n, lu * B, acc);
       continue;
@@ -307,17 +401,16 @@ __global__ void __launch_bounds__(kIntersectThreads) intersect_kernel(DevIndex i
     const uint32_t nbS = tS.nblocks;
 
     if (mode == kModeMerge) {
-      // ---- coarse merge path over the block heads (no decode) ----
+      // ---- coarse merge path over the block heads (skip pointers, no decode) ----
       auto hR = [&](uint32_t i) -> uint32_t {
         return RC ? __ldg(ix.first + tR.block0 + i) : Rq[i * B].x;
       };
       auto hS = [&](uint32_t j) -> uint32_t { return __ldg(fS + j); };
       const uint32_t tot = nbR + nbS;
       const uint32_t d0 = lu * D, d1 = min(d0 + D, tot);
-      uint32_t si = 0, sj = 0;
-      if (lane < 2) merge_path_split(hR, nbR, hS, nbS, lane ? d1 : d0, false, &si, &sj);
-      const uint32_t i0 = __shfl_sync(0xffffffffu, si, 0), j0 = __shfl_sync(0xffffffffu, sj, 0);
-      const uint32_t i1 = __shfl_sync(0xffffffffu, si, 1), j1 = __shfl_sync(0xffffffffu, sj, 1);
+      uint32_t i0, i1;
+      warp_mp_search2(hR, nbR, hS, nbS, d0, d1, &i0, &i1);
+      const uint32_t j0 = d0 - i0, j1 = d1 - i1;
       const uint64_t INF = 1ull << 32;
       uint64_t lo_v = 0, hi_v = INF;
       if (lane == 0 && d0 > 0)
@@ -328,43 +421,91 @@ __global__ void __launch_bounds__(kIntersectThreads) intersect_kernel(DevIndex i
       hi_v = __shfl_sync(0xffffffffu, hi_v, 1);
       const uint32_t rb0 = i0 ? i0 - 1 : 0, rb1 = i1;
       const uint32_t sb0 = j0 ? j0 - 1 : 0, sb1 = j1;
-      // accounting: blocks whose head lies in this unit
-      if (lane == 0) {
-        for (uint32_t k = i0; k < i1; ++k) {
-          uint32_t pay;
-          if (RC) {
-            const uint2 m = ix.meta[(uint64_t)tR.block0 + k];
-            pay = ((low_words(meta_n(m.y), meta_b(m.y)) + meta_hw(m.y) + 3u) >> 2) * 16u;
-            acc.post += meta_n(m.y);
-            acc.pay += pay;
-            acc.alg += pay + 8u;
-          } else {
-            acc.alg += (unsigned long long)min(B, nR - k * B) * 8u;
-          }
-        }
-        for (uint32_t k = j0; k < j1; ++k) {
-          const uint2 m = ix.meta[(uint64_t)tS.block0 + k];
-          const uint32_t pay = ((low_words(meta_n(m.y), meta_b(m.y)) + meta_hw(m.y) + 3u) >> 2) * 16u;
-          acc.post += meta_n(m.y);
-          acc.pay += pay;
-          acc.alg += pay + 8u;
-        }
-      }
-      if (rb1 <= rb0 || sb1 <= sb0 || lo_v >= hi_v) {
+      const uint32_t nRb = rb1 > rb0 ? rb1 - rb0 : 0, nSb = sb1 > sb0 ? sb1 - sb0 : 0;
+      if (nRb == 0 || nSb == 0 || lo_v >= hi_v) {
         if (lane == 0) {
           a.unit_off[u] = 0;
           a.unit_cnt[u] = 0;
+          // accounting: heads in this unit are still "read" (skip entries only)
         }
         continue;
       }
+      // ---- metas: lanes [0,nRb) R blocks (compressed R), [nRb, nRb+nSb) S blocks ----
+      const bool isR = lane < nRb, isS = lane >= nRb && lane < nRb + nSb;
+      uint2 m = make_uint2(0, 0);
+      uint32_t f = 0;
+      if ((RC && isR) || isS) {
+        const uint64_t gb = isR ? (uint64_t)tR.block0 + rb0 + lane
+                                : (uint64_t)tS.block0 + sb0 + (lane - nRb);
+        m = ix.meta[gb];
+        f = ix.first[gb];
+      }
+      const uint32_t sz = ((RC && isR) || isS) ? block_size16(m.y) : 0u;
+      // staging layout: R range then S range, each as contiguous as in HBM
+      const uint32_t mR0 = __shfl_sync(0xffffffffu, m.x, 0);
+      const uint32_t mS0 = __shfl_sync(0xffffffffu, m.x, nRb);
+      const uint32_t totR16 = __reduce_add_sync(0xffffffffu, (RC && isR) ? sz : 0u);
+      const uint32_t soff = isR ? m.x - mR0 : (isS ? totR16 + (m.x - mS0) : 0u);
+      // accounting: blocks whose head lies in this unit (straddlers belong to the
+      // previous unit)
+      {
+        const bool own = (isR && rb0 + lane >= i0) || (isS && sb0 + (lane - nRb) >= j0);
+        const uint32_t pay = own ? sz * 16u : 0u;
+        const uint32_t nn = (own && ((RC && isR) || isS)) ? meta_n(m.y) : 0u;
+        const uint32_t rbytes = (!RC && isR && own) ? min(B, nR - (rb0 + lane) * B) * 8u : 0u;
+        const uint32_t sp = __reduce_add_sync(0xffffffffu, pay);
+        const uint32_t sn = __reduce_add_sync(0xffffffffu, nn);
+        const uint32_t sr = __reduce_add_sync(0xffffffffu, rbytes);
+        const uint32_t so = __reduce_add_sync(0xffffffffu, (own && ((RC && isR) || isS)) ? 8u : 0u);
+        if (lane == 0) {
+          acc.pay += sp;
+          acc.post += sn;
+          acc.alg += sp + sr + so;
+        }
+      }
+      if (RC) {
+        // two contiguous ranges: issue as per-lane copies of the range heads
+        const uint32_t totS16 = __reduce_add_sync(0xffffffffu, isS ? sz : 0u);
+        if (lane == 0) {
+          fence_proxy_async();
+          mbar_expect_tx(sm.mbar, (totR16 + totS16) * 16u);
+          bulk_g2s(sm.stg, ix.payload + mR0, totR16 * 16u, sm.mbar);
+          bulk_g2s(sm.stg + totR16 * 4u, ix.payload + mS0, totS16 * 16u, sm.mbar);
+        }
+        mbar_wait(sm.mbar, sm.phase);
+        sm.phase ^= 1u;
+      } else {
+        // S only: lanes shifted so the S metas start at lane 0 for stage_blocks
+        const uint2 ms = make_uint2(__shfl_sync(0xffffffffu, m.x, (lane + nRb) & 31),
+                                    __shfl_sync(0xffffffffu, m.y, (lane + nRb) & 31));
+        const uint32_t szs = __shfl_sync(0xffffffffu, sz, (lane + nRb) & 31);
+        stage_blocks(ix, sm, nSb, ms, 0, szs, true);
+      }
       // ---- decode the unit's blocks into the smem tiles ----
-      uint32_t nRt = 0;
-      for (uint32_t k = rb0; k < rb1; ++k)
-        nRt += load_r_block<RC>(ix, tR, Rq, nR, k, sm.tile + nRt, sm.scratch);
-      uint32_t *tileS = sm.tile + nRt;
-      uint32_t nSt = 0;
-      for (uint32_t k = sb0; k < sb1; ++k)
-        nSt += warp_decode_block(ix, (uint64_t)tS.block0 + k, tileS + nSt, sm.scratch);
+      uint32_t nRt;
+      if (RC) {
+        for (uint32_t i = 0; i < nRb; ++i) {
+          const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
+          const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
+          const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
+          warp_decode_staged(sm.stg + so * 4u, fi, y, sm.tile + i * B, sm.cnt, sm.lut);
+        }
+        nRt = (nRb - 1) * B + meta_n(__shfl_sync(0xffffffffu, m.y, nRb - 1));
+      } else {
+        const uint32_t s0 = rb0 * B, s1 = min(rb1 * B, nR);
+        for (uint32_t i = lane; i < s1 - s0; i += 32) sm.tile[i] = Rq[s0 + i].x;
+        nRt = s1 - s0;
+        __syncwarp();
+      }
+      uint32_t *tileS = sm.tile + nRb * B;
+      for (uint32_t i = 0; i < nSb; ++i) {
+        const uint32_t y = __shfl_sync(0xffffffffu, m.y, nRb + i);
+        const uint32_t fi = __shfl_sync(0xffffffffu, f, nRb + i);
+        const uint32_t so = RC ? __shfl_sync(0xffffffffu, soff, nRb + i)
+                               : __shfl_sync(0xffffffffu, m.x, nRb + i) - mS0;
+        warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+      }
+      const uint32_t nSt = (nSb - 1) * B + meta_n(__shfl_sync(0xffffffffu, m.y, nRb + nSb - 1));
       // ranges inside [lo, hi)
       uint32_t r_lo = 0;
       if (lane == 0) r_lo = lower_bound_s(sm.tile, 0, nRt, lo_v);
@@ -373,7 +514,8 @@ __global__ void __launch_bounds__(kIntersectThreads) intersect_kernel(DevIndex i
       if (lane == 3) r_lo = lower_bound_s(tileS, 0, nSt, hi_v);
       const uint32_t ra = __shfl_sync(0xffffffffu, r_lo, 0), rb = __shfl_sync(0xffffffffu, r_lo, 1);
       const uint32_t sa = __shfl_sync(0xffffffffu, r_lo, 2), sb = __shfl_sync(0xffffffffu, r_lo, 3);
-      for (uint32_t i = ra + lane; i < rb; i += 32) sm.match[i] = kNone;
+      uint32_t *match = sm.stg;   // staging is free after decode
+      for (uint32_t i = ra + lane; i < rb; i += 32) match[i] = kNone;
       __syncwarp();
       const uint32_t nr = rb - ra, ns = sb - sa;
       if (nr && ns) {
@@ -390,7 +532,7 @@ __global__ void __launch_bounds__(kIntersectThreads) intersect_kernel(DevIndex i
         while (is < ie && js < je) {
           const uint32_t x = A[is], y = Bv[js];
           if (x == y) {
-            sm.match[ra + is] = posS0 + js;
+            match[ra + is] = posS0 + js;
             ++is;
             ++js;
           } else if (x < y) {
@@ -402,79 +544,115 @@ __global__ void __launch_bounds__(kIntersectThreads) intersect_kernel(DevIndex i
       }
       __syncwarp();
       if (RC)
-        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, sm.match, ra, rb, rb0 * B, acc);
+        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, match, ra, rb, rb0 * B, acc);
       else
-        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, sm.match, ra, rb, rb0 * B, acc);
+        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, match, ra, rb, rb0 * B, acc);
       __syncwarp();
     } else {
-      // ---- gallop: R chunk lu, skip-pointer search into S ----
-      uint32_t *tileR = sm.tile, *tileS = sm.tile + B;
-      int *kidx = reinterpret_cast<int *>(sm.tile + 2 * B);
-      uint32_t payR = 0;
-      const uint32_t n = load_r_block<RC>(ix, tR, Rq, nR, lu, tileR, sm.scratch, &payR);
-      if (lane == 0) {
-        acc.alg += payR + (RC ? 8u : 0u);
-        if (RC) {
-          acc.pay += payR;
+      // ---- gallop: R chunk lu, skip-pointer search into S (Fig. 9) ----
+      uint32_t *tileR = sm.tile, *kidx = sm.tile + B, *match = sm.tile + 2 * B;
+      uint32_t *tileS = sm.tile + 3 * B;
+      uint32_t *dblk = sm.aux, *sn = sm.aux + B;
+      uint32_t n;
+      if (RC) {
+        const uint64_t gb = (uint64_t)tR.block0 + lu;
+        const uint2 m = ix.meta[gb];
+        const uint32_t f = ix.first[gb];
+        const uint32_t sz = block_size16(m.y);
+        stage_blocks(ix, sm, 1, m, 0, sz, true);
+        warp_decode_staged(sm.stg, f, m.y, tileR, sm.cnt, sm.lut);
+        n = meta_n(m.y);
+        if (lane == 0) {
+          acc.pay += sz * 16u;
           acc.post += n;
+          acc.alg += sz * 16u + 8u;
         }
+      } else {
+        n = load_r_chunk(Rq, nR, B, lu, tileR);
+        if (lane == 0) acc.alg += n * 8u;
       }
       uint32_t kk = 0;
       if (lane == 0) kk = upper_bound_g(fS, 0, nbS, tileR[0]);
       if (lane == 1) kk = upper_bound_g(fS, 0, nbS, tileR[n - 1]);
       const uint32_t k_lo = __shfl_sync(0xffffffffu, kk, 0), k_hi = __shfl_sync(0xffffffffu, kk, 1);
       for (uint32_t e = lane; e < n; e += 32) {
-        kidx[e] = (int)upper_bound_g(fS, k_lo, k_hi, tileR[e]) - 1;
-        sm.match[e] = kNone;
+        kidx[e] = upper_bound_g(fS, k_lo, k_hi, tileR[e]) - 1u;   // kNone: below S's first docID
+        match[e] = kNone;
       }
       __syncwarp();
-      const int k_first = kidx[0];
-      // skip R elements below S's first docID (no block)
-      uint32_t e0 = 0;
-      while (e0 < n) {
-        const uint32_t e = e0 + lane;
-        const uint32_t bal = __ballot_sync(0xffffffffu, e < n && kidx[e] < 0);
-        if (bal == 0xffffffffu) {
-          e0 += 32;
-          continue;
-        }
-        e0 += __popc(bal);
-        break;
+      const uint32_t k_first = kidx[0];
+      // distinct touched blocks (kidx is non-decreasing): dblk[], and kidx[e] :=
+      // index of e's block in dblk (kNone if none)
+      uint32_t nd = 0, prev = kNone, e_first = n;
+      for (uint32_t c0 = 0; c0 < n; c0 += 32) {
+        const uint32_t e = c0 + lane;
+        const uint32_t kv = e < n ? kidx[e] : kNone;
+        uint32_t kp = __shfl_up_sync(0xffffffffu, kv, 1);
+        if (lane == 0) kp = prev;
+        const bool newb = e < n && kv != kNone && kv != kp;
+        const uint32_t bal = __ballot_sync(0xffffffffu, newb);
+        const uint32_t rank = __popc(bal & lanemask_lt());
+        if (newb) dblk[nd + rank] = kv;
+        const uint32_t gi = nd + __popc(bal & (lanemask_lt() | (1u << lane))) - 1u;
+        if (e < n) kidx[e] = kv == kNone ? kNone : gi;
+        const uint32_t valid = __ballot_sync(0xffffffffu, e < n && kv != kNone);
+        if (e_first == n && valid) e_first = c0 + __ffs(valid) - 1u;
+        nd += __popc(bal);
+        prev = __shfl_sync(0xffffffffu, kv, 31);
       }
-      while (e0 < n) {
-        const int kb = kidx[e0];
-        uint32_t pay = 0;
-        const uint32_t ns = warp_decode_block(ix, (uint64_t)tS.block0 + kb, tileS, sm.scratch, &pay);
-        if (lane == 0 && !(lu > 0 && kb == k_first)) {
-          acc.pay += pay;
-          acc.post += ns;
-          acc.alg += pay + 8u;
+      __syncwarp();
+      uint32_t ep = e_first;
+      for (uint32_t g0 = 0; g0 < nd; g0 += G) {
+        const uint32_t ng = min(G, nd - g0);
+        uint2 m = make_uint2(0, 0);
+        uint32_t f = 0, sz = 0, blk = 0;
+        if (lane < ng) {
+          blk = dblk[g0 + lane];
+          m = ix.meta[(uint64_t)tS.block0 + blk];
+          f = ix.first[(uint64_t)tS.block0 + blk];
+          sz = block_size16(m.y);
+          sn[lane] = meta_n(m.y);
         }
-        uint32_t e = e0;
+        const uint32_t soff = warp_incl_scan(sz) - sz;
+        {
+          const bool own = lane < ng && !(lu > 0 && blk == k_first);
+          const uint32_t sp = __reduce_add_sync(0xffffffffu, own ? sz * 16u : 0u);
+          const uint32_t spn = __reduce_add_sync(0xffffffffu, own ? meta_n(m.y) : 0u);
+          const uint32_t so = __reduce_add_sync(0xffffffffu, own ? 8u : 0u);
+          if (lane == 0) {
+            acc.pay += sp;
+            acc.post += spn;
+            acc.alg += sp + so;
+          }
+        }
+        stage_blocks(ix, sm, ng, m, soff, sz, false);
+        for (uint32_t i = 0; i < ng; ++i) {
+          const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
+          const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
+          const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
+          warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+        }
+        // elements mapping to this group: contiguous from ep
         for (;;) {
-          const uint32_t ee = e + lane;
-          const bool in = ee < n && kidx[ee] == kb;
+          const uint32_t e = ep + lane;
+          const uint32_t gi = e < n ? kidx[e] : kNone;
+          const bool in = gi != kNone && gi < g0 + ng;
           if (in) {
-            const uint32_t x = tileR[ee];
-            const uint32_t p = lower_bound_s(tileS, 0, ns, x);
-            if (p < ns && tileS[p] == x) sm.match[ee] = (uint32_t)kb * B + p;
+            const uint32_t x = tileR[e];
+            const uint32_t *seg = tileS + (gi - g0) * B;
+            const uint32_t p = lower_bound_s(seg, 0, sn[gi - g0], x);
+            if (p < sn[gi - g0] && seg[p] == x) match[e] = dblk[gi] * B + p;
           }
           const uint32_t bal = __ballot_sync(0xffffffffu, in);
-          if (bal == 0xffffffffu) {
-            e += 32;
-            continue;
-          }
-          e += __popc(bal);
-          break;
+          ep += __popc(bal);
+          if (bal != 0xffffffffu) break;
         }
-        e0 = e;
         __syncwarp();
       }
-      __syncwarp();
       if (RC)
-        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, sm.match, 0, n, lu * B, acc);
+        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
       else
-        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, sm.match, 0, n, lu * B, acc);
+        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
       __syncwarp();
     }
   }
@@ -488,36 +666,80 @@ __global__ void __launch_bounds__(kIntersectThreads) intersect_kernel(DevIndex i
 
 // ------------------------------------------------------------------- compaction
 
-__global__ void compact_kernel(RoundArgs a) {
+// Global exclusive scan of the per-unit survivor counts (n = total units, read
+// on the device; CTAs past n exit).  Units of one query are contiguous, so a
+// query's output offset of unit u is udst[u] - udst[first unit of q].
+__global__ void __launch_bounds__(kScanThreads) unit_scan_sums(const uint32_t *cnt,
+                                                               const uint64_t *n_dev,
+                                                               uint64_t *tsum) {
+  __shared__ uint64_t ws[32];
+  __shared__ uint64_t tot;
+  const uint64_t n = *n_dev;
+  const uint64_t t0 = (uint64_t)blockIdx.x * kScanTile;
+  if (t0 >= n) {
+    if (threadIdx.x == 0) tsum[blockIdx.x] = 0;
+    return;
+  }
+  uint64_t s = 0;
+#pragma unroll
+  for (int i = 0; i < kScanItems; ++i) {
+    const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
+    if (idx < n) s += cnt[idx];
+  }
+  block_excl_scan<uint64_t>(s, ws, &tot);
+  if (threadIdx.x == 0) tsum[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(kScanThreads) unit_scan_apply(const uint32_t *cnt,
+                                                                const uint64_t *n_dev,
+                                                                const uint64_t *toff,
+                                                                uint64_t *out) {
+  __shared__ uint64_t ws[32];
+  __shared__ uint64_t tot;
+  const uint64_t n = *n_dev;
+  const uint64_t t0 = (uint64_t)blockIdx.x * kScanTile;
+  if (t0 >= n) return;
+  uint64_t loc[kScanItems];
+  uint64_t s = 0;
+#pragma unroll
+  for (int i = 0; i < kScanItems; ++i) {
+    const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
+    loc[i] = idx < n ? cnt[idx] : 0;
+    s += loc[i];
+  }
+  uint64_t run = toff[blockIdx.x] + block_excl_scan<uint64_t>(s, ws, &tot);
+#pragma unroll
+  for (int i = 0; i < kScanItems; ++i) {
+    const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
+    if (idx < n) out[idx] = run;
+    run += loc[i];
+  }
+}
+
+// Warp per unit: copy its survivors from the bump area to the query's region of
+// the next intermediate, in unit (= docID) order.  The warp holding a query's
+// last unit publishes the query's new |R|.
+__global__ void __launch_bounds__(256) compact_copy_kernel(RoundArgs a, const uint64_t *udst) {
   const uint32_t lane = lane_id();
-  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
   const uint64_t *ubase = a.unit_base;
-  for (uint32_t q = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); q < a.nq; q += nwarps) {
-    if (a.qmode[q] == kModeNone) {
-      // inactive this round: a query that ran out of terms keeps its result; one
-      // whose plan was empty keeps count 0
-      continue;
+  const uint64_t total = ubase[a.nq];
+  const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
+  for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); u < total;
+       u += nwarps) {
+    uint32_t lo = 0, hi = a.nq;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (ubase[mid] <= u) lo = mid; else hi = mid;
     }
-    const uint64_t u0 = ubase[q], u1 = ubase[q + 1];
-    uint2 *dst = a.rnext + a.cap_off[q];
-    uint32_t run = 0;
-    for (uint64_t c0 = u0; c0 < u1; c0 += 32) {
-      const uint64_t uu = c0 + lane;
-      const uint32_t cnt = uu < u1 ? a.unit_cnt[uu] : 0u;
-      const uint64_t off = uu < u1 ? a.unit_off[uu] : 0ull;
-      const uint32_t incl = warp_incl_scan(cnt);
-      const uint32_t excl = incl - cnt;
-      const uint32_t nu = (uint32_t)((u1 - c0) < 32 ? (u1 - c0) : 32);
-      for (uint32_t j = 0; j < nu; ++j) {
-        const uint32_t cj = __shfl_sync(0xffffffffu, cnt, j);
-        const uint64_t oj = __shfl_sync(0xffffffffu, off, j);
-        const uint32_t ej = __shfl_sync(0xffffffffu, excl, j);
-        for (uint32_t i = lane; i < cj; i += 32) dst[run + ej + i] = a.bump[oj + i];
-      }
-      run += __shfl_sync(0xffffffffu, incl, 31);
-    }
-    if (lane == 0) {
-      a.rcount[q] = run;
+    const uint32_t q = lo;
+    const uint64_t base = udst[ubase[q]];
+    const uint64_t my = udst[u];
+    const uint32_t cnt = a.unit_cnt[u];
+    const uint2 *src = a.bump + a.unit_off[u];
+    uint2 *dst = a.rnext + a.cap_off[q] + (my - base);
+    for (uint32_t i = lane; i < cnt; i += 32) dst[i] = src[i];
+    if (lane == 0 && u + 1 == ubase[q + 1]) {
+      a.rcount[q] = (uint32_t)(my + cnt - base);
       a.rsel[q] = (uint8_t)(a.round & 1u);
     }
   }
@@ -548,75 +770,179 @@ __device__ void bitonic_desc(uint64_t *s, uint32_t n) {
   }
 }
 
-__global__ void __launch_bounds__(kTopkThreads) topk_kernel(DevIndex ix, uint32_t nq, uint32_t k,
-                                                            const uint32_t *rcount,
-                                                            const uint8_t *rsel,
-                                                            const uint64_t *cap_off,
-                                                            const uint2 *rb0, const uint2 *rb1,
-                                                            uint64_t *out_keys,
-                                                            uint32_t *out_counts) {
+struct SelectSmem {
+  uint32_t hist[256];
+  uint64_t prefix;
+  uint32_t need, digit, bcount, cnt;
+};
+
+// Warp 0 finds, scanning the 256 digit bins from the top, the bin holding the
+// need-th largest key; updates prefix/need.  Caller synchronises.
+__device__ __forceinline__ void select_digit(SelectSmem &ss, int shift) {
+  if (threadIdx.x < 32) {
+    const uint32_t lane = threadIdx.x;
+    uint32_t loc[8], s = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {  // lane l owns bins 255-8l .. 248-8l (descending)
+      loc[i] = ss.hist[255 - 8 * lane - i];
+      s += loc[i];
+    }
+    const uint32_t incl = warp_incl_scan(s);
+    const uint32_t need = ss.need;
+    const uint32_t excl = incl - s;
+    if (excl < need && need <= incl) {
+      uint32_t cum = excl;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        if (cum < need && need <= cum + loc[i]) {
+          const uint32_t d = 255 - 8 * lane - i;
+          ss.prefix |= (uint64_t)d << shift;
+          ss.need = need - cum;
+          ss.bcount = loc[i];
+        }
+        cum += loc[i];
+      }
+    }
+  }
+}
+
+// Exact CTA radix select on unique keys: returns thr such that exactly kk of the
+// keys produced by key(i), i < n, are >= thr (8-bit digits, MSB first; stops
+// when the selected bin holds a single key).
+template <class KeyF>
+__device__ uint64_t cta_radix_select(KeyF key, uint32_t n, uint32_t kk, SelectSmem &ss) {
+  if (threadIdx.x == 0) {
+    ss.prefix = 0;
+    ss.need = kk;
+  }
+  uint64_t mask = 0;
+  for (int shift = 56; shift >= 0; shift -= 8) {
+    for (uint32_t i = threadIdx.x; i < 256; i += blockDim.x) ss.hist[i] = 0;
+    __syncthreads();
+    const uint64_t prefix = ss.prefix;
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+      const uint64_t x = key(i);
+      if ((x & mask) == prefix) atomicAdd(&ss.hist[(x >> shift) & 255u], 1u);
+    }
+    __syncthreads();
+    select_digit(ss, shift);
+    __syncthreads();
+    mask |= 0xFFull << shift;
+    if (ss.bcount == 1 && ss.need == 1) {
+      // the single key in the bin is the threshold
+      const uint64_t p = ss.prefix;
+      __syncthreads();
+      for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+        const uint64_t x = key(i);
+        if ((x & mask) == p) ss.prefix = x;
+      }
+      __syncthreads();
+      return ss.prefix;
+    }
+  }
+  return ss.prefix;
+}
+
+// Level 1: every query with more than kTopkSmem survivors is cut into chunks of
+// kTopkSmem; each chunk (one CTA, keys staged in smem) keeps its top min(k, len)
+// keys in cand[(cbase[q] + ci) * k ...] (zero-padded).
+__global__ void __launch_bounds__(kTopkThreads) topk_chunk_kernel(
+    DevIndex ix, uint32_t nq, uint32_t k, const uint32_t *rcount, const uint8_t *rsel,
+    const uint64_t *cap_off, const uint2 *rb0, const uint2 *rb1, const uint64_t *cbase,
+    uint64_t *cand) {
   __shared__ uint64_t sk[kTopkSmem];
-  __shared__ uint32_t hist[256];
-  __shared__ uint64_t s_prefix;
-  __shared__ uint32_t s_need, s_cnt;
+  __shared__ SelectSmem ss;
+  const uint64_t total = cbase[nq];
+  for (uint64_t c = blockIdx.x; c < total; c += gridDim.x) {
+    uint32_t lo = 0, hi = nq;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (cbase[mid] <= c) lo = mid; else hi = mid;
+    }
+    const uint32_t q = lo;
+    const uint32_t ci = (uint32_t)(c - cbase[q]);
+    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q] + (size_t)ci * kTopkSmem;
+    const uint32_t len = min(kTopkSmem, rcount[q] - ci * kTopkSmem);
+    for (uint32_t i = threadIdx.x; i < len; i += blockDim.x) sk[i] = make_key(R[i], ix.doc_base);
+    __syncthreads();
+    uint64_t *out = cand + c * k;
+    const uint32_t kk = min(k, len);
+    if (kk == len) {
+      for (uint32_t i = threadIdx.x; i < k; i += blockDim.x) out[i] = i < len ? sk[i] : 0ull;
+    } else {
+      const uint64_t thr = cta_radix_select([&](uint32_t i) { return sk[i]; }, len, kk, ss);
+      if (threadIdx.x == 0) ss.cnt = 0;
+      __syncthreads();
+      for (uint32_t i = threadIdx.x; i < len; i += blockDim.x)
+        if (sk[i] >= thr) out[atomicAdd(&ss.cnt, 1u)] = sk[i];
+      for (uint32_t i = kk + threadIdx.x; i < k; i += blockDim.x) out[i] = 0ull;
+    }
+    __syncthreads();
+  }
+}
+
+// Level 2, per query: the survivors (<= kTopkSmem) or the level-1 candidates;
+// select the top kk in smem (or by global radix passes when the candidates do
+// not fit), bitonic-sort them, write keys + count.
+__global__ void __launch_bounds__(kTopkThreads) topk_final_kernel(
+    DevIndex ix, uint32_t nq, uint32_t k, const uint32_t *rcount, const uint8_t *rsel,
+    const uint64_t *cap_off, const uint2 *rb0, const uint2 *rb1, const uint64_t *cbase,
+    const uint64_t *cand, uint64_t *out_keys, uint32_t *out_counts) {
+  __shared__ uint64_t sk[kTopkSmem];
+  __shared__ SelectSmem ss;
   for (uint32_t q = blockIdx.x; q < nq; q += gridDim.x) {
     const uint32_t c = rcount[q];
-    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q];
     const uint32_t kk = min(k, c);
-    uint32_t nsort;
-    if (c <= kTopkSmem) {
-      nsort = 1;
-      while (nsort < c) nsort <<= 1;
-      for (uint32_t i = threadIdx.x; i < nsort; i += blockDim.x)
-        sk[i] = i < c ? make_key(R[i], ix.doc_base) : 0ull;
+    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q];
+    const bool big = c > kTopkSmem;
+    const uint64_t *C = cand + cbase[q] * k;
+    const uint32_t n = big ? (uint32_t)((cbase[q + 1] - cbase[q]) * k) : c;
+    auto key = [&](uint32_t i) -> uint64_t { return big ? C[i] : make_key(R[i], ix.doc_base); };
+    uint32_t nsel;
+    if (n <= kTopkSmem) {
+      for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) sk[i] = key(i);
       __syncthreads();
+      if (kk < n) {
+        const uint64_t thr = cta_radix_select([&](uint32_t i) { return sk[i]; }, n, kk, ss);
+        if (threadIdx.x == 0) ss.cnt = 0;
+        __syncthreads();
+        uint64_t mine[kTopkSmem / kTopkThreads];
+        uint32_t nm = 0;
+        for (uint32_t i = threadIdx.x; i < n; i += blockDim.x)
+          if (sk[i] >= thr) mine[nm++] = sk[i];
+        __syncthreads();
+        for (uint32_t j = 0; j < nm; ++j) sk[atomicAdd(&ss.cnt, 1u)] = mine[j];
+        __syncthreads();
+      }
+      nsel = kk;
     } else {
-      // exact radix select of the k-th largest unique key, 8 bits per pass
-      if (threadIdx.x == 0) {
-        s_prefix = 0;
-        s_need = kk;
-        s_cnt = 0;
-      }
-      uint64_t mask = 0;
-      for (int shift = 56; shift >= 0; shift -= 8) {
-        for (uint32_t i = threadIdx.x; i < 256; i += blockDim.x) hist[i] = 0;
-        __syncthreads();
-        const uint64_t prefix = s_prefix;
-        for (uint32_t i = threadIdx.x; i < c; i += blockDim.x) {
-          const uint64_t key = make_key(R[i], ix.doc_base);
-          if ((key & mask) == prefix) atomicAdd(&hist[(key >> shift) & 255u], 1u);
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-          uint32_t cum = 0, need = s_need;
-          for (int d = 255; d >= 0; --d) {
-            if (cum + hist[d] >= need) {
-              s_prefix = prefix | ((uint64_t)d << shift);
-              s_need = need - cum;
-              break;
-            }
-            cum += hist[d];
-          }
-        }
-        mask |= 0xFFull << shift;
-        __syncthreads();
-      }
-      const uint64_t thr = s_prefix;
-      for (uint32_t i = threadIdx.x; i < c; i += blockDim.x) {
-        const uint64_t key = make_key(R[i], ix.doc_base);
-        if (key >= thr) sk[atomicAdd(&s_cnt, 1u)] = key;
+      const uint64_t thr = cta_radix_select(key, n, kk, ss);
+      if (threadIdx.x == 0) ss.cnt = 0;
+      __syncthreads();
+      for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+        const uint64_t x = key(i);
+        if (x >= thr) sk[atomicAdd(&ss.cnt, 1u)] = x;
       }
       __syncthreads();
-      nsort = 1;
-      while (nsort < kk) nsort <<= 1;
-      for (uint32_t i = kk + threadIdx.x; i < nsort; i += blockDim.x) sk[i] = 0ull;
-      __syncthreads();
+      nsel = kk;
     }
+    uint32_t nsort = 1;
+    while (nsort < nsel) nsort <<= 1;
+    for (uint32_t i = nsel + threadIdx.x; i < nsort; i += blockDim.x) sk[i] = 0ull;
+    __syncthreads();
     bitonic_desc(sk, nsort);
     for (uint32_t i = threadIdx.x; i < k; i += blockDim.x)
       out_keys[(size_t)q * k + i] = i < kk ? sk[i] : 0ull;
     if (threadIdx.x == 0) out_counts[q] = kk;
     __syncthreads();
+  }
+}
+
+__global__ void topk_plan_kernel(uint32_t nq, const uint32_t *rcount, uint32_t *nch) {
+  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q < nq) {
+    const uint32_t c = rcount[q];
+    nch[q] = c > kTopkSmem ? (c + kTopkSmem - 1) / kTopkSmem : 0u;
   }
 }
 
@@ -667,34 +993,77 @@ __global__ void keys_to_results_kernel(uint32_t nq, uint32_t k, const uint64_t *
 
 // ------------------------------------------------------------------- debug decode
 
-__global__ void __launch_bounds__(256) decode_list_kernel(DevIndex ix, uint32_t block0,
+// Warp decodes the consecutive blocks [k0, k0+nb) (nb <= D+2) of the shard into
+// w.tile via one TMA bulk copy; returns total postings and payload bytes.
+__device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, uint64_t k0,
+                                               uint32_t nb, uint32_t *pay_bytes) {
+  const uint32_t lane = lane_id();
+  uint2 m = make_uint2(0, 0);
+  uint32_t f = 0, sz = 0;
+  if (lane < nb) {
+    m = ix.meta[k0 + lane];
+    f = ix.first[k0 + lane];
+    sz = block_size16(m.y);
+  }
+  const uint32_t m0 = __shfl_sync(0xffffffffu, m.x, 0);
+  stage_blocks(ix, w, nb, m, 0, sz, true);
+  uint32_t tot = 0;
+  for (uint32_t i = 0; i < nb; ++i) {
+    const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
+    const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
+    const uint32_t so = __shfl_sync(0xffffffffu, m.x, i) - m0;
+    warp_decode_staged(w.stg + so * 4u, fi, y, w.tile + i * ix.B, w.cnt, w.lut);
+    tot += meta_n(y);
+  }
+  *pay_bytes = __reduce_add_sync(0xffffffffu, sz) * 16u;
+  return tot;
+}
+
+__global__ void __launch_bounds__(256) decode_list_kernel(DevIndex ix, uint32_t D, uint32_t block0,
                                                           uint32_t nblocks, uint32_t *out) {
   extern __shared__ uint4 smem4[];
-  const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
-  uint32_t *w = reinterpret_cast<uint32_t *>(smem4) + wid * (scratch_words(ix.B) + ix.B);
+  const uint32_t lane = lane_id();
+  WarpSmem w = carve_warp_smem(smem4, ix.B, D);
+  cta_smem_init(smem4, w);
+  const uint32_t run = D + 2;
+  const uint32_t nruns = (nblocks + run - 1) / run;
   const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
-  for (uint32_t k = blockIdx.x * (blockDim.x >> 5) + wid; k < nblocks; k += nwarps) {
-    const uint32_t n = warp_decode_block(ix, (uint64_t)block0 + k, w + scratch_words(ix.B), w);
-    for (uint32_t i = lane; i < n; i += 32) out[(size_t)k * ix.B + i] = w[scratch_words(ix.B) + i] + ix.doc_base;
+  for (uint32_t r = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); r < nruns; r += nwarps) {
+    const uint32_t k = r * run, nb = min(run, nblocks - k);
+    uint32_t pay;
+    const uint32_t n = decode_run(ix, w, (uint64_t)block0 + k, nb, &pay);
+    for (uint32_t i = lane; i < n; i += 32) out[(size_t)k * ix.B + i] = w.tile[i] + ix.doc_base;
     __syncwarp();
   }
 }
 
-__global__ void __launch_bounds__(256) decode_all_kernel(DevIndex ix, uint64_t nblocks,
+// Decode sweep: every block of the shard once (runs of D+2 blocks per warp).
+__global__ void __launch_bounds__(256) decode_all_kernel(DevIndex ix, uint32_t D, uint64_t nblocks,
                                                          unsigned long long *acc) {
   extern __shared__ uint4 smem4[];
-  const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
-  uint32_t *w = reinterpret_cast<uint32_t *>(smem4) + wid * (scratch_words(ix.B) + ix.B);
+  const uint32_t lane = lane_id();
+  WarpSmem w = carve_warp_smem(smem4, ix.B, D);
+  cta_smem_init(smem4, w);
+  const uint32_t run = D + 2;
+  const uint64_t nruns = (nblocks + run - 1) / run;
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   uint32_t x = 0;
   unsigned long long post = 0, pay = 0;
-  for (uint64_t k = blockIdx.x * (uint64_t)(blockDim.x >> 5) + wid; k < nblocks; k += nwarps) {
-    uint32_t p = 0;
-    const uint32_t n = warp_decode_block(ix, k, w + scratch_words(ix.B), w, &p);
-    for (uint32_t i = lane; i < n; i += 32) x ^= w[scratch_words(ix.B) + i];
+  for (uint64_t r = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); r < nruns;
+       r += nwarps) {
+    const uint64_t k = r * run;
+    const uint32_t nb = (uint32_t)((nblocks - k) < run ? (nblocks - k) : run);
+    uint32_t p;
+    const uint32_t n = decode_run(ix, w, k, nb, &p);
+    // blocks of a run may belong to different terms: only each term's last block
+    // is short, so XOR block by block
+    for (uint32_t bi = 0; bi < nb; ++bi) {
+      const uint32_t nbk = meta_n(ix.meta[k + bi].y);
+      for (uint32_t i = lane; i < nbk; i += 32) x ^= w.tile[bi * ix.B + i];
+    }
     __syncwarp();
     post += n;
-    pay += p + 8u;
+    pay += p + 8u * nb;
   }
   for (int d = 16; d; d >>= 1) x ^= __shfl_xor_sync(0xffffffffu, x, d);
   if (lane == 0) {
@@ -730,6 +1099,7 @@ griffin_status reserve_ws(griffin_index *ix, uint32_t nq, uint64_t units, uint64
   GRIFFIN_CUDA_TRY(w.unit_base.reserve(q * 8 + 8 + (q / kScanTile + 8) * 8));
   GRIFFIN_CUDA_TRY(w.unit_off.reserve((units + 1) * 8));
   GRIFFIN_CUDA_TRY(w.unit_cnt.reserve((units + 1) * 4));
+  GRIFFIN_CUDA_TRY(w.unit_dst.reserve((units + 2) * 8 + (units / kScanTile + 2) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf0.reserve((entries + 1) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf1.reserve((entries + 1) * 8));
   GRIFFIN_CUDA_TRY(w.bump.reserve((entries + 1) * 8));
@@ -737,13 +1107,10 @@ griffin_status reserve_ws(griffin_index *ix, uint32_t nq, uint64_t units, uint64
     GRIFFIN_CUDA_TRY(w.scal.reserve(kScalCount * 8));
     GRIFFIN_CUDA_TRY(cudaMemset(w.scal.p, 0, w.scal.bytes));
   }
+  // every buffer above was reserved for at least these sizes (grow-only)
   w.nq_cap = std::max<size_t>(w.nq_cap, nq);
   w.unit_cap = std::max<size_t>(w.unit_cap, units);
   w.entry_cap = std::max<size_t>(w.entry_cap, entries);
-  // derive the real capacities from the buffers (reserve over-allocates)
-  w.nq_cap = std::min(w.plan_m.bytes / 4 - 1, w.cap_off.bytes / 8 - 2);
-  w.unit_cap = std::min(w.unit_off.bytes / 8 - 1, w.unit_cnt.bytes / 4 - 1);
-  w.entry_cap = std::min(std::min(w.rbuf0.bytes, w.rbuf1.bytes), w.bump.bytes) / 8 - 1;
   return GRIFFIN_OK;
 }
 
@@ -774,7 +1141,7 @@ struct StageTimer {
 
 template <bool RC>
 static cudaError_t launch_intersect(griffin_index *ix, const RoundArgs &ra, cudaStream_t st) {
-  const size_t smem = (size_t)warp_smem_words(ix->B, ix->D) * 4 * kWarpsPerCta;
+  const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * kWarpsPerCta;
   static thread_local int configured_dev[2] = {-1, -1};
   static thread_local size_t configured_smem[2] = {0, 0};
   if (configured_dev[RC] != ix->device || configured_smem[RC] < smem) {
@@ -859,17 +1226,34 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
     }
     {
       StageTimer t(ix, st, 2);
-      compact_kernel<<<std::min<unsigned>((nq + 7) / 8, 148 * 8), 256, 0, st>>>(ra);
+      const uint64_t *n_dev = w.unit_base.as<uint64_t>() + nq;
+      const unsigned tiles = (unsigned)(w.unit_cap / kScanTile + 1);
+      uint64_t *tsum = w.unit_dst.as<uint64_t>() + (w.unit_cap + 2);
+      unit_scan_sums<<<tiles, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum);
+      scan_single_kernel<uint64_t><<<1, kScanThreads, 0, st>>>(tsum, tsum, tiles, nullptr);
+      unit_scan_apply<<<tiles, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum,
+                                                      w.unit_dst.as<uint64_t>());
+      compact_copy_kernel<<<num_sms(ix->device) * 8, 256, 0, st>>>(ra, w.unit_dst.as<uint64_t>());
       GRIFFIN_CUDA_TRY(cudaGetLastError());
+      ix->launch_count += 3;
     }
   }
   if (final_topk) {
     StageTimer t(ix, st, 3);
-    ix->launch_count += 1;
-    topk_kernel<<<std::min<uint32_t>(nq, 148 * 4), kTopkThreads, 0, st>>>(
+    uint32_t *nch = qunits;  // reuse the per-query unit-count scratch
+    uint64_t *cbase = w.unit_base.as<uint64_t>();
+    const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
+    GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8));
+    topk_plan_kernel<<<qblocks, 256, 0, st>>>(nq, w.rcount.as<uint32_t>(), nch);
+    GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(nch, cbase, nq, scan_tmp, st, &ix->launch_count));
+    topk_chunk_kernel<<<num_sms(ix->device) * 4, kTopkThreads, 0, st>>>(
         di, nq, k, w.rcount.as<uint32_t>(), w.rsel.as<uint8_t>(), w.cap_off.as<uint64_t>(),
-        w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), d_keys, d_counts);
+        w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), cbase, w.cand.as<uint64_t>());
+    topk_final_kernel<<<std::min<uint32_t>(nq, 148 * 4), kTopkThreads, 0, st>>>(
+        di, nq, k, w.rcount.as<uint32_t>(), w.rsel.as<uint8_t>(), w.cap_off.as<uint64_t>(),
+        w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), cbase, w.cand.as<uint64_t>(), d_keys, d_counts);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
+    ix->launch_count += 3;
   }
   return GRIFFIN_OK;
 }
@@ -902,24 +1286,26 @@ griffin_status launch_decode_list(griffin_index *ix, uint32_t term, uint32_t *d_
                                   cudaStream_t st) {
   const TermInfo &t = ix->h_terms[term];
   if (!t.nblocks) return GRIFFIN_OK;
-  const size_t smem = (size_t)(scratch_words(ix->B) + ix->B) * 4 * 8;
+  const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * 8;
   GRIFFIN_CUDA_TRY(cudaFuncSetAttribute(decode_list_kernel,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  decode_list_kernel<<<std::min<uint32_t>((t.nblocks + 7) / 8, 148 * 8), 256, smem, st>>>(
-      ix->dev(), t.block0, t.nblocks, d_out);
+  const uint32_t runs = (t.nblocks + ix->D + 1) / (ix->D + 2);
+  decode_list_kernel<<<std::min<uint32_t>((runs + 7) / 8, 148 * 8), 256, smem, st>>>(
+      ix->dev(), ix->D, t.block0, t.nblocks, d_out);
   GRIFFIN_CUDA_TRY(cudaGetLastError());
   return GRIFFIN_OK;
 }
 
 griffin_status launch_decode_all(griffin_index *ix, unsigned long long *d_acc, cudaStream_t st) {
   if (!ix->nblocks) return GRIFFIN_OK;
-  const size_t smem = (size_t)(scratch_words(ix->B) + ix->B) * 4 * 8;
+  const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * 8;
   GRIFFIN_CUDA_TRY(cudaFuncSetAttribute(decode_all_kernel,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, decode_all_kernel, 256, smem);
+  ix->launch_count += 1;
   decode_all_kernel<<<num_sms(ix->device) * std::max(1, per_sm), 256, smem, st>>>(
-      ix->dev(), ix->nblocks, d_acc);
+      ix->dev(), ix->D, ix->nblocks, d_acc);
   GRIFFIN_CUDA_TRY(cudaGetLastError());
   return GRIFFIN_OK;
 }
