@@ -164,6 +164,7 @@ def run_gpu(args):
     import torch.distributed as dist
 
     import paper_conf_ppopp_0044ws18_b200 as g
+    from paper_conf_ppopp_0044ws18_b200.sharded import ShardedSearcher, gather_runs
     from synth import make_workload
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -190,8 +191,6 @@ def run_gpu(args):
     keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
     cnts = torch.zeros(nq, dtype=torch.int32, device="cuda")
     if world > 1:
-        all_keys = torch.zeros(world, nq * k, dtype=torch.int64, device="cuda")
-        all_cnts = torch.zeros(world, nq, dtype=torch.int32, device="cuda")
         out_keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
         out_cnts = torch.zeros(nq, dtype=torch.int32, device="cuda")
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device="cuda")  # 256 MB > L2
@@ -199,10 +198,8 @@ def run_gpu(args):
     def step():
         ix.griffin_query_batch_device(d_off, d_terms, max_terms, k, keys, cnts, stream)
         if world > 1:
-            dist.all_gather_into_tensor(all_keys.view(-1), keys)
-            dist.all_gather_into_tensor(all_cnts.view(-1), cnts)
-            ix.griffin_merge_topk_device(world, nq, k, all_keys, all_cnts, out_keys, out_cnts,
-                                         stream)
+            ak, ac = gather_runs(keys, cnts)
+            ix.griffin_merge_topk_device(world, nq, k, ak, ac, out_keys, out_cnts, stream)
 
     for _ in range(args.warmup):
         step()
@@ -247,16 +244,21 @@ def run_gpu(args):
     # ---- e2e: the public host-buffer C-ABI call, H2D of the step's queries and
     # D2H of its results inside every timed step (wall clock, max over ranks)
     e2e_times = []
+    if world > 1:
+        searcher = ShardedSearcher.from_index(ix)
+        h_off = torch.from_numpy(ql.offsets.astype(np.int32)).pin_memory()
+        h_terms = torch.from_numpy(ql.terms.astype(np.int32)).pin_memory()
     for i in range(args.warmup + args.steps):
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
-        dd, ss, cc = ix.griffin_query_batch(ql.offsets, ql.terms, k)
-        if world > 1:
-            # per-shard results are merged the same way (device all-gather + merge)
-            keys.copy_(torch.from_numpy(
-                ((ss.view(np.uint32).astype(np.uint64) << 32) |
-                 (0xFFFFFFFF - dd.astype(np.uint64))).view(np.int64).reshape(-1)))
+        if world == 1:
+            dd, ss, cc = ix.griffin_query_batch(ql.offsets, ql.terms, k)
+        else:
+            e_off = h_off.to("cuda", non_blocking=True)
+            e_terms = h_terms.to("cuda", non_blocking=True)
+            dd, ss, cc = searcher.search(e_off, e_terms, max_terms, k, stream)
+            dd, ss, cc = dd.cpu(), ss.cpu(), cc.cpu()
         dt = time.perf_counter() - t0
         if i >= args.warmup:
             e2e_times.append(dt)
@@ -311,6 +313,12 @@ def run_gpu(args):
                 "how": "griffin_query_batch (host buffers; pinned staging, H2D queries, D2H results)"},
         "clocks": clk,
     }
+    # decode-only sweep over every block of the shard (SURVEY §8(d) C5 sweep row)
+    sw = ix.griffin_debug_decode_all(iters=3)
+    line["decode_sweep"] = {"ms": sw["ms"], "postings": sw["postings"], "bytes": sw["bytes"],
+                            "gbs": sw["bytes"] / (sw["ms"] / 1e3) / 1e9,
+                            "postings_per_s": sw["postings"] / (sw["ms"] / 1e3),
+                            "frac_of_hbm_peak": sw["bytes"] / (sw["ms"] / 1e3) / 1e9 / peak}
     traffic = _ncu_traffic(args.config)
     if traffic is not None:
         line["roofline"]["traffic"] = traffic

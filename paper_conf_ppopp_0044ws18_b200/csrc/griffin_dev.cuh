@@ -163,41 +163,107 @@ __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ 
   const uint32_t lw = low_words(n, b);
   const uint32_t *hs = stg + lw;
   const uint32_t w0 = lane < hw ? hs[lane] : 0u;
-  const uint32_t i0 = warp_incl_scan(__popc(w0));
-  cnt[lane] = i0;
-  if (hw > 32) {
-    const uint32_t w1 = lane + 32 < hw ? hs[lane + 32] : 0u;
-    cnt[lane + 32] = __shfl_sync(0xffffffffu, i0, 31) + warp_incl_scan(__popc(w1));
-  }
-  __syncwarp();
+  const uint32_t c0 = __popc(w0);
+  const uint32_t i0 = warp_incl_scan(c0);
   const uint32_t E = (n + 31u) >> 5;
   const uint32_t k0 = lane * E;
-  if (k0 < n) {
-    const uint32_t ne = min(E, n - k0);
+  uint32_t w, x, ex, nx;
+  if (hw <= 32 && (E & (E - 1u)) == 0) {
+    // Owner of element k0 without a search: word w holds elements
+    // [excl_w, incl_w), i.e. the targets of lanes [ceil(excl_w/E), ceil(incl_w/E)).
+    // Mark each such range's first lane with w+1, then an inclusive max-scan
+    // hands every lane its owner word.
+    const uint32_t lgE = __ffs(E) - 1u;
+    const uint32_t ex0 = i0 - c0;
+    const uint32_t a = (ex0 + E - 1u) >> lgE, bnd = (i0 + E - 1u) >> lgE;
+    cnt[lane] = 0u;
+    __syncwarp();
+    if (lane < hw && a < bnd && a < 32u) cnt[a] = lane + 1u;
+    __syncwarp();
+    uint32_t v = cnt[lane];
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, v, d);
+      if (lane >= (uint32_t)d) v = max(v, t);
+    }
+    w = v ? v - 1u : 0u;
+    x = __shfl_sync(0xffffffffu, w0, w);
+    ex = __shfl_sync(0xffffffffu, ex0, w);
+    nx = __shfl_sync(0xffffffffu, w0, (w + 1u) & 31u);
+    if (w + 1u >= hw) nx = 0u;
+  } else {
+    cnt[lane] = i0;
+    if (hw > 32) {
+      const uint32_t w1 = lane + 32 < hw ? hs[lane + 32] : 0u;
+      cnt[lane + 32] = __shfl_sync(0xffffffffu, i0, 31) + warp_incl_scan(__popc(w1));
+    }
+    __syncwarp();
     // word holding element k0: smallest w with cnt[w] > k0
     uint32_t lo = 0, hi = hw - 1;
     while (lo < hi) {
       const uint32_t mid = (lo + hi) >> 1;
       if (cnt[mid] > k0) hi = mid; else lo = mid + 1;
     }
-    uint32_t w = lo;
-    uint32_t cur = hs[w];
-    const uint32_t pos = select_in_word(cur, k0 - (w ? cnt[w - 1] : 0u), lut);
-    cur &= 0xFFFFFFFEu << pos;  // ones after element k0 in this word
-    uint32_t p = (w << 5) + pos;
+    w = lo;
+    x = hs[w];
+    ex = w ? cnt[w - 1] : 0u;
+    nx = hs[w + 1];
+  }
+  if (k0 < n) {
+    const uint32_t ne = min(E, n - k0);
+    const uint32_t pos = select_in_word(x, k0 - ex, lut);
+    const uint32_t p0 = (w << 5) + pos;
+    // the 32 bits following element k0's one (clamped funnel: pos+1 may be 32)
+    uint32_t win = __funnelshift_rc(x, nx, pos + 1u);
     const uint32_t mask = b ? (0xFFFFFFFFu >> (32u - b)) : 0u;
-    uint32_t bp = k0 * b;
-    for (uint32_t j = 0; j < ne; ++j) {
-      if (j) {
-        while (cur == 0u) cur = hs[++w];
-        p = (w << 5) + (__ffs(cur) - 1u);
-        cur &= cur - 1u;
+    if (E == 4 && ne == 4 && __popc(win) >= 3u) {
+      // fast path (B = 128): the next three ones are inside the window
+      const uint32_t t1 = __ffs(win);
+      win &= win - 1u;
+      const uint32_t t2 = __ffs(win);
+      win &= win - 1u;
+      const uint32_t t3 = __ffs(win);
+      const uint32_t h0 = p0 - k0, h1 = p0 + t1 - (k0 + 1), h2 = p0 + t2 - (k0 + 2),
+                     h3 = p0 + t3 - (k0 + 3);
+      uint32_t l0, l1, l2, l3;
+      const uint32_t bp = k0 * b;
+      if (b <= 8) {  // all four low fields inside one 32-bit window
+        const uint32_t lw32 = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp);
+        l0 = lw32 & mask;
+        l1 = (lw32 >> b) & mask;
+        l2 = (lw32 >> (2 * b)) & mask;
+        l3 = (lw32 >> (3 * b)) & mask;
+      } else {
+        uint32_t q = bp;
+        l0 = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
+        q += b;
+        l1 = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
+        q += b;
+        l2 = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
+        q += b;
+        l3 = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
       }
-      const uint32_t h = p - (k0 + j);
-      const uint32_t wi = bp >> 5;
-      const uint32_t lo_bits = __funnelshift_r(stg[wi], stg[wi + 1], bp) & mask;
-      dst[k0 + j] = first + ((h << b) | lo_bits);
-      bp += b;
+      *reinterpret_cast<uint4 *>(dst + k0) =
+          make_uint4(first + ((h0 << b) | l0), first + ((h1 << b) | l1),
+                     first + ((h2 << b) | l2), first + ((h3 << b) | l3));
+    } else {
+      // generic path: walk the ones with a 32-bit window, refilling when empty
+      uint32_t wb = p0 + 1u;  // absolute bit position of win's bit 0
+      uint32_t p = p0;
+      uint32_t bp = k0 * b;
+      for (uint32_t j = 0; j < ne; ++j) {
+        if (j) {
+          while (win == 0u) {
+            wb += 32u;
+            win = __funnelshift_r(hs[wb >> 5], hs[(wb >> 5) + 1], wb);
+          }
+          p = wb + (__ffs(win) - 1u);
+          win &= win - 1u;
+        }
+        const uint32_t lo_bits = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp) & mask;
+        dst[k0 + j] = first + (((p - (k0 + j)) << b) | lo_bits);
+        bp += b;
+      }
     }
   }
   __syncwarp();

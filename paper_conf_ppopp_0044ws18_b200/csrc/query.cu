@@ -996,7 +996,8 @@ __global__ void keys_to_results_kernel(uint32_t nq, uint32_t k, const uint64_t *
 // Warp decodes the consecutive blocks [k0, k0+nb) (nb <= D+2) of the shard into
 // w.tile via one TMA bulk copy; returns total postings and payload bytes.
 __device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, uint64_t k0,
-                                               uint32_t nb, uint32_t *pay_bytes) {
+                                               uint32_t nb, uint32_t *pay_bytes,
+                                               uint32_t *my_n = nullptr) {
   const uint32_t lane = lane_id();
   uint2 m = make_uint2(0, 0);
   uint32_t f = 0, sz = 0;
@@ -1016,6 +1017,7 @@ __device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, 
     tot += meta_n(y);
   }
   *pay_bytes = __reduce_add_sync(0xffffffffu, sz) * 16u;
+  if (my_n) *my_n = lane < nb ? meta_n(m.y) : 0u;
   return tot;
 }
 
@@ -1054,11 +1056,12 @@ __global__ void __launch_bounds__(256) decode_all_kernel(DevIndex ix, uint32_t D
     const uint64_t k = r * run;
     const uint32_t nb = (uint32_t)((nblocks - k) < run ? (nblocks - k) : run);
     uint32_t p;
-    const uint32_t n = decode_run(ix, w, k, nb, &p);
+    uint32_t mn;
+    const uint32_t n = decode_run(ix, w, k, nb, &p, &mn);
     // blocks of a run may belong to different terms: only each term's last block
     // is short, so XOR block by block
     for (uint32_t bi = 0; bi < nb; ++bi) {
-      const uint32_t nbk = meta_n(ix.meta[k + bi].y);
+      const uint32_t nbk = __shfl_sync(0xffffffffu, mn, bi);
       for (uint32_t i = lane; i < nbk; i += 32) x ^= w.tile[bi * ix.B + i];
     }
     __syncwarp();
