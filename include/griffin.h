@@ -108,6 +108,12 @@ typedef struct {
   uint64_t payload_bytes;    /* compressed EF bytes of the blocks the method had to read */
   uint64_t decoded_postings; /* postings of those blocks */
   uint64_t survivors;        /* (docID, score) pairs emitted by intersection rounds */
+  /* batch decode-once stage (griffin_set_reuse): EF-decode of hot lists into HBM */
+  double ms_decode;
+  uint64_t launches_decode;
+  uint64_t dec_alg_bytes;    /* compressed bytes + skip entries read, decoded u32 written */
+  uint64_t dec_payload_bytes;
+  uint64_t dec_postings;
 } griffin_profile;
 
 /* ---- index ------------------------------------------------------------------
@@ -170,6 +176,12 @@ griffin_status griffin_keys_to_results_device(griffin_index *ix, uint32_t nq, ui
 /* ---- configuration / instrumentation ---------------------------------------- */
 griffin_status griffin_set_mode(griffin_index *ix, int mode); /* griffin_mode; default AUTO */
 griffin_status griffin_set_profiling(griffin_index *ix, int on);
+/* Batch list reuse: 0 = off (every round decodes its blocks, fused), 1 = on,
+ * 2 = auto (default; on for batches of >= 8 queries).  When on, lists whose
+ * estimated block demand in the batch is >= 1.5x their block count are
+ * EF-decoded once per batch into an HBM arena (the paper's decompress-then-
+ * intersect pipeline, Alg. 1 output `decmp_array`) and intersected from there. */
+griffin_status griffin_set_reuse(griffin_index *ix, int mode);
 griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out); /* syncs */
 griffin_status griffin_reset_profile(griffin_index *ix);
 const char *griffin_last_error(void);

@@ -67,7 +67,9 @@ class Profile(ctypes.Structure):
                 ("ms_merge", ctypes.c_double), ("launches_intersect", ctypes.c_uint64),
                 ("launches_total", ctypes.c_uint64), ("alg_bytes", ctypes.c_uint64),
                 ("payload_bytes", ctypes.c_uint64), ("decoded_postings", ctypes.c_uint64),
-                ("survivors", ctypes.c_uint64)]
+                ("survivors", ctypes.c_uint64), ("ms_decode", ctypes.c_double),
+                ("launches_decode", ctypes.c_uint64), ("dec_alg_bytes", ctypes.c_uint64),
+                ("dec_payload_bytes", ctypes.c_uint64), ("dec_postings", ctypes.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -88,6 +90,7 @@ _SIGS = {
     "griffin_keys_to_results_device": [_vp, _u32, _u32, _vp, _vp, _vp, _vp, _vp],
     "griffin_set_mode": [_vp, ctypes.c_int],
     "griffin_set_profiling": [_vp, ctypes.c_int],
+    "griffin_set_reuse": [_vp, ctypes.c_int],
     "griffin_get_profile": [_vp, ctypes.POINTER(Profile)],
     "griffin_reset_profile": [_vp],
     "griffin_shard_range": [_u32, _u32, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u32)],
@@ -246,6 +249,10 @@ class GriffinIndex:
     # -- configuration / instrumentation
     def griffin_set_mode(self, mode: int):
         _check(load_library().griffin_set_mode(self.h, mode))
+
+    def griffin_set_reuse(self, mode: int):
+        """0 off (fused decode every round), 1 on (decode hot lists once per batch), 2 auto."""
+        _check(load_library().griffin_set_reuse(self.h, mode))
 
     def griffin_set_profiling(self, on: bool):
         _check(load_library().griffin_set_profiling(self.h, int(on)))

@@ -252,8 +252,9 @@ void griffin_index_destroy(griffin_index *ix) {
     cudaFree(ix->d_norm);
     Workspace &w = ix->ws;
     for (DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel, &w.qmode,
-                      &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.scal,
-                      &w.keys, &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms})
+                      &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.scal,
+                      &w.keys, &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand,
+                      &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.arena})
       b->release();
     if (w.h_pinned) cudaFreeHost(w.h_pinned);
     for (cudaEvent_t e : ix->ev_pool) cudaEventDestroy(e);
@@ -396,6 +397,13 @@ griffin_status griffin_set_mode(griffin_index *ix, int mode) {
   return GRIFFIN_OK;
 }
 
+griffin_status griffin_set_reuse(griffin_index *ix, int mode) {
+  if (!ix || mode < 0 || mode > 2) return invalid("reuse must be 0 (off), 1 (on) or 2 (auto)");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  ix->reuse = mode;
+  return GRIFFIN_OK;
+}
+
 griffin_status griffin_set_profiling(griffin_index *ix, int on) {
   if (!ix) return invalid("null index");
   std::lock_guard<std::mutex> lk(ix->mu);
@@ -412,7 +420,10 @@ griffin_status griffin_reset_profile(griffin_index *ix) {
   ix->pending.clear();
   ix->ev_next = 0;
   ix->launch_count = 0;
-  if (ix->ws.scal.p) GRIFFIN_CUDA_TRY(cudaMemset(ix->ws.scal.p, 0, 4 * 8));
+  if (ix->ws.scal.p) {
+    GRIFFIN_CUDA_TRY(cudaMemset(ix->ws.scal.p, 0, 4 * 8));
+    GRIFFIN_CUDA_TRY(cudaMemset(ix->ws.scal.as<unsigned long long>() + kScalDec, 0, 3 * 8));
+  }
   return GRIFFIN_OK;
 }
 
@@ -424,22 +435,26 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
   for (auto &p : ix->pending) {
     float ms = 0.f;
     GRIFFIN_CUDA_TRY(cudaEventElapsedTime(&ms, p.second.first, p.second.second));
-    double *slot[5] = {&ix->prof.ms_plan, &ix->prof.ms_intersect, &ix->prof.ms_compact,
-                       &ix->prof.ms_topk, &ix->prof.ms_merge};
+    double *slot[6] = {&ix->prof.ms_plan, &ix->prof.ms_intersect, &ix->prof.ms_compact,
+                       &ix->prof.ms_topk, &ix->prof.ms_merge, &ix->prof.ms_decode};
     *slot[p.first] += ms;
     if (p.first == 1) ix->prof.launches_intersect += 1;
+    if (p.first == 5) ix->prof.launches_decode += 1;
   }
   ix->pending.clear();
   ix->ev_next = 0;
   *out = ix->prof;
   out->launches_total = ix->launch_count;
   if (ix->ws.scal.p) {
-    unsigned long long c[4];
+    unsigned long long c[kScalCount];
     GRIFFIN_CUDA_TRY(cudaMemcpy(c, ix->ws.scal.p, sizeof(c), cudaMemcpyDeviceToHost));
     out->alg_bytes = c[0];
     out->payload_bytes = c[1];
     out->decoded_postings = c[2];
     out->survivors = c[3];
+    out->dec_alg_bytes = c[kScalDec + 0];
+    out->dec_payload_bytes = c[kScalDec + 1];
+    out->dec_postings = c[kScalDec + 2];
   }
   return GRIFFIN_OK;
 }

@@ -54,10 +54,12 @@ struct DevBuf {
 // Query workspace (all grow-only; sized by griffin_reserve / the host API).
 struct Workspace {
   DevBuf plan_terms, plan_m, cap, cap_off, rcount, rsel, qmode, unit_base;  // per query
-  DevBuf unit_off, unit_cnt, unit_dst;                                      // per unit
+  DevBuf unit_off, unit_cnt, unit_dst, urec;                                // per unit
   DevBuf rbuf0, rbuf1, bump, cand;                                          // per survivor
   DevBuf scal;       // scalars: counters, status, bump ctr, unit ctr
   DevBuf keys, counts, docids, scores, qoffs, qterms;  // host-API staging on device
+  DevBuf demand, tdec, runs, run_base, vtmp;           // per term (batch reuse)
+  DevBuf arena;                                        // decoded lists, nblocks * B u32
   size_t nq_cap = 0, unit_cap = 0, entry_cap = 0;
   // pinned host staging
   void *h_pinned = nullptr;
@@ -71,7 +73,8 @@ enum : int {
   kScalUnitCtr = 5,   // u32 unit ticket counter (in a u64 slot)
   kScalStatus = 6,    // int status
   kScalTotals = 7,    // u64 x2: sum cap, sum units (written by plan kernels)
-  kScalCount = 10
+  kScalDec = 10,      // 3 x u64: decode-once alg bytes, payload bytes, postings
+  kScalCount = 13
 };
 
 struct RoundArgs {
@@ -93,6 +96,9 @@ struct RoundArgs {
   uint2 *bump;
   uint64_t entry_cap;
   unsigned long long *scal;
+  uint4 *urec;            // per unit: {q, i0|lu, j0, lo docID} (partition stage)
+  const uint32_t *dec;    // batch decoded arena (global block * B + i), or null
+  const uint8_t *tdec;    // per term: 1 = decoded in the arena this batch
 };
 
 }  // namespace griffin
@@ -118,6 +124,7 @@ struct griffin_index {
   // query state
   griffin::Workspace ws;
   int mode = 0;
+  int reuse = 2;
   bool profiling = false;
   griffin_profile prof{};
   std::vector<cudaEvent_t> ev_pool;

@@ -350,6 +350,87 @@ __device__ __forceinline__ void warp_mp_search2(HR hR, uint32_t nbR, HS hS, uint
   *i1 = __shfl_sync(0xffffffffu, lo, 16);
 }
 
+// Partitioning stage ("Partitioning and Merging"): one thread per
+// unit locates the unit's query and, for merge units, the crossing of the merge
+// path with the unit's first diagonal over the two lists' block heads
+// and the unit's first docID.  The merging stage reads {q, i0, j0, lo} of unit u
+// and of unit u+1 (its end), so no warp ever searches on the critical path.
+template <bool RC>
+__global__ void partition_kernel(DevIndex ix, RoundArgs a) {
+  const uint64_t total = a.unit_base[a.nq];
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u <= total; u += stride) {
+    if (u == total) {
+      a.urec[u] = make_uint4(kNone, 0, 0, 0);
+      continue;
+    }
+    uint32_t lo = 0, hi = a.nq;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (a.unit_base[mid] <= u) lo = mid; else hi = mid;
+    }
+    const uint32_t q = lo;
+    const uint32_t lu = (uint32_t)(u - a.unit_base[q]);
+    uint4 rec = make_uint4(q, lu, 0, 0);
+    if (a.qmode[q] == kModeMerge) {
+      const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
+      const TermInfo tR = ix.terms[pt[0]];
+      const TermInfo tS = ix.terms[pt[a.round]];
+      const uint2 *Rq = RC ? nullptr : a.rprev + a.cap_off[q];
+      const uint32_t nbR = RC ? tR.nblocks : (a.rcount[q] + ix.B - 1) / ix.B;
+      const uint32_t nbS = tS.nblocks;
+      auto hR = [&](uint32_t i) -> uint32_t {
+        return RC ? __ldg(ix.first + tR.block0 + i) : Rq[(size_t)i * ix.B].x;
+      };
+      auto hS = [&](uint32_t j) -> uint32_t { return __ldg(ix.first + tS.block0 + j); };
+      const uint32_t d0 = lu * a.D;
+      uint32_t i0, j0;
+      merge_path_split(hR, nbR, hS, nbS, d0, false, &i0, &j0);
+      uint32_t lov = 0;
+      if (d0 > 0) {
+        const uint64_t INF = 1ull << 32;
+        lov = (uint32_t)min(i0 < nbR ? (uint64_t)hR(i0) : INF, j0 < nbS ? (uint64_t)hS(j0) : INF);
+      }
+      rec = make_uint4(q, i0, j0, lov);
+    }
+    a.urec[u] = rec;
+  }
+}
+
+// Warp-cooperative upper_bound over a[0..n) (global): lanes 0-15 search x0,
+// lanes 16-31 search x1, 16 probes per step (log16 steps instead of log2).
+__device__ __forceinline__ void warp_upper_bound2(const uint32_t *__restrict__ a, uint32_t n,
+                                                  uint32_t x0, uint32_t x1, uint32_t *r0,
+                                                  uint32_t *r1) {
+  const uint32_t lane = lane_id(), half = lane >> 4, hl = lane & 15u;
+  const uint32_t x = half ? x1 : x0;
+  uint32_t lo = 0, hi = n;   // answer: smallest i in [lo, hi] with a[i] > x (a[n] := inf)
+  for (;;) {
+    const bool done = lo >= hi;
+    if (__all_sync(0xffffffffu, done)) break;
+    const uint32_t span = hi - lo;
+    auto cand = [&](uint32_t p) -> uint32_t {
+      return lo + (uint32_t)(((uint64_t)(p + 1) * span + 15u) / 16u) - 1u;
+    };
+    bool pred = true;
+    if (!done) pred = __ldg(a + cand(hl)) > x;
+    const uint32_t hb = (__ballot_sync(0xffffffffu, pred) >> (half * 16u)) & 0xFFFFu;
+    if (!done) {
+      if (hb == 0) {
+        lo = hi;
+      } else {
+        const uint32_t ps = __ffs(hb) - 1u;
+        const uint32_t nhi = cand(ps);
+        const uint32_t nlo = ps ? cand(ps - 1) + 1u : lo;
+        hi = nhi;
+        lo = nlo;
+      }
+    }
+  }
+  *r0 = __shfl_sync(0xffffffffu, lo, 0);
+  *r1 = __shfl_sync(0xffffffffu, lo, 16);
+}
+
 template <bool RC>
 __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevIndex ix, RoundArgs a) {
   extern __shared__ uint4 smem4[];
@@ -357,68 +438,68 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
   const uint32_t B = ix.B, D = a.D;
   WarpSmem sm = carve_warp_smem(smem4, B, D);
   cta_smem_init(smem4, sm);
-  const uint64_t *ubase = a.unit_base;
-  const uint64_t total = ubase[a.nq];
+  const uint64_t total = a.unit_base[a.nq];
   const uint32_t G = min(D - 1u, 31u);   // gallop: S blocks staged per group
+  const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   Acc acc;
-  for (;;) {
-    unsigned long long u = 0;
-    if (lane == 0) u = atomicAdd(a.scal + kScalUnitCtr, 1ull);
-    u = __shfl_sync(0xffffffffu, u, 0);
-    if (u >= total) break;
-    uint32_t qlo = 0, qhi = a.nq;
-    while (qhi - qlo > 1) {
-      const uint32_t mid = (qlo + qhi) >> 1;
-      if (ubase[mid] <= u) qlo = mid; else qhi = mid;
-    }
-    const uint32_t q = qlo;
-    const uint32_t lu = (uint32_t)(u - ubase[q]);
+  for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); u < total;
+       u += nwarps) {
+    const uint4 rec = a.urec[u];
+    const uint4 nxt = a.urec[u + 1];
+    const uint32_t q = rec.x;
+    const uint32_t lu = rec.y;   // gallop/all: unit index within the query
     const uint32_t mode = a.qmode[q];
     const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
-    const TermInfo tR = ix.terms[pt[0]];
+    const uint32_t t0 = pt[0];
+    const TermInfo tR = ix.terms[t0];
     const uint2 *Rq = RC ? nullptr : a.rprev + a.cap_off[q];
     const uint32_t nR = RC ? tR.df_local : a.rcount[q];
     const uint32_t nbR = RC ? tR.nblocks : (nR + B - 1) / B;
+    // R source: compressed EF, the batch's decoded arena, or the intermediate
+    const bool rdec = RC && a.tdec && a.tdec[t0];
+    const uint32_t *decR = rdec ? a.dec + (size_t)tR.block0 * B : nullptr;
 
     if (RC && mode == kModeAll) {  // single-term query: the whole list is the result
-      const uint64_t gb = (uint64_t)tR.block0 + lu;
-      const uint2 m = ix.meta[gb];
-      const uint32_t f = ix.first[gb];
-      const uint32_t sz = block_size16(m.y);
-      stage_blocks(ix, sm, 1, m, 0, sz, true);
-      warp_decode_staged(sm.stg, f, m.y, sm.tile, sm.cnt, sm.lut);
-      const uint32_t n = meta_n(m.y);
-      if (lane == 0) {
-        acc.pay += sz * 16u;
-        acc.post += n;
-        acc.alg += sz * 16u + 8u;
+      const uint32_t n = min(B, nR - lu * B);
+      if (rdec) {
+        if (lane == 0) {
+          fence_proxy_async();
+          mbar_expect_tx(sm.mbar, ((n + 3u) & ~3u) * 4u);
+          bulk_g2s(sm.tile, decR + (size_t)lu * B, ((n + 3u) & ~3u) * 4u, sm.mbar);
+        }
+        mbar_wait(sm.mbar, sm.phase);
+        sm.phase ^= 1u;
+        if (lane == 0) acc.alg += n * 4u;
+      } else {
+        const uint64_t gb = (uint64_t)tR.block0 + lu;
+        const uint2 m = ix.meta[gb];
+        const uint32_t f = ix.first[gb];
+        const uint32_t sz = block_size16(m.y);
+        stage_blocks(ix, sm, 1, m, 0, sz, true);
+        warp_decode_staged(sm.stg, f, m.y, sm.tile, sm.cnt, sm.lut);
+        if (lane == 0) {
+          acc.pay += sz * 16u;
+          acc.post += n;
+          acc.alg += sz * 16u + 8u;
+        }
       }
       emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, 0, n, lu * B, acc);
       continue;
     }
-    const TermInfo tS = ix.terms[pt[a.round]];
+    const uint32_t tSid = pt[a.round];
+    const TermInfo tS = ix.terms[tSid];
     const uint32_t *fS = ix.first + tS.block0;
     const uint32_t nbS = tS.nblocks;
+    const bool sdec = a.tdec && a.tdec[tSid];
+    const uint32_t *decS = sdec ? a.dec + (size_t)tS.block0 * B : nullptr;
 
     if (mode == kModeMerge) {
-      // ---- coarse merge path over the block heads (skip pointers, no decode) ----
-      auto hR = [&](uint32_t i) -> uint32_t {
-        return RC ? __ldg(ix.first + tR.block0 + i) : Rq[i * B].x;
-      };
-      auto hS = [&](uint32_t j) -> uint32_t { return __ldg(fS + j); };
-      const uint32_t tot = nbR + nbS;
-      const uint32_t d0 = lu * D, d1 = min(d0 + D, tot);
-      uint32_t i0, i1;
-      warp_mp_search2(hR, nbR, hS, nbS, d0, d1, &i0, &i1);
-      const uint32_t j0 = d0 - i0, j1 = d1 - i1;
-      const uint64_t INF = 1ull << 32;
-      uint64_t lo_v = 0, hi_v = INF;
-      if (lane == 0 && d0 > 0)
-        lo_v = min(i0 < nbR ? (uint64_t)hR(i0) : INF, j0 < nbS ? (uint64_t)hS(j0) : INF);
-      if (lane == 1 && d1 < tot)
-        hi_v = min(i1 < nbR ? (uint64_t)hR(i1) : INF, j1 < nbS ? (uint64_t)hS(j1) : INF);
-      lo_v = __shfl_sync(0xffffffffu, lo_v, 0);
-      hi_v = __shfl_sync(0xffffffffu, hi_v, 1);
+      // ---- the unit's docID range [lo, hi) and block ranges, from the partition
+      // stage's merge-path crossings (unit u and unit u+1) ----
+      const uint32_t i0 = rec.y, j0 = rec.z;
+      const bool last = nxt.x != q;
+      const uint32_t i1 = last ? nbR : nxt.y, j1 = last ? nbS : nxt.z;
+      const uint64_t lo_v = rec.w, hi_v = last ? (1ull << 32) : (uint64_t)nxt.w;
       const uint32_t rb0 = i0 ? i0 - 1 : 0, rb1 = i1;
       const uint32_t sb0 = j0 ? j0 - 1 : 0, sb1 = j1;
       const uint32_t nRb = rb1 > rb0 ? rb1 - rb0 : 0, nSb = sb1 > sb0 ? sb1 - sb0 : 0;
@@ -426,86 +507,94 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
         if (lane == 0) {
           a.unit_off[u] = 0;
           a.unit_cnt[u] = 0;
-          // accounting: heads in this unit are still "read" (skip entries only)
         }
         continue;
       }
-      // ---- metas: lanes [0,nRb) R blocks (compressed R), [nRb, nRb+nSb) S blocks ----
+      const uint32_t nRt = min(rb1 * B, nR) - rb0 * B;
+      const uint32_t nSt = min(sb1 * B, tS.df_local) - sb0 * B;
+      uint32_t *tileS = sm.tile + nRb * B;
+      // ---- metas of the compressed lists: lanes [0,nRb) R, [nRb, nRb+nSb) S ----
+      const bool rcomp = RC && !rdec;
       const bool isR = lane < nRb, isS = lane >= nRb && lane < nRb + nSb;
+      const bool lm = (rcomp && isR) || (!sdec && isS);
       uint2 m = make_uint2(0, 0);
       uint32_t f = 0;
-      if ((RC && isR) || isS) {
+      if (lm) {
         const uint64_t gb = isR ? (uint64_t)tR.block0 + rb0 + lane
                                 : (uint64_t)tS.block0 + sb0 + (lane - nRb);
         m = ix.meta[gb];
         f = ix.first[gb];
       }
-      const uint32_t sz = ((RC && isR) || isS) ? block_size16(m.y) : 0u;
-      // staging layout: R range then S range, each as contiguous as in HBM
+      const uint32_t sz = lm ? block_size16(m.y) : 0u;
       const uint32_t mR0 = __shfl_sync(0xffffffffu, m.x, 0);
       const uint32_t mS0 = __shfl_sync(0xffffffffu, m.x, nRb);
-      const uint32_t totR16 = __reduce_add_sync(0xffffffffu, (RC && isR) ? sz : 0u);
+      const uint32_t totR16 = __reduce_add_sync(0xffffffffu, (lm && isR) ? sz : 0u);
+      const uint32_t totS16 = __reduce_add_sync(0xffffffffu, (lm && isS) ? sz : 0u);
       const uint32_t soff = isR ? m.x - mR0 : (isS ? totR16 + (m.x - mS0) : 0u);
-      // accounting: blocks whose head lies in this unit (straddlers belong to the
-      // previous unit)
+      // ---- accounting: blocks whose head lies in this unit ----
       {
         const bool own = (isR && rb0 + lane >= i0) || (isS && sb0 + (lane - nRb) >= j0);
-        const uint32_t pay = own ? sz * 16u : 0u;
-        const uint32_t nn = (own && ((RC && isR) || isS)) ? meta_n(m.y) : 0u;
-        const uint32_t rbytes = (!RC && isR && own) ? min(B, nR - (rb0 + lane) * B) * 8u : 0u;
+        const uint32_t nn = isR ? min(B, nR - (rb0 + lane) * B)
+                                : (isS ? min(B, tS.df_local - (sb0 + lane - nRb) * B) : 0u);
+        uint32_t pay = 0, post = 0, alg = 0;
+        if (own) {
+          if (lm) {
+            pay = sz * 16u;
+            post = nn;
+            alg = pay + 8u;
+          } else {
+            alg = nn * (isR && !RC ? 8u : 4u);  // intermediate (docID+score) or decoded arena
+          }
+        }
         const uint32_t sp = __reduce_add_sync(0xffffffffu, pay);
-        const uint32_t sn = __reduce_add_sync(0xffffffffu, nn);
-        const uint32_t sr = __reduce_add_sync(0xffffffffu, rbytes);
-        const uint32_t so = __reduce_add_sync(0xffffffffu, (own && ((RC && isR) || isS)) ? 8u : 0u);
+        const uint32_t sn = __reduce_add_sync(0xffffffffu, post);
+        const uint32_t sa = __reduce_add_sync(0xffffffffu, alg);
         if (lane == 0) {
           acc.pay += sp;
           acc.post += sn;
-          acc.alg += sp + sr + so;
+          acc.alg += sa;
         }
       }
-      if (RC) {
-        // two contiguous ranges: issue as per-lane copies of the range heads
-        const uint32_t totS16 = __reduce_add_sync(0xffffffffu, isS ? sz : 0u);
+      // ---- one TMA round trip: compressed payloads -> stg, decoded ranges -> tiles ----
+      {
+        const uint32_t bR = rdec ? ((nRt + 3u) & ~3u) * 4u : totR16 * 16u;
+        const uint32_t bS = sdec ? ((nSt + 3u) & ~3u) * 4u : totS16 * 16u;
+        const uint32_t tx = (RC ? bR : 0u) + bS;
         if (lane == 0) {
           fence_proxy_async();
-          mbar_expect_tx(sm.mbar, (totR16 + totS16) * 16u);
-          bulk_g2s(sm.stg, ix.payload + mR0, totR16 * 16u, sm.mbar);
-          bulk_g2s(sm.stg + totR16 * 4u, ix.payload + mS0, totS16 * 16u, sm.mbar);
+          mbar_expect_tx(sm.mbar, tx);
+          if (RC) {
+            if (rdec) bulk_g2s(sm.tile, decR + (size_t)rb0 * B, bR, sm.mbar);
+            else bulk_g2s(sm.stg, ix.payload + mR0, bR, sm.mbar);
+          }
+          if (sdec) bulk_g2s(tileS, decS + (size_t)sb0 * B, bS, sm.mbar);
+          else bulk_g2s(sm.stg + totR16 * 4u, ix.payload + mS0, bS, sm.mbar);
+        }
+        if (!RC) {  // intermediate R: docIDs out of the (docID, score) entries
+          const uint32_t s0 = rb0 * B;
+          for (uint32_t i = lane; i < nRt; i += 32) sm.tile[i] = Rq[s0 + i].x;
         }
         mbar_wait(sm.mbar, sm.phase);
         sm.phase ^= 1u;
-      } else {
-        // S only: lanes shifted so the S metas start at lane 0 for stage_blocks
-        const uint2 ms = make_uint2(__shfl_sync(0xffffffffu, m.x, (lane + nRb) & 31),
-                                    __shfl_sync(0xffffffffu, m.y, (lane + nRb) & 31));
-        const uint32_t szs = __shfl_sync(0xffffffffu, sz, (lane + nRb) & 31);
-        stage_blocks(ix, sm, nSb, ms, 0, szs, true);
       }
-      // ---- decode the unit's blocks into the smem tiles ----
-      uint32_t nRt;
-      if (RC) {
+      // ---- EF-decode the compressed blocks into the smem tiles ----
+      if (rcomp) {
         for (uint32_t i = 0; i < nRb; ++i) {
           const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
           const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
           const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
           warp_decode_staged(sm.stg + so * 4u, fi, y, sm.tile + i * B, sm.cnt, sm.lut);
         }
-        nRt = (nRb - 1) * B + meta_n(__shfl_sync(0xffffffffu, m.y, nRb - 1));
-      } else {
-        const uint32_t s0 = rb0 * B, s1 = min(rb1 * B, nR);
-        for (uint32_t i = lane; i < s1 - s0; i += 32) sm.tile[i] = Rq[s0 + i].x;
-        nRt = s1 - s0;
-        __syncwarp();
       }
-      uint32_t *tileS = sm.tile + nRb * B;
-      for (uint32_t i = 0; i < nSb; ++i) {
-        const uint32_t y = __shfl_sync(0xffffffffu, m.y, nRb + i);
-        const uint32_t fi = __shfl_sync(0xffffffffu, f, nRb + i);
-        const uint32_t so = RC ? __shfl_sync(0xffffffffu, soff, nRb + i)
-                               : __shfl_sync(0xffffffffu, m.x, nRb + i) - mS0;
-        warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+      if (!sdec) {
+        for (uint32_t i = 0; i < nSb; ++i) {
+          const uint32_t y = __shfl_sync(0xffffffffu, m.y, nRb + i);
+          const uint32_t fi = __shfl_sync(0xffffffffu, f, nRb + i);
+          const uint32_t so = __shfl_sync(0xffffffffu, soff, nRb + i);
+          warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+        }
       }
-      const uint32_t nSt = (nSb - 1) * B + meta_n(__shfl_sync(0xffffffffu, m.y, nRb + nSb - 1));
+      __syncwarp();
       // ranges inside [lo, hi)
       uint32_t r_lo = 0;
       if (lane == 0) r_lo = lower_bound_s(sm.tile, 0, nRt, lo_v);
@@ -553,31 +642,59 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
       uint32_t *tileR = sm.tile, *kidx = sm.tile + B, *match = sm.tile + 2 * B;
       uint32_t *tileS = sm.tile + 3 * B;
       uint32_t *dblk = sm.aux, *sn = sm.aux + B;
-      uint32_t n;
-      if (RC) {
+      const uint32_t n = min(B, nR - lu * B);
+      if (RC && rdec) {
+        const uint32_t by = ((n + 3u) & ~3u) * 4u;
+        if (lane == 0) {
+          fence_proxy_async();
+          mbar_expect_tx(sm.mbar, by);
+          bulk_g2s(tileR, decR + (size_t)lu * B, by, sm.mbar);
+        }
+        mbar_wait(sm.mbar, sm.phase);
+        sm.phase ^= 1u;
+        if (lane == 0) acc.alg += n * 4u;
+      } else if (RC) {
         const uint64_t gb = (uint64_t)tR.block0 + lu;
         const uint2 m = ix.meta[gb];
         const uint32_t f = ix.first[gb];
         const uint32_t sz = block_size16(m.y);
         stage_blocks(ix, sm, 1, m, 0, sz, true);
         warp_decode_staged(sm.stg, f, m.y, tileR, sm.cnt, sm.lut);
-        n = meta_n(m.y);
         if (lane == 0) {
           acc.pay += sz * 16u;
           acc.post += n;
           acc.alg += sz * 16u + 8u;
         }
       } else {
-        n = load_r_chunk(Rq, nR, B, lu, tileR);
+        load_r_chunk(Rq, nR, B, lu, tileR);
         if (lane == 0) acc.alg += n * 8u;
       }
-      uint32_t kk = 0;
-      if (lane == 0) kk = upper_bound_g(fS, 0, nbS, tileR[0]);
-      if (lane == 1) kk = upper_bound_g(fS, 0, nbS, tileR[n - 1]);
-      const uint32_t k_lo = __shfl_sync(0xffffffffu, kk, 0), k_hi = __shfl_sync(0xffffffffu, kk, 1);
-      for (uint32_t e = lane; e < n; e += 32) {
-        kidx[e] = upper_bound_g(fS, k_lo, k_hi, tileR[e]) - 1u;   // kNone: below S's first docID
-        match[e] = kNone;
+      __syncwarp();
+      uint32_t k_lo, k_hi;
+      warp_upper_bound2(fS, nbS, tileR[0], tileR[n - 1], &k_lo, &k_hi);
+      // skip pointers the chunk can touch: [k_lo-1, k_hi); stage them in smem when
+      // they fit (one round trip), else search them in global memory
+      const uint32_t w0 = k_lo ? k_lo - 1u : 0u, span = k_hi - w0;
+      if (span <= stage_words(B, D)) {
+        uint32_t *win = sm.stg;
+        for (uint32_t i = lane; i < span; i += 32) win[i] = __ldg(fS + w0 + i);
+        __syncwarp();
+        for (uint32_t e = lane; e < n; e += 32) {
+          // upper_bound in the window, shifted back to block indices
+          uint32_t lo2 = 0, hi2 = span;
+          const uint32_t x = tileR[e];
+          while (lo2 < hi2) {
+            const uint32_t mid = (lo2 + hi2) >> 1;
+            if (win[mid] <= x) lo2 = mid + 1; else hi2 = mid;
+          }
+          kidx[e] = w0 + lo2 - 1u;   // kNone: below S's first docID
+          match[e] = kNone;
+        }
+      } else {
+        for (uint32_t e = lane; e < n; e += 32) {
+          kidx[e] = upper_bound_g(fS, k_lo, k_hi, tileR[e]) - 1u;
+          match[e] = kNone;
+        }
       }
       __syncwarp();
       const uint32_t k_first = kidx[0];
@@ -605,33 +722,52 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
       for (uint32_t g0 = 0; g0 < nd; g0 += G) {
         const uint32_t ng = min(G, nd - g0);
         uint2 m = make_uint2(0, 0);
-        uint32_t f = 0, sz = 0, blk = 0;
+        uint32_t f = 0, sz = 0, blk = 0, nn = 0;
         if (lane < ng) {
           blk = dblk[g0 + lane];
-          m = ix.meta[(uint64_t)tS.block0 + blk];
-          f = ix.first[(uint64_t)tS.block0 + blk];
-          sz = block_size16(m.y);
-          sn[lane] = meta_n(m.y);
+          nn = min(B, tS.df_local - blk * B);
+          sn[lane] = nn;
+          if (!sdec) {
+            m = ix.meta[(uint64_t)tS.block0 + blk];
+            f = ix.first[(uint64_t)tS.block0 + blk];
+            sz = block_size16(m.y);
+          }
         }
-        const uint32_t soff = warp_incl_scan(sz) - sz;
         {
           const bool own = lane < ng && !(lu > 0 && blk == k_first);
-          const uint32_t sp = __reduce_add_sync(0xffffffffu, own ? sz * 16u : 0u);
-          const uint32_t spn = __reduce_add_sync(0xffffffffu, own ? meta_n(m.y) : 0u);
-          const uint32_t so = __reduce_add_sync(0xffffffffu, own ? 8u : 0u);
+          const uint32_t sp = __reduce_add_sync(0xffffffffu, (own && !sdec) ? sz * 16u : 0u);
+          const uint32_t spn = __reduce_add_sync(0xffffffffu, (own && !sdec) ? nn : 0u);
+          const uint32_t sa = __reduce_add_sync(
+              0xffffffffu, own ? (sdec ? nn * 4u : sz * 16u + 8u) : 0u);
           if (lane == 0) {
             acc.pay += sp;
             acc.post += spn;
-            acc.alg += sp + so;
+            acc.alg += sa;
           }
         }
-        stage_blocks(ix, sm, ng, m, soff, sz, false);
-        for (uint32_t i = 0; i < ng; ++i) {
-          const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
-          const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
-          const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
-          warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+        if (sdec) {
+          // decoded arena: each touched block straight into its tileS slot
+          const uint32_t by = lane < ng ? ((nn + 3u) & ~3u) * 4u : 0u;
+          const uint32_t tot = __reduce_add_sync(0xffffffffu, by);
+          if (lane == 0) {
+            fence_proxy_async();
+            mbar_expect_tx(sm.mbar, tot);
+          }
+          __syncwarp();
+          if (lane < ng) bulk_g2s(tileS + lane * B, decS + (size_t)blk * B, by, sm.mbar);
+          mbar_wait(sm.mbar, sm.phase);
+          sm.phase ^= 1u;
+        } else {
+          const uint32_t soff = warp_incl_scan(sz) - sz;
+          stage_blocks(ix, sm, ng, m, soff, sz, false);
+          for (uint32_t i = 0; i < ng; ++i) {
+            const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
+            const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
+            const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
+            warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+          }
         }
+        __syncwarp();
         // elements mapping to this group: contiguous from ep
         for (;;) {
           const uint32_t e = ep + lane;
@@ -1076,6 +1212,85 @@ __global__ void __launch_bounds__(256) decode_all_kernel(DevIndex ix, uint32_t D
   }
 }
 
+// ------------------------------------------------------------------- batch reuse
+
+// Estimated block demand of every term in the batch: round 1 reads all blocks
+// of t0; each later term is merged (all its blocks) or galloped (<= |R| blocks),
+// with |R| bounded by the query's region cap after round 1.
+__global__ void demand_kernel(DevIndex ix, RoundArgs a, uint32_t *demand) {
+  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q >= a.nq) return;
+  const uint32_t m = a.plan_m[q];
+  if (!m || !a.cap[q]) return;
+  const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
+  const TermInfo t0 = ix.terms[pt[0]];
+  atomicAdd(&demand[pt[0]], t0.nblocks);
+  uint64_t r_est = t0.df_local;
+  for (uint32_t r = 1; r < m; ++r) {
+    const TermInfo tS = ix.terms[pt[r]];
+    const bool gallop = a.forced_mode == 2 ||
+                        (a.forced_mode == 0 && (uint64_t)tS.df_local > (uint64_t)a.T * r_est);
+    const uint32_t add = gallop ? (uint32_t)(r_est < tS.nblocks ? r_est : tS.nblocks) : tS.nblocks;
+    atomicAdd(&demand[pt[r]], add);
+    if (r == 1) r_est = a.cap[q];
+  }
+}
+
+__global__ void select_kernel(DevIndex ix, const uint32_t *demand, uint8_t *tdec, uint32_t *runs,
+                              uint32_t run_len) {
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= ix.num_terms) return;
+  const uint32_t nb = ix.terms[t].nblocks;
+  // decode once if the batch would otherwise decode >= 1.5x the list's blocks
+  const bool sel = nb > 0 && 2ull * demand[t] >= 3ull * nb;
+  tdec[t] = sel ? 1 : 0;
+  runs[t] = sel ? (nb + run_len - 1) / run_len : 0u;
+}
+
+// Para-EF decode of every block of the selected terms into the arena
+// (slot = global block * B + i): warp per run of <= D+2 consecutive blocks,
+// TMA-staged payloads, decoded tile written back with 128-bit stores.
+__global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t D,
+                                                          const uint64_t *run_base, uint32_t *arena,
+                                                          unsigned long long *scal) {
+  extern __shared__ uint4 smem4[];
+  const uint32_t lane = lane_id();
+  WarpSmem w = carve_warp_smem(smem4, ix.B, D);
+  cta_smem_init(smem4, w);
+  const uint32_t V = ix.num_terms, run = D + 2, B = ix.B;
+  const uint64_t total = run_base[V];
+  const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
+  unsigned long long alg = 0, pay = 0, post = 0;
+  for (uint64_t r = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); r < total;
+       r += nwarps) {
+    uint32_t lo = 0, hi = V;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (run_base[mid] <= r) lo = mid; else hi = mid;
+    }
+    const TermInfo t = ix.terms[lo];
+    const uint32_t ri = (uint32_t)(r - run_base[lo]);
+    const uint32_t k0 = ri * run, nb = min(run, t.nblocks - k0);
+    const uint64_t gb = (uint64_t)t.block0 + k0;
+    uint32_t p;
+    const uint32_t n = decode_run(ix, w, gb, nb, &p);
+    const uint4 *src = reinterpret_cast<const uint4 *>(w.tile);
+    uint4 *dst = reinterpret_cast<uint4 *>(arena + gb * B);
+    for (uint32_t i = lane; i < nb * B / 4u; i += 32) dst[i] = src[i];
+    __syncwarp();
+    if (lane == 0) {
+      pay += p;
+      post += n;
+      alg += p + 8ull * nb + 4ull * n;
+    }
+  }
+  if (lane == 0) {
+    if (alg) atomicAdd(scal + kScalDec + 0, alg);
+    if (pay) atomicAdd(scal + kScalDec + 1, pay);
+    if (post) atomicAdd(scal + kScalDec + 2, post);
+  }
+}
+
 // ------------------------------------------------------------------- host side
 
 static int num_sms(int dev) {
@@ -1102,6 +1317,7 @@ griffin_status reserve_ws(griffin_index *ix, uint32_t nq, uint64_t units, uint64
   GRIFFIN_CUDA_TRY(w.unit_base.reserve(q * 8 + 8 + (q / kScanTile + 8) * 8));
   GRIFFIN_CUDA_TRY(w.unit_off.reserve((units + 1) * 8));
   GRIFFIN_CUDA_TRY(w.unit_cnt.reserve((units + 1) * 4));
+  GRIFFIN_CUDA_TRY(w.urec.reserve((units + 2) * 16));
   GRIFFIN_CUDA_TRY(w.unit_dst.reserve((units + 2) * 8 + (units / kScanTile + 2) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf0.reserve((entries + 1) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf1.reserve((entries + 1) * 8));
@@ -1191,6 +1407,7 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
   ra.unit_base = w.unit_base.as<uint64_t>();
   ra.unit_off = w.unit_off.as<uint64_t>();
   ra.unit_cnt = w.unit_cnt.as<uint32_t>();
+  ra.urec = w.urec.as<uint4>();
   ra.unit_cap = w.unit_cap;
   ra.bump = w.bump.as<uint2>();
   ra.entry_cap = w.entry_cap;
@@ -1209,6 +1426,45 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
     GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(w.cap.as<uint32_t>(), w.cap_off.as<uint64_t>(), nq,
                                               scan_tmp, st, &ix->launch_count));
   }
+  // batch reuse: decode hot lists once into the arena (decompress-then-intersect)
+  const bool reuse = ix->reuse == 1 || (ix->reuse == 2 && nq >= 8);
+  ra.dec = nullptr;
+  ra.tdec = nullptr;
+  if (reuse && ix->V) {
+    StageTimer t(ix, st, 5);
+    const uint32_t V = ix->V;
+    GRIFFIN_CUDA_TRY(w.demand.reserve((size_t)V * 4));
+    GRIFFIN_CUDA_TRY(w.tdec.reserve(V));
+    GRIFFIN_CUDA_TRY(w.runs.reserve((size_t)V * 4));
+    GRIFFIN_CUDA_TRY(w.run_base.reserve(((size_t)V + 2) * 8));
+    GRIFFIN_CUDA_TRY(w.vtmp.reserve(((size_t)V / kScanTile + 4) * 8));
+    GRIFFIN_CUDA_TRY(w.arena.reserve((ix->nblocks * ix->B + 64) * 4));
+    GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.demand.p, 0, (size_t)V * 4, st));
+    ra.T = ix->T;
+    demand_kernel<<<qblocks, 256, 0, st>>>(di, ra, w.demand.as<uint32_t>());
+    select_kernel<<<(V + 255) / 256, 256, 0, st>>>(di, w.demand.as<uint32_t>(),
+                                                   w.tdec.as<uint8_t>(), w.runs.as<uint32_t>(),
+                                                   ix->D + 2);
+    GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(w.runs.as<uint32_t>(), w.run_base.as<uint64_t>(), V,
+                                              w.vtmp.as<uint64_t>(), st, &ix->launch_count));
+    const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * 8;
+    static thread_local int cfg_dev = -1;
+    static thread_local size_t cfg_smem = 0;
+    if (cfg_dev != ix->device || cfg_smem < smem) {
+      GRIFFIN_CUDA_TRY(cudaFuncSetAttribute(decode_once_kernel,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      cfg_dev = ix->device;
+      cfg_smem = smem;
+    }
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, decode_once_kernel, 256, smem);
+    decode_once_kernel<<<num_sms(ix->device) * std::max(1, per_sm), 256, smem, st>>>(
+        di, ix->D, w.run_base.as<uint64_t>(), w.arena.as<uint32_t>(), scal);
+    GRIFFIN_CUDA_TRY(cudaGetLastError());
+    ix->launch_count += 3;
+    ra.dec = w.arena.as<uint32_t>();
+    ra.tdec = w.tdec.as<uint8_t>();
+  }
   const uint32_t rounds = std::max<uint32_t>(1, max_terms > 0 ? max_terms - 1 : 1);
   for (uint32_t r = 1; r <= rounds; ++r) {
     ra.round = r;
@@ -1224,8 +1480,15 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
     }
     {
       StageTimer t(ix, st, 1);
-      if (r == 1) GRIFFIN_CUDA_TRY(launch_intersect<true>(ix, ra, st));
-      else GRIFFIN_CUDA_TRY(launch_intersect<false>(ix, ra, st));
+      const unsigned pgrid = num_sms(ix->device) * 8;
+      if (r == 1) {
+        partition_kernel<true><<<pgrid, 256, 0, st>>>(di, ra);
+        GRIFFIN_CUDA_TRY(launch_intersect<true>(ix, ra, st));
+      } else {
+        partition_kernel<false><<<pgrid, 256, 0, st>>>(di, ra);
+        GRIFFIN_CUDA_TRY(launch_intersect<false>(ix, ra, st));
+      }
+      ix->launch_count += 1;
     }
     {
       StageTimer t(ix, st, 2);

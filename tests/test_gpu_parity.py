@@ -299,3 +299,35 @@ def test_c2_full_size_sampled():
     for q in sample:
         od, os_, oc = ox.query(ql.query(q), k)
         assert_topk_equal(gd[q], gs[q], gc[q], od, os_, oc)
+
+
+# ---------------------------------------------------------------- batch list reuse
+
+@pytest.mark.parametrize("reuse", [0, 1])
+@pytest.mark.parametrize("mode", [g.MODE_AUTO, g.MODE_MERGE, g.MODE_GALLOP])
+def test_reuse_and_modes_bit_exact(tiny, reuse, mode):
+    """Decode-once arena (reuse=1) and fused decode (reuse=0), every intersection
+    mode: identical to the oracle."""
+    c, ql, ox = tiny
+    gx = g.GriffinIndex(c, block_size=128)
+    gx.griffin_set_reuse(reuse)
+    gx.griffin_set_mode(mode)
+    for k in (10, 300):
+        od, os_, oc = ox.query_batch(ql, k)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+def test_reuse_random_batches_and_single_terms():
+    rng = np.random.default_rng(321)
+    for trial in range(4):
+        c = random_corpus(rng, num_docs=int(rng.integers(2000, 80_000)), num_terms=10,
+                          max_df=30_000)
+        ox = oracle.OracleIndex(c)
+        B = int(rng.choice([64, 128, 256, 512]))
+        gx = g.GriffinIndex(c, block_size=B, gallop_ratio=int(rng.choice([0, 3, 500])))
+        gx.griffin_set_reuse(1)
+        ql = random_queries(rng, c.num_terms, 60, max_terms=4)
+        od, os_, oc = ox.query_batch(ql, 50)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 50)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
