@@ -308,6 +308,51 @@ __device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, co
   }
 }
 
+// Ordered emission of per-lane match lists (merge units): lane l found c
+// matches, packed (R tile index | S tile index << 16) at ml[0..c); lanes are in
+// merge-path order, so a warp scan of the counts gives sorted output offsets.
+// Round 1 (RC): s = w_R + w_S; later rounds: s = s_prev + w_S.
+template <bool RC>
+__device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, const TermInfo &tR,
+                           const TermInfo &tS, const uint2 *Rq, const uint32_t *tile,
+                           const uint32_t *ml, uint32_t c, uint32_t posR0, uint32_t posS0,
+                           Acc &acc) {
+  const uint32_t lane = lane_id();
+  const uint32_t incl = warp_incl_scan(c);
+  uint32_t cnt = __shfl_sync(0xffffffffu, incl, 31);
+  unsigned long long off = 0;
+  if (lane == 0 && cnt) off = atomicAdd(a.scal + kScalBump, (unsigned long long)cnt);
+  off = __shfl_sync(0xffffffffu, off, 0);
+  if (off + cnt > a.entry_cap) {
+    if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
+    cnt = 0;
+  }
+  if (cnt) {
+    uint2 *dst = a.bump + off + (incl - c);
+    for (uint32_t j = 0; j < c; ++j) {
+      const uint32_t e = ml[j];
+      const uint32_t i = e & 0xFFFFu;
+      const uint32_t doc = tile[i];
+      const float nrm = __ldg(ix.norm + doc);
+      const float wS = bm25_w(tS.idf, tf_lookup(ix, tS, posS0 + (e >> 16)), nrm, ix.k1p1);
+      float s;
+      if (RC) {
+        s = bm25_w(tR.idf, tf_lookup(ix, tR, posR0 + i), nrm, ix.k1p1);  // first term: s = w
+        s = __fadd_rn(s, wS);
+      } else {
+        s = __fadd_rn(__uint_as_float(Rq[posR0 + i].y), wS);
+      }
+      dst[j] = make_uint2(doc, __float_as_uint(s));
+    }
+  }
+  if (lane == 0) {
+    a.unit_off[u] = off;
+    a.unit_cnt[u] = cnt;
+    acc.surv += cnt;
+    acc.alg += (unsigned long long)cnt * (RC ? 20u : 16u);
+  }
+}
+
 // Coarse merge path over the block heads: lanes 0-15 find the crossing of
 // diagonal d0, lanes 16-31 of d1, with a 16-ary search (each step probes 16
 // points of the diagonal and narrows the range to one interval).
@@ -603,25 +648,30 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
       if (lane == 3) r_lo = lower_bound_s(tileS, 0, nSt, hi_v);
       const uint32_t ra = __shfl_sync(0xffffffffu, r_lo, 0), rb = __shfl_sync(0xffffffffu, r_lo, 1);
       const uint32_t sa = __shfl_sync(0xffffffffu, r_lo, 2), sb = __shfl_sync(0xffffffffu, r_lo, 3);
-      uint32_t *match = sm.stg;   // staging is free after decode
-      for (uint32_t i = ra + lane; i < rb; i += 32) match[i] = kNone;
-      __syncwarp();
       const uint32_t nr = rb - ra, ns = sb - sa;
+      const uint32_t tot2 = nr + ns, L = (tot2 + 31) >> 5;
+      const uint32_t cap = (L >> 1) + 1;           // matches per lane <= ceil(L/2)
+      uint32_t *ml = sm.stg + lane * cap;          // staging is free after decode
+      uint32_t c = 0;
       if (nr && ns) {
-        // ---- fine merge path: lane l owns diagonals [l*L, (l+1)*L) ----
+        // ---- fine merge path: lane l owns diagonals [l*L, (l+1)*L); its end is
+        // the next lane's start, matched pairs never split (A9) ----
         const uint32_t *A = sm.tile + ra, *Bv = tileS + sa;
         auto gA = [&](uint32_t i) -> uint32_t { return A[i]; };
         auto gB = [&](uint32_t j) -> uint32_t { return Bv[j]; };
-        const uint32_t tot2 = nr + ns, L = (tot2 + 31) >> 5;
-        const uint32_t ds = min(lane * L, tot2), de = min(ds + L, tot2);
-        uint32_t is, js, ie, je;
+        const uint32_t ds = min(lane * L, tot2);
+        uint32_t is, js;
         merge_path_split(gA, nr, gB, ns, ds, true, &is, &js);
-        merge_path_split(gA, nr, gB, ns, de, true, &ie, &je);
-        const uint32_t posS0 = sb0 * B + sa;
+        uint32_t ie = __shfl_down_sync(0xffffffffu, is, 1);
+        uint32_t je = __shfl_down_sync(0xffffffffu, js, 1);
+        if (lane == 31) {
+          ie = nr;
+          je = ns;
+        }
         while (is < ie && js < je) {
           const uint32_t x = A[is], y = Bv[js];
           if (x == y) {
-            match[ra + is] = posS0 + js;
+            ml[c++] = (ra + is) | (js << 16);
             ++is;
             ++js;
           } else if (x < y) {
@@ -633,9 +683,9 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
       }
       __syncwarp();
       if (RC)
-        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, match, ra, rb, rb0 * B, acc);
+        emit_lanes<true>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, ml, c, rb0 * B, sb0 * B + sa, acc);
       else
-        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, match, ra, rb, rb0 * B, acc);
+        emit_lanes<false>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, ml, c, rb0 * B, sb0 * B + sa, acc);
       __syncwarp();
     } else {
       // ---- gallop: R chunk lu, skip-pointer search into S (Fig. 9) ----
