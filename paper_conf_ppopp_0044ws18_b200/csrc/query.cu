@@ -175,7 +175,10 @@ struct Acc {
 // the per-R-element match array.  The gallop path carves tile into
 // tileR | kidx | match | tileS[G blocks].
 __host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D) {
-  return (D + 2) * stage_words_per_block(B);
+  // ~2 B per posting of compressed payload for a unit's D+2 blocks (larger units
+  // are staged in capacity-sized batches); also holds the merge's per-lane match
+  // lists (<= 32*((D+2)*B/64+1) words) and always >= one worst-case block.
+  return ((D + 2) * B / 2 + 64 + 3) & ~3u;
 }
 __host__ __device__ inline uint32_t warp_smem_words(uint32_t B, uint32_t D) {
   return 4 + 64 + (B + 32) + stage_words(B, D) + (D + 2) * B;
@@ -236,6 +239,41 @@ __device__ __forceinline__ void stage_blocks(const DevIndex &ix, WarpSmem &w, ui
   }
   mbar_wait(w.mbar, w.phase);
   w.phase ^= 1u;
+}
+
+// EF-decode the consecutive blocks held by lanes [l0, l0+nb) (meta m, first f,
+// payload size sz in 16-B units; contiguous in the payload) into dst + i*B,
+// staging them with TMA bulk copies in batches that fit the staging area.
+__device__ __forceinline__ void stage_decode_lanes(const DevIndex &ix, WarpSmem &w, uint32_t cap16,
+                                                   uint32_t l0, uint32_t nb, uint2 m, uint32_t f,
+                                                   uint32_t sz, uint32_t *dst) {
+  const uint32_t lane = lane_id();
+  const uint32_t incl = warp_incl_scan(lane >= l0 && lane < l0 + nb ? sz : 0u);
+  uint32_t i = 0;
+  while (i < nb) {
+    const uint32_t li = l0 + i;
+    const uint32_t base = __shfl_sync(0xffffffffu, incl - sz, li);   // exclusive prefix at li
+    const uint32_t fits = __ballot_sync(0xffffffffu, lane >= li && lane < l0 + nb &&
+                                                         incl - base <= cap16);
+    uint32_t nbat = __popc(fits);
+    if (nbat == 0) nbat = 1;   // cannot happen (one block always fits); keep progress
+    const uint32_t bytes = (__shfl_sync(0xffffffffu, incl, li + nbat - 1) - base) * 16u;
+    const uint32_t m0 = __shfl_sync(0xffffffffu, m.x, li);
+    if (lane == 0) {
+      fence_proxy_async();
+      mbar_expect_tx(w.mbar, bytes);
+      bulk_g2s(w.stg, ix.payload + m0, bytes, w.mbar);
+    }
+    mbar_wait(w.mbar, w.phase);
+    w.phase ^= 1u;
+    for (uint32_t k = 0; k < nbat; ++k) {
+      const uint32_t y = __shfl_sync(0xffffffffu, m.y, li + k);
+      const uint32_t fk = __shfl_sync(0xffffffffu, f, li + k);
+      const uint32_t so = __shfl_sync(0xffffffffu, m.x, li + k) - m0;
+      warp_decode_staged(w.stg + so * 4u, fk, y, dst + (i + k) * ix.B, w.cnt, w.lut);
+    }
+    i += nbat;
+  }
 }
 
 // Load R "block" k of an intermediate (chunk of B entries) into dst.
@@ -477,7 +515,7 @@ __device__ __forceinline__ void warp_upper_bound2(const uint32_t *__restrict__ a
 }
 
 template <bool RC>
-__global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevIndex ix, RoundArgs a) {
+__global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevIndex ix, RoundArgs a) {
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
   const uint32_t B = ix.B, D = a.D;
@@ -600,44 +638,54 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
           acc.alg += sa;
         }
       }
-      // ---- one TMA round trip: compressed payloads -> stg, decoded ranges -> tiles ----
+      // ---- TMA: decoded-arena ranges -> tiles; compressed payloads -> stg (one
+      // round trip when they fit the staging area, else capacity-sized batches) ----
+      const uint32_t cap16 = stage_words(B, D) / 4u;
+      const bool fit = totR16 + totS16 <= cap16;
       {
-        const uint32_t bR = rdec ? ((nRt + 3u) & ~3u) * 4u : totR16 * 16u;
-        const uint32_t bS = sdec ? ((nSt + 3u) & ~3u) * 4u : totS16 * 16u;
-        const uint32_t tx = (RC ? bR : 0u) + bS;
-        if (lane == 0) {
+        const uint32_t bRd = rdec ? ((nRt + 3u) & ~3u) * 4u : 0u;
+        const uint32_t bSd = sdec ? ((nSt + 3u) & ~3u) * 4u : 0u;
+        const uint32_t bRc = (rcomp && fit) ? totR16 * 16u : 0u;
+        const uint32_t bSc = (!sdec && fit) ? totS16 * 16u : 0u;
+        const uint32_t tx = bRd + bSd + bRc + bSc;
+        if (lane == 0 && tx) {
           fence_proxy_async();
           mbar_expect_tx(sm.mbar, tx);
-          if (RC) {
-            if (rdec) bulk_g2s(sm.tile, decR + (size_t)rb0 * B, bR, sm.mbar);
-            else bulk_g2s(sm.stg, ix.payload + mR0, bR, sm.mbar);
-          }
-          if (sdec) bulk_g2s(tileS, decS + (size_t)sb0 * B, bS, sm.mbar);
-          else bulk_g2s(sm.stg + totR16 * 4u, ix.payload + mS0, bS, sm.mbar);
+          if (bRd) bulk_g2s(sm.tile, decR + (size_t)rb0 * B, bRd, sm.mbar);
+          if (bSd) bulk_g2s(tileS, decS + (size_t)sb0 * B, bSd, sm.mbar);
+          if (bRc) bulk_g2s(sm.stg, ix.payload + mR0, bRc, sm.mbar);
+          if (bSc) bulk_g2s(sm.stg + totR16 * 4u, ix.payload + mS0, bSc, sm.mbar);
         }
         if (!RC) {  // intermediate R: docIDs out of the (docID, score) entries
           const uint32_t s0 = rb0 * B;
           for (uint32_t i = lane; i < nRt; i += 32) sm.tile[i] = Rq[s0 + i].x;
         }
-        mbar_wait(sm.mbar, sm.phase);
-        sm.phase ^= 1u;
+        if (tx) {
+          mbar_wait(sm.mbar, sm.phase);
+          sm.phase ^= 1u;
+        }
       }
       // ---- EF-decode the compressed blocks into the smem tiles ----
-      if (rcomp) {
-        for (uint32_t i = 0; i < nRb; ++i) {
-          const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
-          const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
-          const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
-          warp_decode_staged(sm.stg + so * 4u, fi, y, sm.tile + i * B, sm.cnt, sm.lut);
+      if (fit) {
+        if (rcomp) {
+          for (uint32_t i = 0; i < nRb; ++i) {
+            const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
+            const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
+            const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
+            warp_decode_staged(sm.stg + so * 4u, fi, y, sm.tile + i * B, sm.cnt, sm.lut);
+          }
         }
-      }
-      if (!sdec) {
-        for (uint32_t i = 0; i < nSb; ++i) {
-          const uint32_t y = __shfl_sync(0xffffffffu, m.y, nRb + i);
-          const uint32_t fi = __shfl_sync(0xffffffffu, f, nRb + i);
-          const uint32_t so = __shfl_sync(0xffffffffu, soff, nRb + i);
-          warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+        if (!sdec) {
+          for (uint32_t i = 0; i < nSb; ++i) {
+            const uint32_t y = __shfl_sync(0xffffffffu, m.y, nRb + i);
+            const uint32_t fi = __shfl_sync(0xffffffffu, f, nRb + i);
+            const uint32_t so = __shfl_sync(0xffffffffu, soff, nRb + i);
+            warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+          }
         }
+      } else {
+        if (rcomp) stage_decode_lanes(ix, sm, cap16, 0, nRb, m, f, sz, sm.tile);
+        if (!sdec) stage_decode_lanes(ix, sm, cap16, nRb, nSb, m, f, sz, tileS);
       }
       __syncwarp();
       // ranges inside [lo, hi)
@@ -769,20 +817,28 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
       }
       __syncwarp();
       uint32_t ep = e_first;
-      for (uint32_t g0 = 0; g0 < nd; g0 += G) {
-        const uint32_t ng = min(G, nd - g0);
+      const uint32_t cap16 = stage_words(B, D) / 4u;
+      for (uint32_t g0 = 0; g0 < nd;) {
+        uint32_t ng = min(G, nd - g0);
         uint2 m = make_uint2(0, 0);
         uint32_t f = 0, sz = 0, blk = 0, nn = 0;
         if (lane < ng) {
           blk = dblk[g0 + lane];
           nn = min(B, tS.df_local - blk * B);
-          sn[lane] = nn;
           if (!sdec) {
             m = ix.meta[(uint64_t)tS.block0 + blk];
             f = ix.first[(uint64_t)tS.block0 + blk];
             sz = block_size16(m.y);
           }
         }
+        if (!sdec) {  // as many touched blocks as the staging area holds
+          const uint32_t inc = warp_incl_scan(sz);
+          const uint32_t nfit = __popc(__ballot_sync(0xffffffffu, lane < ng && inc <= cap16));
+          ng = nfit ? nfit : 1u;
+          if (lane >= ng) sz = 0;
+        }
+        if (lane < ng) sn[lane] = nn;
+        __syncwarp();
         {
           const bool own = lane < ng && !(lu > 0 && blk == k_first);
           const uint32_t sp = __reduce_add_sync(0xffffffffu, (own && !sdec) ? sz * 16u : 0u);
@@ -834,6 +890,7 @@ __global__ void __launch_bounds__(kIntersectThreads, 2) intersect_kernel(DevInde
           if (bal != 0xffffffffu) break;
         }
         __syncwarp();
+        g0 += ng;
       }
       if (RC)
         emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
@@ -1181,8 +1238,8 @@ __global__ void keys_to_results_kernel(uint32_t nq, uint32_t k, const uint64_t *
 
 // Warp decodes the consecutive blocks [k0, k0+nb) (nb <= D+2) of the shard into
 // w.tile via one TMA bulk copy; returns total postings and payload bytes.
-__device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, uint64_t k0,
-                                               uint32_t nb, uint32_t *pay_bytes,
+__device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, uint32_t D,
+                                               uint64_t k0, uint32_t nb, uint32_t *pay_bytes,
                                                uint32_t *my_n = nullptr) {
   const uint32_t lane = lane_id();
   uint2 m = make_uint2(0, 0);
@@ -1192,16 +1249,8 @@ __device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, 
     f = ix.first[k0 + lane];
     sz = block_size16(m.y);
   }
-  const uint32_t m0 = __shfl_sync(0xffffffffu, m.x, 0);
-  stage_blocks(ix, w, nb, m, 0, sz, true);
-  uint32_t tot = 0;
-  for (uint32_t i = 0; i < nb; ++i) {
-    const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
-    const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
-    const uint32_t so = __shfl_sync(0xffffffffu, m.x, i) - m0;
-    warp_decode_staged(w.stg + so * 4u, fi, y, w.tile + i * ix.B, w.cnt, w.lut);
-    tot += meta_n(y);
-  }
+  stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, w.tile);
+  const uint32_t tot = __reduce_add_sync(0xffffffffu, lane < nb ? meta_n(m.y) : 0u);
   *pay_bytes = __reduce_add_sync(0xffffffffu, sz) * 16u;
   if (my_n) *my_n = lane < nb ? meta_n(m.y) : 0u;
   return tot;
@@ -1219,7 +1268,7 @@ __global__ void __launch_bounds__(256) decode_list_kernel(DevIndex ix, uint32_t 
   for (uint32_t r = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); r < nruns; r += nwarps) {
     const uint32_t k = r * run, nb = min(run, nblocks - k);
     uint32_t pay;
-    const uint32_t n = decode_run(ix, w, (uint64_t)block0 + k, nb, &pay);
+    const uint32_t n = decode_run(ix, w, D, (uint64_t)block0 + k, nb, &pay);
     for (uint32_t i = lane; i < n; i += 32) out[(size_t)k * ix.B + i] = w.tile[i] + ix.doc_base;
     __syncwarp();
   }
@@ -1243,7 +1292,7 @@ __global__ void __launch_bounds__(256) decode_all_kernel(DevIndex ix, uint32_t D
     const uint32_t nb = (uint32_t)((nblocks - k) < run ? (nblocks - k) : run);
     uint32_t p;
     uint32_t mn;
-    const uint32_t n = decode_run(ix, w, k, nb, &p, &mn);
+    const uint32_t n = decode_run(ix, w, D, k, nb, &p, &mn);
     // blocks of a run may belong to different terms: only each term's last block
     // is short, so XOR block by block
     for (uint32_t bi = 0; bi < nb; ++bi) {
@@ -1323,7 +1372,7 @@ __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t 
     const uint32_t k0 = ri * run, nb = min(run, t.nblocks - k0);
     const uint64_t gb = (uint64_t)t.block0 + k0;
     uint32_t p;
-    const uint32_t n = decode_run(ix, w, gb, nb, &p);
+    const uint32_t n = decode_run(ix, w, D, gb, nb, &p);
     const uint4 *src = reinterpret_cast<const uint4 *>(w.tile);
     uint4 *dst = reinterpret_cast<uint4 *>(arena + gb * B);
     for (uint32_t i = lane; i < nb * B / 4u; i += 32) dst[i] = src[i];
