@@ -252,7 +252,7 @@ void griffin_index_destroy(griffin_index *ix) {
     cudaFree(ix->d_norm);
     Workspace &w = ix->ws;
     for (DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel, &w.qmode,
-                      &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.scal,
+                      &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal,
                       &w.keys, &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand,
                       &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.arena})
       b->release();

@@ -55,7 +55,7 @@ struct DevBuf {
 struct Workspace {
   DevBuf plan_terms, plan_m, cap, cap_off, rcount, rsel, qmode, unit_base;  // per query
   DevBuf unit_off, unit_cnt, unit_dst, urec;                                // per unit
-  DevBuf rbuf0, rbuf1, bump, cand;                                          // per survivor
+  DevBuf rbuf0, rbuf1, bump, cand, tkstate;                                 // per survivor
   DevBuf scal;       // scalars: counters, status, bump ctr, unit ctr
   DevBuf keys, counts, docids, scores, qoffs, qterms;  // host-API staging on device
   DevBuf demand, tdec, runs, run_base, vtmp;           // per term (batch reuse)

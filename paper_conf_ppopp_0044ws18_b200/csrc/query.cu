@@ -1086,13 +1086,54 @@ __device__ uint64_t cta_radix_select(KeyF key, uint32_t n, uint32_t kk, SelectSm
   return ss.prefix;
 }
 
-// Level 1: every query with more than kTopkSmem survivors is cut into chunks of
-// kTopkSmem; each chunk (one CTA, keys staged in smem) keeps its top min(k, len)
-// keys in cand[(cbase[q] + ci) * k ...] (zero-padded).
+constexpr int kTopkMaxLevels = 5;
+struct CandBufs {
+  uint64_t *lv[kTopkMaxLevels + 1];   // lv[L] = candidates produced by level L (L >= 1)
+};
+
+// Per query, where its current top-k candidates live: qlev 0 = the survivor
+// entries of the final intersection round, qlev L >= 1 = cand level L at qoff.
+struct TopkState {
+  uint8_t *qlev;
+  uint64_t *qoff;
+  uint32_t *qn;
+};
+
+__global__ void topk_init_kernel(uint32_t nq, const uint32_t *rcount, TopkState ts) {
+  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q < nq) {
+    ts.qlev[q] = 0;
+    ts.qoff[q] = 0;
+    ts.qn[q] = rcount[q];
+  }
+}
+
+__global__ void topk_plan_kernel(uint32_t nq, TopkState ts, uint32_t *nch) {
+  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q < nq) {
+    const uint32_t c = ts.qn[q];
+    nch[q] = c > kTopkSmem ? (c + kTopkSmem - 1) / kTopkSmem : 0u;
+  }
+}
+
+__global__ void topk_update_kernel(uint32_t nq, uint32_t k, uint32_t level, TopkState ts,
+                                   const uint32_t *nch, const uint64_t *cbase) {
+  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q < nq && nch[q]) {
+    ts.qlev[q] = (uint8_t)level;
+    ts.qoff[q] = cbase[q] * k;
+    ts.qn[q] = nch[q] * k;
+  }
+}
+
+// One selection level: every query with more than kTopkSmem candidates is cut
+// into chunks of kTopkSmem; each chunk (one CTA, keys staged in smem) keeps its
+// top min(k, len) keys at out[(cbase[q] + ci) * k ...] (zero-padded).  Levels
+// repeat until every query's candidates fit one CTA's shared memory.
 __global__ void __launch_bounds__(kTopkThreads) topk_chunk_kernel(
-    DevIndex ix, uint32_t nq, uint32_t k, const uint32_t *rcount, const uint8_t *rsel,
-    const uint64_t *cap_off, const uint2 *rb0, const uint2 *rb1, const uint64_t *cbase,
-    uint64_t *cand) {
+    DevIndex ix, uint32_t nq, uint32_t k, const uint8_t *rsel, const uint64_t *cap_off,
+    const uint2 *rb0, const uint2 *rb1, TopkState ts, CandBufs cb, const uint64_t *cbase,
+    uint64_t *out_lv) {
   __shared__ uint64_t sk[kTopkSmem];
   __shared__ SelectSmem ss;
   const uint64_t total = cbase[nq];
@@ -1104,43 +1145,53 @@ __global__ void __launch_bounds__(kTopkThreads) topk_chunk_kernel(
     }
     const uint32_t q = lo;
     const uint32_t ci = (uint32_t)(c - cbase[q]);
-    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q] + (size_t)ci * kTopkSmem;
-    const uint32_t len = min(kTopkSmem, rcount[q] - ci * kTopkSmem);
-    for (uint32_t i = threadIdx.x; i < len; i += blockDim.x) sk[i] = make_key(R[i], ix.doc_base);
+    const uint32_t lev = ts.qlev[q];
+    const uint32_t len = min(kTopkSmem, ts.qn[q] - ci * kTopkSmem);
+    if (lev == 0) {
+      const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q] + (size_t)ci * kTopkSmem;
+      for (uint32_t i = threadIdx.x; i < len; i += blockDim.x) sk[i] = make_key(R[i], ix.doc_base);
+    } else {
+      const uint64_t *K = cb.lv[lev] + ts.qoff[q] + (size_t)ci * kTopkSmem;
+      for (uint32_t i = threadIdx.x; i < len; i += blockDim.x) sk[i] = K[i];
+    }
     __syncthreads();
-    uint64_t *out = cand + c * k;
+    uint64_t *out = out_lv + c * k;
     const uint32_t kk = min(k, len);
     if (kk == len) {
       for (uint32_t i = threadIdx.x; i < k; i += blockDim.x) out[i] = i < len ? sk[i] : 0ull;
     } else {
+      // inputs of levels >= 2 carry zero padding (below every real key; not
+      // unique): keep the nonzero keys >= thr — exactly kk when thr > 0, all of
+      // them (< kk) when thr == 0 — and zero-fill the rest of the k slots
       const uint64_t thr = cta_radix_select([&](uint32_t i) { return sk[i]; }, len, kk, ss);
       if (threadIdx.x == 0) ss.cnt = 0;
       __syncthreads();
       for (uint32_t i = threadIdx.x; i < len; i += blockDim.x)
-        if (sk[i] >= thr) out[atomicAdd(&ss.cnt, 1u)] = sk[i];
-      for (uint32_t i = kk + threadIdx.x; i < k; i += blockDim.x) out[i] = 0ull;
+        if (sk[i] >= thr && sk[i] != 0ull) out[atomicAdd(&ss.cnt, 1u)] = sk[i];
+      __syncthreads();
+      for (uint32_t i = ss.cnt + threadIdx.x; i < k; i += blockDim.x) out[i] = 0ull;
     }
     __syncthreads();
   }
 }
 
-// Level 2, per query: the survivors (<= kTopkSmem) or the level-1 candidates;
-// select the top kk in smem (or by global radix passes when the candidates do
-// not fit), bitonic-sort them, write keys + count.
+// Final, per query: select the top kk of its current candidates in smem (or by
+// global radix passes when they still do not fit), bitonic-sort, write keys +
+// count.  Zero keys (chunk padding) are below every real key.
 __global__ void __launch_bounds__(kTopkThreads) topk_final_kernel(
     DevIndex ix, uint32_t nq, uint32_t k, const uint32_t *rcount, const uint8_t *rsel,
-    const uint64_t *cap_off, const uint2 *rb0, const uint2 *rb1, const uint64_t *cbase,
-    const uint64_t *cand, uint64_t *out_keys, uint32_t *out_counts) {
+    const uint64_t *cap_off, const uint2 *rb0, const uint2 *rb1, TopkState ts, CandBufs cb,
+    uint64_t *out_keys, uint32_t *out_counts) {
   __shared__ uint64_t sk[kTopkSmem];
   __shared__ SelectSmem ss;
   for (uint32_t q = blockIdx.x; q < nq; q += gridDim.x) {
     const uint32_t c = rcount[q];
     const uint32_t kk = min(k, c);
     const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q];
-    const bool big = c > kTopkSmem;
-    const uint64_t *C = cand + cbase[q] * k;
-    const uint32_t n = big ? (uint32_t)((cbase[q + 1] - cbase[q]) * k) : c;
-    auto key = [&](uint32_t i) -> uint64_t { return big ? C[i] : make_key(R[i], ix.doc_base); };
+    const uint32_t lev = ts.qlev[q];
+    const uint64_t *C = lev ? cb.lv[lev] + ts.qoff[q] : nullptr;
+    const uint32_t n = ts.qn[q];
+    auto key = [&](uint32_t i) -> uint64_t { return lev ? C[i] : make_key(R[i], ix.doc_base); };
     uint32_t nsel;
     if (n <= kTopkSmem) {
       for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) sk[i] = key(i);
@@ -1178,14 +1229,6 @@ __global__ void __launch_bounds__(kTopkThreads) topk_final_kernel(
       out_keys[(size_t)q * k + i] = i < kk ? sk[i] : 0ull;
     if (threadIdx.x == 0) out_counts[q] = kk;
     __syncthreads();
-  }
-}
-
-__global__ void topk_plan_kernel(uint32_t nq, const uint32_t *rcount, uint32_t *nch) {
-  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
-  if (q < nq) {
-    const uint32_t c = rcount[q];
-    nch[q] = c > kTopkSmem ? (c + kTopkSmem - 1) / kTopkSmem : 0u;
   }
 }
 
@@ -1607,18 +1650,36 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
     StageTimer t(ix, st, 3);
     uint32_t *nch = qunits;  // reuse the per-query unit-count scratch
     uint64_t *cbase = w.unit_base.as<uint64_t>();
+    // candidates per level <= (entries / kTopkSmem + nq + 1) * k (each level shrinks them
+    // by kTopkSmem / k; small k needs 2 levels, large k up to kTopkMaxLevels)
     const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
-    GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8));
-    topk_plan_kernel<<<qblocks, 256, 0, st>>>(nq, w.rcount.as<uint32_t>(), nch);
-    GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(nch, cbase, nq, scan_tmp, st, &ix->launch_count));
-    topk_chunk_kernel<<<num_sms(ix->device) * 4, kTopkThreads, 0, st>>>(
-        di, nq, k, w.rcount.as<uint32_t>(), w.rsel.as<uint8_t>(), w.cap_off.as<uint64_t>(),
-        w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), cbase, w.cand.as<uint64_t>());
+    const int levels = k <= 64 ? 2 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
+    GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8 * std::max(levels, 1)));
+    GRIFFIN_CUDA_TRY(w.tkstate.reserve(((size_t)nq + 1) * (1 + 8 + 4) + 64));
+    CandBufs cb{};
+    for (int L = 1; L <= levels; ++L) cb.lv[L] = w.cand.as<uint64_t>() + (size_t)(L - 1) * cand_cap;
+    TopkState ts;
+    ts.qoff = w.tkstate.as<uint64_t>();
+    ts.qn = reinterpret_cast<uint32_t *>(ts.qoff + nq + 1);
+    ts.qlev = reinterpret_cast<uint8_t *>(ts.qn + nq + 1);
+    const uint32_t *rc = w.rcount.as<uint32_t>();
+    const uint8_t *rs = w.rsel.as<uint8_t>();
+    topk_init_kernel<<<qblocks, 256, 0, st>>>(nq, rc, ts);
+    ix->launch_count += 1;
+    for (int L = 1; L <= levels; ++L) {
+      topk_plan_kernel<<<qblocks, 256, 0, st>>>(nq, ts, nch);
+      GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(nch, cbase, nq, scan_tmp, st, &ix->launch_count));
+      topk_chunk_kernel<<<num_sms(ix->device) * 4, kTopkThreads, 0, st>>>(
+          di, nq, k, rs, w.cap_off.as<uint64_t>(), w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), ts,
+          cb, cbase, cb.lv[L]);
+      topk_update_kernel<<<qblocks, 256, 0, st>>>(nq, k, L, ts, nch, cbase);
+      ix->launch_count += 3;
+    }
     topk_final_kernel<<<std::min<uint32_t>(nq, 148 * 4), kTopkThreads, 0, st>>>(
-        di, nq, k, w.rcount.as<uint32_t>(), w.rsel.as<uint8_t>(), w.cap_off.as<uint64_t>(),
-        w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), cbase, w.cand.as<uint64_t>(), d_keys, d_counts);
+        di, nq, k, rc, rs, w.cap_off.as<uint64_t>(), w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), ts,
+        cb, d_keys, d_counts);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
-    ix->launch_count += 3;
+    ix->launch_count += 1;
   }
   return GRIFFIN_OK;
 }

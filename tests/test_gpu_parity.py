@@ -331,3 +331,23 @@ def test_reuse_random_batches_and_single_terms():
         od, os_, oc = ox.query_batch(ql, 50)
         gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 50)
         assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+@pytest.mark.parametrize("k", [64, 65, 1000, 2048])
+def test_multilevel_topk_large_results(k):
+    """Survivor sets of 10^4..10^5 per query force several chunked selection
+    levels (zero-padded candidate arrays) before the final sort."""
+    rng = np.random.default_rng(700 + k)
+    N = 400_000
+    lists = [np.sort(rng.choice(N, size=n, replace=False))
+             for n in (300_000, 250_000, 200_000, 60_000, 9_000)]
+    tfs = [rng.integers(1, 40, size=len(l)) for l in lists]
+    c = corpus_from_lists(N, lists, tfs, rng.integers(1, 5000, size=N))
+    ox = oracle.OracleIndex(c)
+    gx = g.GriffinIndex(c)
+    qs = [[0, 1], [0, 1, 2], [0], [1, 3], [2, 4], [0, 2], [1]]
+    ql = QueryLog(offsets=np.cumsum([0] + [len(q) for q in qs]).astype(np.uint32),
+                  terms=np.concatenate(qs).astype(np.uint32))
+    od, os_, oc = ox.query_batch(ql, k)
+    gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+    assert_topk_equal(gd, gs, gc, od, os_, oc)

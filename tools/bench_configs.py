@@ -1,0 +1,151 @@
+"""Measurements for the BASELINE.json configs beyond bench.py's headline C2 line.
+
+  python tools/bench_configs.py c1        single-query closed-loop latency (p50/p99), C1
+  python tools/bench_configs.py c3        merge-vs-gallop crossover over the paper's ratio
+                                          groups (Fig. 8 / Fig. 13 analog, GPU only)
+  python tools/bench_configs.py c5 [nq]   10K-query top-1000 batch on the 50M-doc index +
+                                          decode-only sweep over block sizes 64..512
+
+Each prints JSON lines (one per measurement).  Timing: CUDA events on the
+launching stream for device-side numbers, perf_counter for host-API latency.
+"""
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import paper_conf_ppopp_0044ws18_b200 as g  # noqa: E402
+from synth import make_pair_workload, make_workload  # noqa: E402
+
+
+def dev_batch(ix, ql, k):
+    nq = ql.num_queries
+    ix.griffin_reserve(ql.offsets, ql.terms, k)
+    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
+    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
+    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(nq, dtype=torch.int32, device="cuda")
+    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    st = torch.cuda.current_stream()
+
+    def run():
+        ix.griffin_query_batch_device(d_off, d_t, mt, k, keys, cnt, st)
+    return run
+
+
+def time_dev(run, iters=10, warmup=3):
+    for _ in range(warmup):
+        run()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(iters):
+        run()
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / iters
+
+
+def c1():
+    c, ql, cfg = make_workload("c1")
+    ix = g.GriffinIndex(c, block_size=128)
+    terms = ql.query(0)
+    for _ in range(200):
+        ix.griffin_query(terms, 10)
+    lat = []
+    for _ in range(10_000):
+        t0 = time.perf_counter()
+        ix.griffin_query(terms, 10)
+        lat.append((time.perf_counter() - t0) * 1e3)
+    lat.sort()
+    run = dev_batch(ix, ql, 10)
+    ms = time_dev(run, iters=200)
+    prof = None
+    print(json.dumps({"config": "c1", "metric": "single-query latency (griffin_query, host buffers)",
+                      "p50_ms": lat[len(lat) // 2], "p99_ms": lat[int(0.99 * len(lat)) - 1],
+                      "closed_loop_qps": 1e3 / (sum(lat) / len(lat)),
+                      "device_ms_per_query": ms, "df": [int(c.df()[t]) for t in terms]}),
+          flush=True)
+
+
+def c3():
+    groups = [(1, 16), (16, 32), (32, 64), (64, 128), (128, 256), (256, 512), (512, 1024),
+              (1000, 1001)]
+    rng = np.random.default_rng(0x6733)
+    per = 8
+    ratios, gid = [], []
+    for gi, (lo, hi) in enumerate(groups):
+        for _ in range(per):
+            ratios.append(float(np.exp(rng.uniform(np.log(lo), np.log(hi)))))
+            gid.append(gi)
+    c, ql = make_pair_workload(25_000_000, 1_500_000, ratios, seed=0x4752494646494E03)
+    ix = g.GriffinIndex(c, block_size=128)
+    ix.griffin_set_reuse(0)
+    for gi, (lo, hi) in enumerate(groups):
+        qs = [i for i in range(len(ratios)) if gid[i] == gi]
+        sub = ql.slice(qs[0], qs[-1] + 1)
+        res = {"config": "c3", "group": [lo, hi], "pairs": len(qs),
+               "S_len_mean": float(np.mean([c.df()[2 * i + 1] for i in qs])),
+               "R_len_mean": float(np.mean([c.df()[2 * i] for i in qs]))}
+        for name, mode in (("merge", g.MODE_MERGE), ("gallop", g.MODE_GALLOP),
+                           ("auto", g.MODE_AUTO)):
+            ix.griffin_set_mode(mode)
+            run = dev_batch(ix, sub, 10)
+            ix.griffin_reset_profile()
+            ix.griffin_set_profiling(True)
+            ms = time_dev(run, iters=5, warmup=2)
+            ix.griffin_set_profiling(False)
+            p = ix.griffin_get_profile()
+            res[name] = {"ms_per_pair": ms / len(qs),
+                         "payload_MB_per_pair": p["payload_bytes"] / 7 / len(qs) / 1e6,
+                         "decoded_postings_per_pair": p["decoded_postings"] / 7 / len(qs)}
+        res["winner"] = "merge" if res["merge"]["ms_per_pair"] <= res["gallop"]["ms_per_pair"] else "gallop"
+        print(json.dumps(res), flush=True)
+
+
+def c5(nq=None):
+    t0 = time.time()
+    c, ql, cfg = make_workload("c5", num_queries=nq)
+    gen_s = time.time() - t0
+    k = cfg["k"]
+    for B in (128, 64, 256, 512):
+        t0 = time.time()
+        ix = g.GriffinIndex(c, block_size=B)
+        build_s = time.time() - t0
+        st = ix.griffin_index_stats()
+        sw = ix.griffin_debug_decode_all(iters=3)
+        line = {"config": "c5", "block_size": B, "num_postings": c.num_postings,
+                "gen_s": gen_s, "build_s": build_s, "index_bytes": st["payload_bytes"] +
+                st["skip_bytes"] + st["tf_bytes"],
+                "decode_sweep": {"ms": sw["ms"], "gbs": sw["bytes"] / (sw["ms"] / 1e3) / 1e9,
+                                 "gpostings_per_s": sw["postings"] / (sw["ms"] / 1e3) / 1e9}}
+        if B == 128:
+            run = dev_batch(ix, ql, k)
+            ix.griffin_reset_profile()
+            ix.griffin_set_profiling(True)
+            ms = time_dev(run, iters=3, warmup=2)
+            ix.griffin_set_profiling(False)
+            p = ix.griffin_get_profile()
+            line.update({"queries": ql.num_queries, "k": k, "ms_per_batch": ms,
+                         "qps": ql.num_queries / (ms / 1e3),
+                         "stage_ms": {kk: p[kk] / 5 for kk in ("ms_plan", "ms_decode",
+                                                                 "ms_intersect", "ms_compact",
+                                                                 "ms_topk")}})
+        print(json.dumps(line), flush=True)
+        ix.close()
+
+
+if __name__ == "__main__":
+    which = sys.argv[1]
+    if which == "c1":
+        c1()
+    elif which == "c3":
+        c3()
+    elif which == "c5":
+        c5(int(sys.argv[2]) if len(sys.argv) > 2 else None)
