@@ -795,6 +795,62 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
         }
       }
       __syncwarp();
+      if (sdec) {
+        // S decoded in the arena: each R element binary-searches its touched
+        // block in place (no staging); a lane's elements are independent chains,
+        // so their probes overlap (log2(B) dependent steps per unit).
+        constexpr int kEpl = 4;   // elements per lane per 128-element slice
+        uint32_t probes = 0;
+        for (uint32_t base = 0; base < n; base += 128) {
+          uint32_t lo[kEpl], hi[kEpl], xv[kEpl], kb[kEpl];
+#pragma unroll
+          for (int j = 0; j < kEpl; ++j) {
+            const uint32_t e = base + lane + 32u * j;
+            lo[j] = 0;
+            hi[j] = 0;
+            xv[j] = 0;
+            kb[j] = kNone;
+            if (e < n) {
+              kb[j] = kidx[e];
+              if (kb[j] != kNone) {
+                hi[j] = min(B, tS.df_local - kb[j] * B);
+                xv[j] = tileR[e];
+              }
+            }
+          }
+          const uint32_t nb0 = hi[0], nb1 = hi[1], nb2 = hi[2], nb3 = hi[3];
+          for (;;) {
+            bool any = false;
+#pragma unroll
+            for (int j = 0; j < kEpl; ++j) {
+              if (lo[j] < hi[j]) {
+                const uint32_t mid = (lo[j] + hi[j]) >> 1;
+                if (__ldg(decS + (size_t)kb[j] * B + mid) < xv[j]) lo[j] = mid + 1; else hi[j] = mid;
+                any = true;
+                ++probes;
+              }
+            }
+            if (!__any_sync(0xffffffffu, any)) break;
+          }
+          const uint32_t nbs[kEpl] = {nb0, nb1, nb2, nb3};
+#pragma unroll
+          for (int j = 0; j < kEpl; ++j) {
+            const uint32_t e = base + lane + 32u * j;
+            if (kb[j] != kNone && lo[j] < nbs[j] &&
+                __ldg(decS + (size_t)kb[j] * B + lo[j]) == xv[j])
+              match[e] = kb[j] * B + lo[j];
+          }
+        }
+        const uint32_t sp = __reduce_add_sync(0xffffffffu, probes);
+        if (lane == 0) acc.alg += sp * 4ull;
+        __syncwarp();
+        if (RC)
+          emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
+        else
+          emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
+        __syncwarp();
+        continue;
+      }
       const uint32_t k_first = kidx[0];
       // distinct touched blocks (kidx is non-decreasing): dblk[], and kidx[e] :=
       // index of e's block in dblk (kNone if none)
