@@ -258,6 +258,7 @@ void griffin_index_destroy(griffin_index *ix) {
       b->release();
     if (w.h_pinned) cudaFreeHost(w.h_pinned);
     for (cudaEvent_t e : ix->ev_pool) cudaEventDestroy(e);
+    for (auto &g : ix->graphs) cudaGraphExecDestroy(g.exec);
     if (ix->stream) cudaStreamDestroy(ix->stream);
   }
   delete ix;
@@ -329,9 +330,116 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
   return GRIFFIN_OK;
 }
 
+// identity of the workspace buffers a captured graph points into
+static uint64_t ws_identity(const Workspace &w) {
+  uint64_t h = 1469598103934665603ull;
+  for (const DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel,
+                          &w.qmode, &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec,
+                          &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys,
+                          &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms})
+    h = (h ^ (uint64_t)(uintptr_t)b->p) * 1099511628211ull;
+  return h ^ (uint64_t)(uintptr_t)w.h_pinned;
+}
+
+// Single query through a cached CUDA graph: H2D of the terms, every kernel of
+// the path, D2H of the results and status, one graph launch (removes per-launch
+// CPU overhead from the latency path).  Workspace is pre-sized once for the
+// largest possible single query so captured addresses stay valid.
+static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint32_t nterms,
+                                  uint32_t k, uint32_t *out_docids, float *out_scores,
+                                  uint32_t *out_count) {
+  Workspace &w = ix->ws;
+  const uint32_t offs[2] = {0, nterms};
+  uint32_t mt = 1;
+  // validation + bounds (same rules as the batch path)
+  griffin_status s = reserve_for(ix, 1, offs, terms, k, &mt);
+  if (s) return s;
+  if (!ix->single_ws) {
+    uint64_t mx = 0, mb = 0;
+    for (const TermInfo &t : ix->h_terms) {
+      mx = std::max<uint64_t>(mx, t.df_local);
+      mb = std::max<uint64_t>(mb, t.nblocks);
+    }
+    if ((s = reserve_ws(ix, 1, 2 * mb + 1, mx + 1))) return s;
+    if ((s = reserve_topk(ix, 1, GRIFFIN_MAX_K))) return s;
+    if ((s = reserve_topk(ix, 1, 2048))) return s;   // the k with the most selection levels
+    GRIFFIN_CUDA_TRY(w.qoffs.reserve(8));
+    GRIFFIN_CUDA_TRY(w.qterms.reserve(GRIFFIN_MAX_TERMS * 4 * 4));
+    GRIFFIN_CUDA_TRY(w.keys.reserve(GRIFFIN_MAX_K * 8));
+    GRIFFIN_CUDA_TRY(w.counts.reserve(8));
+    GRIFFIN_CUDA_TRY(w.docids.reserve(GRIFFIN_MAX_K * 4));
+    GRIFFIN_CUDA_TRY(w.scores.reserve(GRIFFIN_MAX_K * 4));
+    if ((s = ensure_pinned(ix, 64 * 4 + GRIFFIN_MAX_K * 8 + 64))) return s;
+    ix->single_ws = true;
+  }
+  if (nterms > GRIFFIN_MAX_TERMS * 4) return GRIFFIN_ERR_UNSUPPORTED;  // caller falls back
+  // pinned layout: [qoffs 2][terms 64][status 2] then results
+  uint32_t *hp = static_cast<uint32_t *>(w.h_pinned);
+  uint32_t *h_off = hp, *h_terms = hp + 2, *h_status = hp + 66;
+  uint8_t *h_res = reinterpret_cast<uint8_t *>(hp + 68);
+  const uint64_t id = ws_identity(w);
+  cudaGraphExec_t exec = nullptr;
+  for (auto &g : ix->graphs)
+    if (g.mt == mt && g.k == k && g.mode == ix->mode && g.ws_id == id) exec = g.exec;
+  cudaStream_t st = ix->stream;
+  if (!exec) {
+    if (ix->graphs.size() >= 64) {
+      for (auto &g : ix->graphs) cudaGraphExecDestroy(g.exec);
+      ix->graphs.clear();
+    }
+    cudaGraph_t graph = nullptr;
+    GRIFFIN_CUDA_TRY(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+    cudaMemcpyAsync(w.qoffs.p, h_off, 8, cudaMemcpyHostToDevice, st);
+    cudaMemcpyAsync(w.qterms.p, h_terms, GRIFFIN_MAX_TERMS * 4 * 4, cudaMemcpyHostToDevice, st);
+    griffin_status rs = run_batch(ix, 1, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), mt, k,
+                                  w.keys.as<uint64_t>(), w.counts.as<uint32_t>(), st, true,
+                                  ix->mode);
+    if (!rs)
+      rs = launch_keys_to_results(ix, 1, k, w.keys.as<uint64_t>(), w.counts.as<uint32_t>(),
+                                  w.docids.as<uint32_t>(), w.scores.as<float>(), st);
+    cudaMemcpyAsync(h_res, w.docids.p, (size_t)k * 4, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(h_res + (size_t)k * 4, w.scores.p, (size_t)k * 4, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(h_res + (size_t)k * 8, w.counts.p, 4, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(h_status, w.scal.as<unsigned long long>() + kScalStatus, 4,
+                    cudaMemcpyDeviceToHost, st);
+    cudaError_t e = cudaStreamEndCapture(st, &graph);
+    if (rs || e != cudaSuccess) {
+      if (graph) cudaGraphDestroy(graph);
+      cudaGetLastError();
+      return GRIFFIN_ERR_UNSUPPORTED;  // caller falls back to the plain launches
+    }
+    e = cudaGraphInstantiate(&exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return GRIFFIN_ERR_UNSUPPORTED;
+    }
+    ix->graphs.push_back({mt, k, ix->mode, id, exec});
+  }
+  h_off[0] = 0;
+  h_off[1] = nterms;
+  std::memcpy(h_terms, terms, (size_t)nterms * 4);
+  GRIFFIN_CUDA_TRY(cudaGraphLaunch(exec, st));
+  GRIFFIN_CUDA_TRY(cudaStreamSynchronize(st));
+  if (*h_status) {
+    if ((s = read_status(ix))) return s;   // clears the device flag
+  }
+  std::memcpy(out_docids, h_res, (size_t)k * 4);
+  std::memcpy(out_scores, h_res + (size_t)k * 4, (size_t)k * 4);
+  std::memcpy(out_count, h_res + (size_t)k * 8, 4);
+  return GRIFFIN_OK;
+}
+
 griffin_status griffin_query(griffin_index *ix, const uint32_t *terms, uint32_t nterms, uint32_t k,
                              uint32_t *out_docids, float *out_scores, uint32_t *out_count) {
   if (nterms == 0) return invalid("nterms must be > 0");
+  if (!ix || !terms || !out_docids || !out_scores || !out_count) return invalid("null argument");
+  if (ix->use_graphs && !ix->profiling) {
+    std::lock_guard<std::mutex> lk(ix->mu);
+    DeviceGuard guard(ix->device);
+    griffin_status s = query_graph(ix, terms, nterms, k, out_docids, out_scores, out_count);
+    if (s != GRIFFIN_ERR_UNSUPPORTED) return s;
+  }
   const uint32_t offs[2] = {0, nterms};
   return griffin_query_batch(ix, 1, offs, terms, k, out_docids, out_scores, out_count);
 }

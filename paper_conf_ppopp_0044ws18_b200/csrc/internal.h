@@ -125,6 +125,16 @@ struct griffin_index {
   griffin::Workspace ws;
   int mode = 0;
   int reuse = 2;
+  // single-query CUDA graphs, keyed by (distinct terms, k, mode, workspace identity)
+  struct QueryGraph {
+    uint32_t mt, k;
+    int mode;
+    uint64_t ws_id;
+    cudaGraphExec_t exec;
+  };
+  std::vector<QueryGraph> graphs;
+  bool single_ws = false;
+  int use_graphs = 1;
   bool profiling = false;
   griffin_profile prof{};
   std::vector<cudaEvent_t> ev_pool;
@@ -161,6 +171,7 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
                          uint64_t *d_keys, uint32_t *d_counts, cudaStream_t st, bool final_topk,
                          int forced_mode);
 griffin_status reserve_ws(griffin_index *ix, uint32_t nq, uint64_t units, uint64_t entries);
+griffin_status reserve_topk(griffin_index *ix, uint32_t nq, uint32_t k);
 griffin_status launch_merge_topk(griffin_index *ix, uint32_t G, uint32_t nq, uint32_t k,
                                  const uint64_t *d_keys, const uint32_t *d_counts,
                                  uint64_t *d_out_keys, uint32_t *d_out_counts, cudaStream_t st);

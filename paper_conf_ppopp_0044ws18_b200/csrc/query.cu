@@ -1577,6 +1577,17 @@ static cudaError_t launch_intersect(griffin_index *ix, const RoundArgs &ra, cuda
   return cudaGetLastError();
 }
 
+// Top-k candidate buffers for a batch of nq queries with this k (grow-only;
+// called before a CUDA-graph capture so no allocation happens inside it).
+griffin_status reserve_topk(griffin_index *ix, uint32_t nq, uint32_t k) {
+  Workspace &w = ix->ws;
+  const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
+  const int levels = k <= 64 ? 2 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
+  GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8 * std::max(levels, 1)));
+  GRIFFIN_CUDA_TRY(w.tkstate.reserve(((size_t)nq + 1) * (1 + 8 + 4) + 64));
+  return GRIFFIN_OK;
+}
+
 griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs,
                          const uint32_t *d_terms, uint32_t max_terms, uint32_t k, uint64_t *d_keys,
                          uint32_t *d_counts, cudaStream_t st, bool final_topk, int forced_mode) {
@@ -1710,8 +1721,8 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
     // by kTopkSmem / k; small k needs 2 levels, large k up to kTopkMaxLevels)
     const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
     const int levels = k <= 64 ? 2 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
-    GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8 * std::max(levels, 1)));
-    GRIFFIN_CUDA_TRY(w.tkstate.reserve(((size_t)nq + 1) * (1 + 8 + 4) + 64));
+    griffin_status rs_ = reserve_topk(ix, nq, k);
+    if (rs_) return rs_;
     CandBufs cb{};
     for (int L = 1; L <= levels; ++L) cb.lv[L] = w.cand.as<uint64_t>() + (size_t)(L - 1) * cand_cap;
     TopkState ts;
