@@ -81,6 +81,10 @@ typedef struct {
   int32_t device;        /* CUDA device ordinal to build on; < 0 -> current device */
   uint32_t shard_index;  /* docID-range shard g of num_shards */
   uint32_t num_shards;   /* 0 or 1 -> unsharded */
+  uint32_t gallop_ratio_decoded; /* T for rounds whose S list was decoded once into the batch
+                                    arena (griffin_set_reuse): galloping there costs ~log2(B)
+                                    probes per R element instead of a block decode, so the
+                                    crossover is lower; 0 -> max(4, block_size/8) */
 } griffin_build_opts;
 
 typedef struct {

@@ -46,7 +46,7 @@ class _Opts(ctypes.Structure):
     _fields_ = [("block_size", ctypes.c_uint32), ("bm25_k1", ctypes.c_double),
                 ("bm25_b", ctypes.c_double), ("gallop_ratio", ctypes.c_uint32),
                 ("device", ctypes.c_int32), ("shard_index", ctypes.c_uint32),
-                ("num_shards", ctypes.c_uint32)]
+                ("num_shards", ctypes.c_uint32), ("gallop_ratio_decoded", ctypes.c_uint32)]
 
 
 class Stats(ctypes.Structure):
@@ -163,7 +163,7 @@ class GriffinIndex:
 
     def __init__(self, corpus, block_size: int = 128, k1: float = 1.2, b: float = 0.75,
                  gallop_ratio: int = 0, device: int = -1, shard_index: int = 0,
-                 num_shards: int = 1):
+                 num_shards: int = 1, gallop_ratio_decoded: int = 0):
         lib = load_library()
         self._arrays = [np.ascontiguousarray(corpus.offsets, np.uint64),
                         np.ascontiguousarray(corpus.docids, np.uint32),
@@ -172,7 +172,8 @@ class GriffinIndex:
         off, doc, tf, dl = self._arrays
         c = _Corpus(corpus.num_docs, len(off) - 1, off.ctypes.data, doc.ctypes.data,
                     tf.ctypes.data, dl.ctypes.data)
-        o = _Opts(block_size, k1, b, gallop_ratio, device, shard_index, num_shards)
+        o = _Opts(block_size, k1, b, gallop_ratio, device, shard_index, num_shards,
+                  gallop_ratio_decoded)
         h = ctypes.c_void_p()
         status = lib.griffin_index_build(ctypes.byref(c), ctypes.byref(o), ctypes.byref(h))
         self._arrays = None

@@ -175,6 +175,7 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   ix->device = dev;
   ix->B = B;
   ix->T = opts.gallop_ratio ? opts.gallop_ratio : B;
+  ix->Tdec = opts.gallop_ratio_decoded ? opts.gallop_ratio_decoded : std::max<uint32_t>(4, B / 8);
   ix->D = std::max<uint32_t>(2, 1024 / B);
   ix->k1 = k1;
   ix->bm25_b = bb;

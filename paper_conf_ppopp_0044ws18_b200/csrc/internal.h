@@ -78,7 +78,7 @@ enum : int {
 };
 
 struct RoundArgs {
-  uint32_t nq, round, D, T;
+  uint32_t nq, round, D, T, Tdec;
   int forced_mode;
   const uint32_t *plan_terms;
   const uint32_t *plan_m;
@@ -108,7 +108,7 @@ struct griffin_index {
   int device = 0;
   cudaStream_t stream = nullptr;
   // options
-  uint32_t B = 128, T = 128, D = 8;
+  uint32_t B = 128, T = 128, Tdec = 16, D = 8;
   double k1 = 1.2, bm25_b = 0.75;
   uint32_t shard = 0, nshards = 1, doc_base = 0, doc_end = 0, N = 0, V = 0;
   float k1p1 = 0.f;

@@ -152,9 +152,13 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
       pair = true;
     }
     if (pair) {
-      const TermInfo tS = ix.terms[a.plan_terms[q * kMaxTerms + a.round]];
+      const uint32_t sid = a.plan_terms[q * kMaxTerms + a.round];
+      const TermInfo tS = ix.terms[sid];
+      // crossover: T for compressed S (gallop decodes one block per
+      // touched block), Tdec when S sits decoded in the batch arena
+      const uint64_t T = (a.tdec && a.tdec[sid]) ? a.Tdec : a.T;
       const bool gallop = a.forced_mode == 2 ||
-                          (a.forced_mode == 0 && (uint64_t)tS.df_local > (uint64_t)a.T * nR);
+                          (a.forced_mode == 0 && (uint64_t)tS.df_local > T * nR);
       mode = gallop ? kModeGallop : kModeMerge;
       units = gallop ? nbR : (nbR + tS.nblocks + a.D - 1) / a.D;
     }
@@ -455,6 +459,26 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
     const uint32_t q = lo;
     const uint32_t lu = (uint32_t)(u - a.unit_base[q]);
     uint4 rec = make_uint4(q, lu, 0, 0);
+    if (a.qmode[q] == kModeGallop) {
+      // skip-pointer range the R chunk can touch: [upper_bound(first elem) - 1,
+      // upper_bound(last elem)); for a compressed R block the next block's head
+      // bounds its last element
+      const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
+      const TermInfo tR = ix.terms[pt[0]];
+      const TermInfo tS = ix.terms[pt[a.round]];
+      uint32_t x0, x1;
+      if (RC) {
+        x0 = __ldg(ix.first + tR.block0 + lu);
+        x1 = lu + 1 < tR.nblocks ? __ldg(ix.first + tR.block0 + lu + 1) - 1u : 0xFFFFFFFFu;
+      } else {
+        const uint2 *Rq = a.rprev + a.cap_off[q];
+        const uint32_t s0 = lu * ix.B, s1 = min(s0 + ix.B, a.rcount[q]);
+        x0 = Rq[s0].x;
+        x1 = Rq[s1 - 1].x;
+      }
+      rec.z = upper_bound_g(ix.first + tS.block0, 0, tS.nblocks, x0);
+      rec.w = upper_bound_g(ix.first + tS.block0, rec.z, tS.nblocks, x1);
+    }
     if (a.qmode[q] == kModeMerge) {
       const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
       const TermInfo tR = ix.terms[pt[0]];
@@ -768,8 +792,7 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
         if (lane == 0) acc.alg += n * 8u;
       }
       __syncwarp();
-      uint32_t k_lo, k_hi;
-      warp_upper_bound2(fS, nbS, tileR[0], tileR[n - 1], &k_lo, &k_hi);
+      const uint32_t k_lo = rec.z, k_hi = rec.w;   // from the partition stage
       // skip pointers the chunk can touch: [k_lo-1, k_hi); stage them in smem when
       // they fit (one round trip), else search them in global memory
       const uint32_t w0 = k_lo ? k_lo - 1u : 0u, span = k_hi - w0;
@@ -1605,6 +1628,7 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
   ra.nq = nq;
   ra.D = ix->D;
   ra.T = ix->T;
+  ra.Tdec = ix->Tdec;
   ra.forced_mode = forced_mode;
   ra.plan_terms = w.plan_terms.as<uint32_t>();
   ra.plan_m = w.plan_m.as<uint32_t>();
