@@ -371,20 +371,39 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
   }
   if (cnt) {
     uint2 *dst = a.bump + off + (incl - c);
-    for (uint32_t j = 0; j < c; ++j) {
-      const uint32_t e = ml[j];
-      const uint32_t i = e & 0xFFFFu;
-      const uint32_t doc = tile[i];
-      const float nrm = __ldg(ix.norm + doc);
-      const float wS = bm25_w(tS.idf, tf_lookup(ix, tS, posS0 + (e >> 16)), nrm, ix.k1p1);
-      float s;
-      if (RC) {
-        s = bm25_w(tR.idf, tf_lookup(ix, tR, posR0 + i), nrm, ix.k1p1);  // first term: s = w
-        s = __fadd_rn(s, wS);
-      } else {
-        s = __fadd_rn(__uint_as_float(Rq[posR0 + i].y), wS);
+    // gathers (norm, tf words, previous score) of up to 4 matches are issued
+    // together before any is consumed, so their latencies overlap
+    for (uint32_t j0 = 0; j0 < c; j0 += 4) {
+      uint32_t doc[4], tS_[4], tR_[4], prev[4];
+      float nrm[4];
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        const uint32_t j = j0 + t;
+        if (j < c) {
+          const uint32_t e = ml[j];
+          const uint32_t i = e & 0xFFFFu;
+          doc[t] = tile[i];
+          nrm[t] = __ldg(ix.norm + doc[t]);
+          tS_[t] = tf_lookup(ix, tS, posS0 + (e >> 16));
+          if (RC) tR_[t] = tf_lookup(ix, tR, posR0 + i);
+          else prev[t] = Rq[posR0 + i].y;
+        }
       }
-      dst[j] = make_uint2(doc, __float_as_uint(s));
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        const uint32_t j = j0 + t;
+        if (j < c) {
+          const float wS = bm25_w(tS.idf, tS_[t], nrm[t], ix.k1p1);
+          float s;
+          if (RC) {
+            s = bm25_w(tR.idf, tR_[t], nrm[t], ix.k1p1);  // first term: s = w
+            s = __fadd_rn(s, wS);
+          } else {
+            s = __fadd_rn(__uint_as_float(prev[t]), wS);
+          }
+          dst[j] = make_uint2(doc[t], __float_as_uint(s));
+        }
+      }
     }
   }
   if (lane == 0) {
@@ -812,9 +831,37 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
           match[e] = kNone;
         }
       } else {
-        for (uint32_t e = lane; e < n; e += 32) {
-          kidx[e] = upper_bound_g(fS, k_lo, k_hi, tileR[e]) - 1u;
-          match[e] = kNone;
+        // wide range: the lane's elements search the skip pointers in global
+        // memory as independent interleaved chains (one round trip per step)
+        for (uint32_t base = 0; base < n; base += 128) {
+          uint32_t lo[4], hi[4], xv[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const uint32_t e = base + lane + 32u * j;
+            lo[j] = k_lo;
+            hi[j] = e < n ? k_hi : k_lo;
+            xv[j] = e < n ? tileR[e] : 0u;
+          }
+          for (;;) {
+            bool any = false;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              if (lo[j] < hi[j]) {
+                const uint32_t mid = (lo[j] + hi[j]) >> 1;
+                if (__ldg(fS + mid) <= xv[j]) lo[j] = mid + 1; else hi[j] = mid;
+                any = true;
+              }
+            }
+            if (!__any_sync(0xffffffffu, any)) break;
+          }
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const uint32_t e = base + lane + 32u * j;
+            if (e < n) {
+              kidx[e] = lo[j] - 1u;   // kNone: below S's first docID
+              match[e] = kNone;
+            }
+          }
         }
       }
       __syncwarp();
