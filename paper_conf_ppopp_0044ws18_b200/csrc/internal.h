@@ -27,7 +27,7 @@ void set_error(const std::string &msg);
 enum : int { kStatusBadTerm = 1, kStatusOverflow = 2, kStatusTooManyTerms = 4 };
 
 // Query modes per (query, round).
-enum : uint32_t { kModeNone = 0, kModeMerge = 1, kModeGallop = 2, kModeAll = 3 };
+enum : uint32_t { kModeNone = 0, kModeMerge = 1, kModeGallop = 2, kModeAll = 3, kModeProbe = 4 };
 
 // Grow-only device buffer.
 struct DevBuf {
@@ -80,6 +80,7 @@ enum : int {
 struct RoundArgs {
   uint32_t nq, round, D, T, Tdec;
   int forced_mode;
+  int probe;
   const uint32_t *plan_terms;
   const uint32_t *plan_m;
   const uint32_t *cap;
@@ -135,6 +136,7 @@ struct griffin_index {
   std::vector<QueryGraph> graphs;
   bool single_ws = false;
   int use_graphs = 1;
+  int probe = 1;
   bool profiling = false;
   griffin_profile prof{};
   std::vector<cudaEvent_t> ev_pool;

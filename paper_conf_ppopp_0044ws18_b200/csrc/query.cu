@@ -149,7 +149,12 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
     } else if (m > a.round && a.rcount[q] > 0) {
       nR = a.rcount[q];
       nbR = (uint32_t)((nR + ix.B - 1) / ix.B);
-      pair = true;
+      if (a.probe) {   // rounds 2..m-1 as one multi-list probe pass
+        mode = kModeProbe;
+        units = nbR;
+      } else {
+        pair = true;
+      }
     }
     if (pair) {
       const uint32_t sid = a.plan_terms[q * kMaxTerms + a.round];
@@ -557,6 +562,233 @@ __device__ __forceinline__ void warp_upper_bound2(const uint32_t *__restrict__ a
   *r1 = __shfl_sync(0xffffffffu, lo, 16);
 }
 
+// Multi-list probe (SvS rounds 2..m-1 in one pass): every round-1 survivor is
+// looked up in each remaining list in canonical order — skip-pointer search,
+// then an in-place binary search of the decoded-arena block or a staged EF
+// decode of the touched compressed blocks — its BM25 contribution added
+// (s = s + w_t, SURVEY O6 order), and dropped at the first list that misses it.
+// The surviving set equals SvS's; only the loop order differs.
+__device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm, uint64_t u,
+                           uint32_t q, uint32_t lu, Acc &acc) {
+  const uint32_t lane = lane_id(), lt = lanemask_lt();
+  const uint32_t B = ix.B, D = a.D;
+  const uint32_t G = min(D - 3u, 31u);
+  const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
+  const uint32_t m = a.plan_m[q];
+  const uint2 *Rq = a.rprev + a.cap_off[q];
+  const uint32_t nR = a.rcount[q];
+  uint32_t *tileR = sm.tile, *sc = sm.tile + B, *nrm = sm.tile + 2 * B, *kidx = sm.tile + 3 * B;
+  uint32_t *match = sm.tile + 4 * B, *tileS = sm.tile + 5 * B;
+  uint32_t *dblk = sm.aux, *sn = sm.aux + B;
+  const uint32_t s0 = lu * B;
+  uint32_t n = min(B, nR - s0);
+  for (uint32_t e = lane; e < n; e += 32) {
+    const uint2 v = Rq[s0 + e];
+    tileR[e] = v.x;
+    sc[e] = v.y;
+    nrm[e] = __float_as_uint(__ldg(ix.norm + v.x));
+  }
+  __syncwarp();
+  if (lane == 0) acc.alg += n * 12u;
+  for (uint32_t r = 2; r < m && n > 0; ++r) {
+    const uint32_t sid = pt[r];
+    const TermInfo tS = ix.terms[sid];
+    const uint32_t *fS = ix.first + tS.block0;
+    const bool sdec = a.tdec && a.tdec[sid];
+    const uint32_t *decS = sdec ? a.dec + (size_t)tS.block0 * B : nullptr;
+    uint32_t k_lo, k_hi;
+    warp_upper_bound2(fS, tS.nblocks, tileR[0], tileR[n - 1], &k_lo, &k_hi);
+    // ---- skip-pointer block of every element: interleaved chains ----
+    for (uint32_t base = 0; base < n; base += 128) {
+      uint32_t lo[4], hi[4], xv[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t e = base + lane + 32u * j;
+        lo[j] = k_lo;
+        hi[j] = e < n ? k_hi : k_lo;
+        xv[j] = e < n ? tileR[e] : 0u;
+      }
+      for (;;) {
+        bool any = false;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          if (lo[j] < hi[j]) {
+            const uint32_t mid = (lo[j] + hi[j]) >> 1;
+            if (__ldg(fS + mid) <= xv[j]) lo[j] = mid + 1; else hi[j] = mid;
+            any = true;
+          }
+        }
+        if (!__any_sync(0xffffffffu, any)) break;
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t e = base + lane + 32u * j;
+        if (e < n) {
+          kidx[e] = lo[j] - 1u;
+          match[e] = kNone;
+        }
+      }
+    }
+    __syncwarp();
+    if (sdec) {
+      // ---- decoded arena: in-place binary search of the touched block ----
+      uint32_t probes = 0;
+      for (uint32_t base = 0; base < n; base += 128) {
+        uint32_t lo[4], hi[4], xv[4], kb[4], nb[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const uint32_t e = base + lane + 32u * j;
+          lo[j] = 0;
+          hi[j] = 0;
+          xv[j] = 0;
+          kb[j] = kNone;
+          nb[j] = 0;
+          if (e < n) {
+            kb[j] = kidx[e];
+            if (kb[j] != kNone) {
+              nb[j] = min(B, tS.df_local - kb[j] * B);
+              hi[j] = nb[j];
+              xv[j] = tileR[e];
+            }
+          }
+        }
+        for (;;) {
+          bool any = false;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            if (lo[j] < hi[j]) {
+              const uint32_t mid = (lo[j] + hi[j]) >> 1;
+              if (__ldg(decS + (size_t)kb[j] * B + mid) < xv[j]) lo[j] = mid + 1; else hi[j] = mid;
+              any = true;
+              ++probes;
+            }
+          }
+          if (!__any_sync(0xffffffffu, any)) break;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const uint32_t e = base + lane + 32u * j;
+          if (kb[j] != kNone && lo[j] < nb[j] && __ldg(decS + (size_t)kb[j] * B + lo[j]) == xv[j])
+            match[e] = kb[j] * B + lo[j];
+        }
+      }
+      const uint32_t sp = __reduce_add_sync(0xffffffffu, probes);
+      if (lane == 0) acc.alg += sp * 4ull;
+    } else {
+      // ---- compressed: distinct touched blocks, staged + decoded in groups ----
+      uint32_t nd = 0, prev = kNone, e_first = n;
+      for (uint32_t c0 = 0; c0 < n; c0 += 32) {
+        const uint32_t e = c0 + lane;
+        const uint32_t kv = e < n ? kidx[e] : kNone;
+        uint32_t kp = __shfl_up_sync(0xffffffffu, kv, 1);
+        if (lane == 0) kp = prev;
+        const bool newb = e < n && kv != kNone && kv != kp;
+        const uint32_t bal = __ballot_sync(0xffffffffu, newb);
+        if (newb) dblk[nd + __popc(bal & lt)] = kv;
+        const uint32_t gi = nd + __popc(bal & (lt | (1u << lane))) - 1u;
+        if (e < n) kidx[e] = kv == kNone ? kNone : gi;
+        const uint32_t valid = __ballot_sync(0xffffffffu, e < n && kv != kNone);
+        if (e_first == n && valid) e_first = c0 + __ffs(valid) - 1u;
+        nd += __popc(bal);
+        prev = __shfl_sync(0xffffffffu, kv, 31);
+      }
+      __syncwarp();
+      uint32_t ep = e_first;
+      const uint32_t cap16 = stage_words(B, D) / 4u;
+      for (uint32_t g0 = 0; g0 < nd;) {
+        uint32_t ng = min(G, nd - g0);
+        uint2 mm = make_uint2(0, 0);
+        uint32_t f = 0, sz = 0, blk = 0, nn = 0;
+        if (lane < ng) {
+          blk = dblk[g0 + lane];
+          nn = min(B, tS.df_local - blk * B);
+          mm = ix.meta[(uint64_t)tS.block0 + blk];
+          f = ix.first[(uint64_t)tS.block0 + blk];
+          sz = block_size16(mm.y);
+        }
+        const uint32_t inc = warp_incl_scan(sz);
+        const uint32_t nfit = __popc(__ballot_sync(0xffffffffu, lane < ng && inc <= cap16));
+        ng = nfit ? nfit : 1u;
+        if (lane >= ng) sz = 0;
+        if (lane < ng) sn[lane] = nn;
+        const uint32_t pay = __reduce_add_sync(0xffffffffu, lane < ng ? sz * 16u : 0u);
+        const uint32_t pst = __reduce_add_sync(0xffffffffu, lane < ng ? nn : 0u);
+        if (lane == 0) {
+          acc.pay += pay;
+          acc.post += pst;
+          acc.alg += pay + 8u * ng;
+        }
+        const uint32_t soff = warp_incl_scan(sz) - sz;
+        stage_blocks(ix, sm, ng, mm, soff, sz, false);
+        for (uint32_t i = 0; i < ng; ++i) {
+          const uint32_t y = __shfl_sync(0xffffffffu, mm.y, i);
+          const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
+          const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
+          warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+        }
+        __syncwarp();
+        for (;;) {
+          const uint32_t e = ep + lane;
+          const uint32_t gi = e < n ? kidx[e] : kNone;
+          const bool in = gi != kNone && gi < g0 + ng;
+          if (in) {
+            const uint32_t x = tileR[e];
+            const uint32_t *seg = tileS + (gi - g0) * B;
+            const uint32_t p = lower_bound_s(seg, 0, sn[gi - g0], x);
+            if (p < sn[gi - g0] && seg[p] == x) match[e] = dblk[gi] * B + p;
+          }
+          const uint32_t bal = __ballot_sync(0xffffffffu, in);
+          ep += __popc(bal);
+          if (bal != 0xffffffffu) break;
+        }
+        __syncwarp();
+        g0 += ng;
+      }
+    }
+    __syncwarp();
+    // ---- add w_t to the members, drop the rest (stable in-place compaction) ----
+    uint32_t nn2 = 0;
+    for (uint32_t c0 = 0; c0 < n; c0 += 32) {
+      const uint32_t e = c0 + lane;
+      const bool in = e < n;
+      const uint32_t x = in ? tileR[e] : 0u, mt = in ? match[e] : kNone;
+      const uint32_t nm = in ? nrm[e] : 0u;
+      float s = in ? __uint_as_float(sc[e]) : 0.f;
+      const bool keep = in && mt != kNone;
+      if (keep) s = __fadd_rn(s, bm25_w(tS.idf, tf_lookup(ix, tS, mt), __uint_as_float(nm), ix.k1p1));
+      const uint32_t bal = __ballot_sync(0xffffffffu, keep);
+      __syncwarp();
+      if (keep) {
+        const uint32_t pos = nn2 + __popc(bal & lt);
+        tileR[pos] = x;
+        sc[pos] = __float_as_uint(s);
+        nrm[pos] = nm;
+      }
+      nn2 += __popc(bal);
+      __syncwarp();
+    }
+    n = nn2;
+    if (lane == 0) acc.alg += n * 4u;
+  }
+  // ---- emit the survivors ----
+  unsigned long long off = 0;
+  uint32_t cnt = n;
+  if (lane == 0 && cnt) off = atomicAdd(a.scal + kScalBump, (unsigned long long)cnt);
+  off = __shfl_sync(0xffffffffu, off, 0);
+  if (off + cnt > a.entry_cap) {
+    if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
+    cnt = 0;
+  }
+  for (uint32_t e = lane; e < cnt; e += 32) a.bump[off + e] = make_uint2(tileR[e], sc[e]);
+  if (lane == 0) {
+    a.unit_off[u] = off;
+    a.unit_cnt[u] = cnt;
+    acc.surv += cnt;
+    acc.alg += cnt * 8ull;
+  }
+  __syncwarp();
+}
+
 template <bool RC>
 __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevIndex ix, RoundArgs a) {
   extern __shared__ uint4 smem4[];
@@ -610,6 +842,10 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
         }
       }
       emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, 0, n, lu * B, acc);
+      continue;
+    }
+    if (!RC && mode == kModeProbe) {
+      probe_unit(ix, a, sm, u, q, lu, acc);
       continue;
     }
     const uint32_t tSid = pt[a.round];
@@ -1745,7 +1981,10 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
     ra.dec = w.arena.as<uint32_t>();
     ra.tdec = w.tdec.as<uint8_t>();
   }
-  const uint32_t rounds = std::max<uint32_t>(1, max_terms > 0 ? max_terms - 1 : 1);
+  // multi-list probe replaces SvS rounds 2..m-1 (auto mode, B small enough for its smem)
+  ra.probe = forced_mode == 0 && ix->probe && ix->D >= 5;
+  uint32_t rounds = std::max<uint32_t>(1, max_terms > 0 ? max_terms - 1 : 1);
+  if (ra.probe) rounds = std::min<uint32_t>(rounds, 2);
   for (uint32_t r = 1; r <= rounds; ++r) {
     ra.round = r;
     ra.rprev = (r & 1) ? w.rbuf0.as<uint2>() : w.rbuf1.as<uint2>();
