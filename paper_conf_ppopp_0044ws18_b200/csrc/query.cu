@@ -800,8 +800,15 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
   const uint32_t G = min(D - 1u, 31u);   // gallop: S blocks staged per group
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   Acc acc;
-  for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); u < total;
-       u += nwarps) {
+  // dynamic unit tickets (balances long gallop/probe units); the next ticket is
+  // requested at the start of a unit so its latency overlaps the unit's work
+  unsigned long long ticket = 0;
+  if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
+  (void)nwarps;
+  for (;;) {
+    const uint64_t u = __shfl_sync(0xffffffffu, ticket, 0);
+    if (u >= total) break;
+    if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
     const uint4 rec = a.urec[u];
     const uint4 nxt = a.urec[u + 1];
     const uint32_t q = rec.x;
