@@ -48,49 +48,75 @@ def _peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    """SM clock + throttle reasons sampled during the timed region: NVML in a
+    background thread every 2 ms (the timed region can be tens of ms), with
+    nvidia-smi as a fallback."""
 
     def __init__(self, gpu_index: int):
         self.gpu = gpu_index
-        self.p = None
+        self.samples = []
+        self.max_mhz = 0.0
+        self.reasons = set()
+        self._stop = None
+        self._th = None
+        self._nvml = None
 
     def start(self):
+        import threading
         try:
-            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
-                                       "--format=csv,noheader,nounits", "-lms", "100"],
-                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-        except OSError:
-            self.p = None
+            import pynvml as nv
+            nv.nvmlInit()
+            h = nv.nvmlDeviceGetHandleByIndex(self.gpu)
+            self.max_mhz = float(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM))
+            self._nvml = (nv, h)
+        except Exception:
+            self._nvml = None
+        self._stop = threading.Event()
+        self._th = threading.Thread(target=self._run, daemon=True)
+        self._th.start()
+
+    def _run(self):
+        names = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+                 "sw_power_cap": 0x4}
+        while not self._stop.is_set():
+            if self._nvml:
+                nv, h = self._nvml
+                try:
+                    self.samples.append(float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)))
+                    fn = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                        nv.nvmlDeviceGetCurrentClocksThrottleReasons
+                    r = fn(h)
+                    for nm, bit in names.items():
+                        if r & bit:
+                            self.reasons.add(nm)
+                except Exception:
+                    pass
+                self._stop.wait(0.002)
+            else:
+                try:
+                    out = subprocess.run(["nvidia-smi", "-i", str(self.gpu),
+                                          "--query-gpu=clocks.sm,clocks.max.sm",
+                                          "--format=csv,noheader,nounits"],
+                                         capture_output=True, text=True, timeout=5).stdout
+                    a, b = out.strip().split(",")[:2]
+                    self.samples.append(float(a))
+                    self.max_mhz = max(self.max_mhz, float(b))
+                except Exception:
+                    pass
+                self._stop.wait(0.05)
 
     def stop(self):
-        if self.p is None:
+        if self._th is None:
             return None
-        self.p.terminate()
-        try:
-            out, _ = self.p.communicate(timeout=5)
-        except subprocess.TimeoutExpired:
-            self.p.kill()
-            out, _ = self.p.communicate()
-        rows = [r.split(",") for r in out.strip().splitlines() if r.strip()]
-        sm, mx, reasons = [], 0.0, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in rows:
-            try:
-                sm.append(float(r[1]))
-                mx = max(mx, float(r[2]))
-                for nm, v in zip(names, r[5:9]):
-                    if v.strip().lower() == "active":
-                        reasons.add(nm)
-            except (ValueError, IndexError):
-                continue
-        if not sm:
+        self._stop.set()
+        self._th.join(timeout=5)
+        if not self.samples:
             return None
-        loaded = [s for s in sm if s > 0.5 * mx] or sm
-        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": mx, "reasons": sorted(reasons),
-                "samples": len(sm)}
+        mx = self.max_mhz or max(self.samples)
+        loaded = [x for x in self.samples if x > 0.5 * mx] or self.samples
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": mx,
+                "reasons": sorted(self.reasons), "samples": len(self.samples),
+                "source": "nvml" if self._nvml else "nvidia-smi"}
 
 
 def _cpu_info():
@@ -208,13 +234,12 @@ def run_gpu(args):
     ix.griffin_reset_profile()
     ix.griffin_set_profiling(True)
     clocks = ClockSampler(dev)
-    clocks.start()
-    time.sleep(0.3)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(args.steps)]
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
+    clocks.start()
     for i in range(args.steps):
         flush.fill_(i)                       # L2 flush between timed steps (outside events)
         ev[i][0].record(stream)
@@ -297,6 +322,8 @@ def run_gpu(args):
     # ---- closed-loop single-query latency (griffin_query, one in flight)
     lat = []
     nlat = min(nq, args.latency_queries)
+    for q in range(min(nlat, 64)):          # warm-up: capture the per-term-count graphs
+        ix.griffin_query(ql.query(q), k)
     for q in range(nlat):
         t0 = time.perf_counter()
         ix.griffin_query(ql.query(q), k)
