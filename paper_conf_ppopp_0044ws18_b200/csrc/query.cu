@@ -1895,7 +1895,7 @@ static cudaError_t launch_intersect(griffin_index *ix, const RoundArgs &ra, cuda
 griffin_status reserve_topk(griffin_index *ix, uint32_t nq, uint32_t k) {
   Workspace &w = ix->ws;
   const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
-  const int levels = k <= 64 ? 2 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
+  const int levels = k <= 64 ? 1 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
   GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8 * std::max(levels, 1)));
   GRIFFIN_CUDA_TRY(w.tkstate.reserve(((size_t)nq + 1) * (1 + 8 + 4) + 64));
   return GRIFFIN_OK;
@@ -2037,7 +2037,7 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
     // candidates per level <= (entries / kTopkSmem + nq + 1) * k (each level shrinks them
     // by kTopkSmem / k; small k needs 2 levels, large k up to kTopkMaxLevels)
     const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
-    const int levels = k <= 64 ? 2 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
+    const int levels = k <= 64 ? 1 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
     griffin_status rs_ = reserve_topk(ix, nq, k);
     if (rs_) return rs_;
     CandBufs cb{};
