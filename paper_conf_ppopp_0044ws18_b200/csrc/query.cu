@@ -1393,6 +1393,7 @@ struct SelectSmem {
 __device__ __forceinline__ void select_digit(SelectSmem &ss, int shift) {
   if (threadIdx.x < 32) {
     const uint32_t lane = threadIdx.x;
+    const uint32_t need = ss.need;   // read by every lane before any lane updates it
     uint32_t loc[8], s = 0;
 #pragma unroll
     for (int i = 0; i < 8; ++i) {  // lane l owns bins 255-8l .. 248-8l (descending)
@@ -1400,7 +1401,7 @@ __device__ __forceinline__ void select_digit(SelectSmem &ss, int shift) {
       s += loc[i];
     }
     const uint32_t incl = warp_incl_scan(s);
-    const uint32_t need = ss.need;
+    __syncwarp();
     const uint32_t excl = incl - s;
     if (excl < need && need <= incl) {
       uint32_t cum = excl;

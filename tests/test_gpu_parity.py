@@ -351,3 +351,19 @@ def test_multilevel_topk_large_results(k):
     od, os_, oc = ox.query_batch(ql, k)
     gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
     assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+def test_single_query_graph_path_reuse_and_recapture(tiny):
+    """griffin_query replays cached CUDA graphs keyed by (distinct terms, k): many
+    different queries, repeated, interleaved with a batch call that grows the
+    workspace (forcing re-capture), all bit-exact."""
+    c, ql, ox = tiny
+    gx = g.GriffinIndex(c, block_size=128)
+    for rep in range(2):
+        for q in range(ql.num_queries):
+            for k in (1, 10):
+                od, os_, oc = ox.query(ql.query(q), k)
+                gd, gs, gc = gx.griffin_query(ql.query(q), k)
+                assert_topk_equal(gd, gs, gc, od, os_, oc)
+        # a batch grows buffers -> the next single queries must re-capture
+        gx.griffin_query_batch(ql.offsets, ql.terms, 3000)
