@@ -262,3 +262,33 @@ def make_pair_workload(num_docs: int, s_len: int, ratios: Sequence[float], seed:
     ql = QueryLog(offsets=np.arange(0, 2 * nq + 1, 2, dtype=np.uint32),
                   terms=np.arange(2 * nq, dtype=np.uint32))
     return corpus, ql
+
+
+def make_ratio_groups(num_docs: int, s_len: int, groups, pairs_per_group: int, seed: int,
+                      overlap: float = 0.10):
+    """G6 at batch scale: per ratio group one long list S (|S| = s_len) and
+    `pairs_per_group` short lists R with |R| = |S|/lambda, lambda log-uniform in
+    the group, |R n S| = overlap*|R|.  Returns (Corpus, QueryLog, group_of_query)."""
+    lists: List[np.ndarray] = []
+    qterms: List[int] = []
+    gid: List[int] = []
+    for gi, (lo, hi) in enumerate(groups):
+        rng = _rng(seed, _K_PAIR, 1_000_000 + gi)
+        s = _random_list(num_docs, s_len, rng)
+        s_id = len(lists)
+        lists.append(s)
+        for p in range(pairs_per_group):
+            rng = _rng(seed, _K_PAIR, gi * 100_000 + p)
+            lam = float(np.exp(rng.uniform(np.log(lo), np.log(hi))))
+            r_len = max(1, int(round(len(s) / lam)))
+            n_common = int(round(overlap * r_len))
+            common = rng.choice(s, size=min(n_common, len(s)), replace=False) if n_common else np.empty(0, np.uint32)
+            rest = _random_list(num_docs, max(1, r_len - len(common)), rng)
+            lists.append(np.union1d(common, rest).astype(np.uint32))
+            qterms.extend([len(lists) - 1, s_id])
+            gid.append(gi)
+    corpus = make_corpus(num_docs, np.zeros(0, dtype=np.int64), seed, queries=None, extra_lists=lists)
+    nq = len(gid)
+    ql = QueryLog(offsets=np.arange(0, 2 * nq + 1, 2, dtype=np.uint32),
+                  terms=np.array(qterms, dtype=np.uint32))
+    return corpus, ql, np.array(gid)

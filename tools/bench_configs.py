@@ -75,37 +75,40 @@ def c1():
 
 
 def c3():
+    """Merge vs gallop per ratio group (P:858-859 groups + lambda = 1000), at batch
+    scale: 64 pairs per group share one |S| = 1.5M list (fused decode, reuse off,
+    as in the paper's per-pair measurement; and with the batch arena, reuse on)."""
+    from synth import make_ratio_groups
     groups = [(1, 16), (16, 32), (32, 64), (64, 128), (128, 256), (256, 512), (512, 1024),
               (1000, 1001)]
-    rng = np.random.default_rng(0x6733)
-    per = 8
-    ratios, gid = [], []
-    for gi, (lo, hi) in enumerate(groups):
-        for _ in range(per):
-            ratios.append(float(np.exp(rng.uniform(np.log(lo), np.log(hi)))))
-            gid.append(gi)
-    c, ql = make_pair_workload(25_000_000, 1_500_000, ratios, seed=0x4752494646494E03)
+    c, ql, gid = make_ratio_groups(25_000_000, 1_500_000, groups, 64, seed=0x4752494646494E03)
     ix = g.GriffinIndex(c, block_size=128)
-    ix.griffin_set_reuse(0)
     for gi, (lo, hi) in enumerate(groups):
-        qs = [i for i in range(len(ratios)) if gid[i] == gi]
-        sub = ql.slice(qs[0], qs[-1] + 1)
+        qs = np.nonzero(gid == gi)[0]
+        sub = ql.slice(int(qs[0]), int(qs[-1]) + 1)
         res = {"config": "c3", "group": [lo, hi], "pairs": len(qs),
-               "S_len_mean": float(np.mean([c.df()[2 * i + 1] for i in qs])),
-               "R_len_mean": float(np.mean([c.df()[2 * i] for i in qs]))}
-        for name, mode in (("merge", g.MODE_MERGE), ("gallop", g.MODE_GALLOP),
-                           ("auto", g.MODE_AUTO)):
-            ix.griffin_set_mode(mode)
-            run = dev_batch(ix, sub, 10)
-            ix.griffin_reset_profile()
-            ix.griffin_set_profiling(True)
-            ms = time_dev(run, iters=5, warmup=2)
-            ix.griffin_set_profiling(False)
-            p = ix.griffin_get_profile()
-            res[name] = {"ms_per_pair": ms / len(qs),
-                         "payload_MB_per_pair": p["payload_bytes"] / 7 / len(qs) / 1e6,
-                         "decoded_postings_per_pair": p["decoded_postings"] / 7 / len(qs)}
-        res["winner"] = "merge" if res["merge"]["ms_per_pair"] <= res["gallop"]["ms_per_pair"] else "gallop"
+               "R_len_mean": float(np.mean([c.df()[sub.query(i)[0]] for i in range(sub.num_queries)])),
+               "S_len": int(c.df()[sub.query(0)[1]])}
+        for reuse in (0, 1):
+            ix.griffin_set_reuse(reuse)
+            for name, mode in (("merge", g.MODE_MERGE), ("gallop", g.MODE_GALLOP),
+                               ("auto", g.MODE_AUTO)):
+                ix.griffin_set_mode(mode)
+                run = dev_batch(ix, sub, 10)
+                ix.griffin_reset_profile()
+                ix.griffin_set_profiling(True)
+                ms = time_dev(run, iters=5, warmup=2)
+                ix.griffin_set_profiling(False)
+                p = ix.griffin_get_profile()
+                res[f"{name}{'_reuse' if reuse else ''}"] = {
+                    "us_per_pair": 1e3 * ms / len(qs),
+                    "intersect_us_per_pair": 1e3 * p["ms_intersect"] / 7 / len(qs),
+                    "payload_KB_per_pair": p["payload_bytes"] / 7 / len(qs) / 1e3,
+                    "decoded_postings_per_pair": p["decoded_postings"] / 7 / len(qs)}
+        res["winner_fused"] = ("merge" if res["merge"]["intersect_us_per_pair"] <=
+                               res["gallop"]["intersect_us_per_pair"] else "gallop")
+        res["winner_reuse"] = ("merge" if res["merge_reuse"]["intersect_us_per_pair"] <=
+                               res["gallop_reuse"]["intersect_us_per_pair"] else "gallop")
         print(json.dumps(res), flush=True)
 
 
