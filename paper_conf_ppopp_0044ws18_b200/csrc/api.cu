@@ -174,7 +174,10 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   griffin_index *ix = new griffin_index();
   ix->device = dev;
   ix->B = B;
-  ix->T = opts.gallop_ratio ? opts.gallop_ratio : B;
+  // B200 crossover measured at batch scale (tools/bench_configs.py c3, profiles/r01_c3_crossover.jsonl):
+  // galloping already wins from lambda ~ 16 for B = 128, fused or arena; the paper's 128 (= B) was the
+  // K20-vs-CPU crossover
+  ix->T = opts.gallop_ratio ? opts.gallop_ratio : std::max<uint32_t>(4, B / 8);
   ix->Tdec = opts.gallop_ratio_decoded ? opts.gallop_ratio_decoded : std::max<uint32_t>(4, B / 8);
   ix->D = std::max<uint32_t>(2, 1024 / B);
   ix->k1 = k1;
