@@ -984,7 +984,7 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
       const uint32_t sa = __shfl_sync(0xffffffffu, r_lo, 2), sb = __shfl_sync(0xffffffffu, r_lo, 3);
       const uint32_t nr = rb - ra, ns = sb - sa;
       const uint32_t tot2 = nr + ns, L = (tot2 + 31) >> 5;
-      const uint32_t cap = (L >> 1) + 1;           // matches per lane <= ceil(L/2)
+      const uint32_t cap = (L >> 1) + 2;           // matches per lane <= ceil(L/2), +1 slack write
       uint32_t *ml = sm.stg + lane * cap;          // staging is free after decode
       uint32_t c = 0;
       if (nr && ns) {
@@ -1002,17 +1002,19 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
           ie = nr;
           je = ns;
         }
-        while (is < ie && js < je) {
-          const uint32_t x = A[is], y = Bv[js];
-          if (x == y) {
-            ml[c++] = (ra + is) | (js << 16);
-            ++is;
-            ++js;
-          } else if (x < y) {
-            ++is;
-          } else {
-            ++js;
-          }
+        // branch-free serial merge: every step writes the candidate pair and
+        // keeps it only when x == y (no divergent branches in the hot loop)
+        uint32_t key = (ra + is) | (js << 16);   // R tile index | S tile index << 16
+        const uint32_t *pa = A + is, *pb = Bv + js;
+        const uint32_t *const pae = A + ie, *const pbe = Bv + je;
+        while (pa < pae && pb < pbe) {
+          const uint32_t x = *pa, y = *pb;
+          ml[c] = key;
+          c += (x == y) ? 1u : 0u;
+          const uint32_t ia = (x <= y) ? 1u : 0u, ib = (y <= x) ? 1u : 0u;
+          pa += ia;
+          pb += ib;
+          key += ia + (ib << 16);
         }
       }
       __syncwarp();
