@@ -562,6 +562,62 @@ __device__ __forceinline__ void warp_upper_bound2(const uint32_t *__restrict__ a
   *r1 = __shfl_sync(0xffffffffu, lo, 16);
 }
 
+// Skip-pointer block of each R element x (upper_bound(fS, x) - 1, kNone when x
+// precedes the list), for element lists whose range spans many skip pointers:
+// every `stride`-th skip pointer of [k_lo, k_hi) is sampled into shared memory
+// in one coalesced pass, each element binary-searches the sample there, and only
+// the last log2(stride) steps touch global memory, as interleaved independent
+// chains (4 elements per lane).  Also resets match[].
+__device__ __forceinline__ void skip_blocks_sampled(const uint32_t *__restrict__ fS, uint32_t k_lo,
+                                                    uint32_t k_hi, const uint32_t *tileR,
+                                                    uint32_t n, uint32_t *kidx, uint32_t *match,
+                                                    uint32_t *samp, uint32_t cap) {
+  const uint32_t lane = lane_id();
+  const uint32_t span = k_hi - k_lo;
+  uint32_t stride = 1;
+  while ((span + stride - 1) / stride > cap) stride <<= 1;
+  const uint32_t ns = (span + stride - 1) / stride;
+  for (uint32_t i = lane; i < ns; i += 32) samp[i] = __ldg(fS + k_lo + i * stride);
+  __syncwarp();
+  for (uint32_t base = 0; base < n; base += 128) {
+    uint32_t lo[4], hi[4], xv[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t e = base + lane + 32u * j;
+      xv[j] = e < n ? tileR[e] : 0u;
+      // sample interval: t = #samples <= x; the answer lies in (k_lo+(t-1)*stride, k_lo+t*stride]
+      uint32_t a = 0, b = ns;
+      while (a < b) {
+        const uint32_t mid = (a + b) >> 1;
+        if (samp[mid] <= xv[j]) a = mid + 1; else b = mid;
+      }
+      lo[j] = a ? k_lo + (a - 1) * stride + 1 : k_lo;
+      hi[j] = (e < n && a) ? min(k_lo + a * stride, k_hi) : lo[j];
+    }
+    for (;;) {
+      bool any = false;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        if (lo[j] < hi[j]) {
+          const uint32_t mid = (lo[j] + hi[j]) >> 1;
+          if (__ldg(fS + mid) <= xv[j]) lo[j] = mid + 1; else hi[j] = mid;
+          any = true;
+        }
+      }
+      if (!__any_sync(0xffffffffu, any)) break;
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t e = base + lane + 32u * j;
+      if (e < n) {
+        kidx[e] = lo[j] - 1u;   // kNone (0 - 1) when x < fS[k_lo] and k_lo == 0
+        match[e] = kNone;
+      }
+    }
+  }
+  __syncwarp();
+}
+
 // Multi-list probe (SvS rounds 2..m-1 in one pass): every round-1 survivor is
 // looked up in each remaining list in canonical order — skip-pointer search,
 // then an in-place binary search of the decoded-arena block or a staged EF
@@ -596,40 +652,8 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
     const uint32_t *fS = ix.first + tS.block0;
     const bool sdec = a.tdec && a.tdec[sid];
     const uint32_t *decS = sdec ? a.dec + (size_t)tS.block0 * B : nullptr;
-    uint32_t k_lo, k_hi;
-    warp_upper_bound2(fS, tS.nblocks, tileR[0], tileR[n - 1], &k_lo, &k_hi);
-    // ---- skip-pointer block of every element: interleaved chains ----
-    for (uint32_t base = 0; base < n; base += 128) {
-      uint32_t lo[4], hi[4], xv[4];
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const uint32_t e = base + lane + 32u * j;
-        lo[j] = k_lo;
-        hi[j] = e < n ? k_hi : k_lo;
-        xv[j] = e < n ? tileR[e] : 0u;
-      }
-      for (;;) {
-        bool any = false;
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          if (lo[j] < hi[j]) {
-            const uint32_t mid = (lo[j] + hi[j]) >> 1;
-            if (__ldg(fS + mid) <= xv[j]) lo[j] = mid + 1; else hi[j] = mid;
-            any = true;
-          }
-        }
-        if (!__any_sync(0xffffffffu, any)) break;
-      }
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const uint32_t e = base + lane + 32u * j;
-        if (e < n) {
-          kidx[e] = lo[j] - 1u;
-          match[e] = kNone;
-        }
-      }
-    }
-    __syncwarp();
+    skip_blocks_sampled(fS, 0, tS.nblocks, tileR, n, kidx, match, sm.stg,
+                        stage_words(B, D));
     if (sdec) {
       // ---- decoded arena: in-place binary search of the touched block ----
       uint32_t probes = 0;
@@ -1076,38 +1100,9 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
           match[e] = kNone;
         }
       } else {
-        // wide range: the lane's elements search the skip pointers in global
-        // memory as independent interleaved chains (one round trip per step)
-        for (uint32_t base = 0; base < n; base += 128) {
-          uint32_t lo[4], hi[4], xv[4];
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const uint32_t e = base + lane + 32u * j;
-            lo[j] = k_lo;
-            hi[j] = e < n ? k_hi : k_lo;
-            xv[j] = e < n ? tileR[e] : 0u;
-          }
-          for (;;) {
-            bool any = false;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-              if (lo[j] < hi[j]) {
-                const uint32_t mid = (lo[j] + hi[j]) >> 1;
-                if (__ldg(fS + mid) <= xv[j]) lo[j] = mid + 1; else hi[j] = mid;
-                any = true;
-              }
-            }
-            if (!__any_sync(0xffffffffu, any)) break;
-          }
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const uint32_t e = base + lane + 32u * j;
-            if (e < n) {
-              kidx[e] = lo[j] - 1u;   // kNone: below S's first docID
-              match[e] = kNone;
-            }
-          }
-        }
+        // wide range: sampled skip pointers in smem, then short global searches
+        skip_blocks_sampled(fS, k_lo ? k_lo - 1u : 0u, k_hi, tileR, n, kidx, match, sm.stg,
+                            stage_words(B, D));
       }
       __syncwarp();
       if (sdec) {
