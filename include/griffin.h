@@ -164,6 +164,24 @@ griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq,
 /* Synchronise the index's work and return (then clear) any device-side error. */
 griffin_status griffin_sync_status(griffin_index *ix);
 
+/* Additional query workspaces, so several batches can be in flight on different
+ * streams at once (a serving engine overlapping batch i+1's planning/decode
+ * with batch i's intersection rounds).  A workspace owns the per-batch device
+ * buffers (plans, intermediates, the decode-once arena, top-k candidates); the
+ * index data is shared read-only.  One call at a time per workspace. */
+typedef struct griffin_workspace griffin_workspace;
+griffin_status griffin_workspace_create(griffin_index *ix, griffin_workspace **out);
+void griffin_workspace_destroy(griffin_index *ix, griffin_workspace *ws);
+griffin_status griffin_workspace_reserve(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
+                                         const uint32_t *query_offsets, const uint32_t *terms,
+                                         uint32_t k);
+griffin_status griffin_query_batch_device_ws(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
+                                             const uint32_t *d_query_offsets,
+                                             const uint32_t *d_terms, uint32_t max_terms,
+                                             uint32_t k, uint64_t *d_out_keys,
+                                             uint32_t *d_out_counts, void *stream);
+griffin_status griffin_workspace_sync_status(griffin_index *ix, griffin_workspace *ws);
+
 /* Shard merge: given G per-shard sorted key runs
  * d_keys[g][nq*k] and counts d_counts[g][nq] (laid out contiguously, g-major, as
  * an all-gather produces them), write the global top-k keys and counts.  Exact:

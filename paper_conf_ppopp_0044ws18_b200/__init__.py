@@ -86,6 +86,11 @@ _SIGS = {
     "griffin_reserve": [_vp, _u32, _vp, _vp, _u32],
     "griffin_query_batch_device": [_vp, _u32, _vp, _vp, _u32, _u32, _vp, _vp, _vp],
     "griffin_sync_status": [_vp],
+    "griffin_workspace_create": [_vp, ctypes.POINTER(_vp)],
+    "griffin_workspace_destroy": [_vp, _vp],
+    "griffin_workspace_reserve": [_vp, _vp, _u32, _vp, _vp, _u32],
+    "griffin_query_batch_device_ws": [_vp, _vp, _u32, _vp, _vp, _u32, _u32, _vp, _vp, _vp],
+    "griffin_workspace_sync_status": [_vp, _vp],
     "griffin_merge_topk_device": [_vp, _u32, _u32, _u32, _vp, _vp, _vp, _vp, _vp],
     "griffin_keys_to_results_device": [_vp, _u32, _u32, _vp, _vp, _vp, _vp, _vp],
     "griffin_set_mode": [_vp, ctypes.c_int],
@@ -118,6 +123,7 @@ def load_library():
             fn.argtypes = args
             fn.restype = ctypes.c_int
         lib.griffin_index_destroy.restype = None
+        lib.griffin_workspace_destroy.restype = None
         lib.griffin_last_error.restype = ctypes.c_char_p
         lib.griffin_last_error.argtypes = []
         _lib = lib
@@ -233,6 +239,9 @@ class GriffinIndex:
     def griffin_sync_status(self):
         _check(load_library().griffin_sync_status(self.h))
 
+    def griffin_workspace_create(self) -> "GriffinWorkspace":
+        return GriffinWorkspace(self)
+
     def griffin_merge_topk_device(self, num_runs: int, nq: int, k: int, d_keys, d_counts,
                                   d_out_keys, d_out_counts, stream=None):
         st = ctypes.c_void_p(stream.cuda_stream if stream is not None else 0)
@@ -306,6 +315,42 @@ class GriffinIndex:
         return out[:n.value]
 
 
-__all__ = ["GriffinIndex", "GriffinError", "load_library", "griffin_last_error",
+class GriffinWorkspace:
+    """An extra query workspace of an index (griffin_workspace): lets several
+    batches be in flight on different streams."""
+
+    def __init__(self, index: GriffinIndex):
+        self.index = index
+        h = ctypes.c_void_p()
+        _check(load_library().griffin_workspace_create(index.h, ctypes.byref(h)))
+        self.h = h
+
+    def close(self):
+        if getattr(self, "h", None) and _lib is not None and getattr(self.index, "h", None):
+            _lib.griffin_workspace_destroy(self.index.h, self.h)
+        self.h = None
+
+    def __del__(self):
+        self.close()
+
+    def griffin_workspace_reserve(self, offsets, terms, k: int):
+        off = np.ascontiguousarray(offsets, np.uint32)
+        t = np.ascontiguousarray(terms, np.uint32)
+        _check(load_library().griffin_workspace_reserve(self.index.h, self.h, len(off) - 1,
+                                                        _ptr(off), _ptr(t), k))
+
+    def griffin_query_batch_device_ws(self, d_offsets, d_terms, max_terms: int, k: int,
+                                      d_out_keys, d_out_counts, stream=None):
+        nq = d_offsets.numel() - 1
+        st = ctypes.c_void_p(stream.cuda_stream if stream is not None else 0)
+        _check(load_library().griffin_query_batch_device_ws(
+            self.index.h, self.h, nq, _dptr(d_offsets), _dptr(d_terms), max_terms, k,
+            _dptr(d_out_keys), _dptr(d_out_counts), st))
+
+    def griffin_workspace_sync_status(self):
+        _check(load_library().griffin_workspace_sync_status(self.index.h, self.h))
+
+
+__all__ = ["GriffinIndex", "GriffinWorkspace", "GriffinError", "load_library", "griffin_last_error",
            "griffin_shard_range", "griffin_merge_path_split", "MODE_AUTO", "MODE_MERGE",
            "MODE_GALLOP", "LIB_PATH"]

@@ -46,8 +46,9 @@ static griffin_status ensure_pinned(griffin_index *ix, size_t bytes) {
 }
 
 // Host validation of one batch's query terms + workspace reservation.
-static griffin_status reserve_for(griffin_index *ix, uint32_t nq, const uint32_t *qoffs,
-                                  const uint32_t *terms, uint32_t k, uint32_t *max_terms) {
+static griffin_status reserve_for(griffin_index *ix, Workspace &w, uint32_t nq,
+                                  const uint32_t *qoffs, const uint32_t *terms, uint32_t k,
+                                  uint32_t *max_terms) {
   if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
   uint64_t caps = 0, units = 0;
   uint32_t mt = 1;
@@ -68,16 +69,16 @@ static griffin_status reserve_for(griffin_index *ix, uint32_t nq, const uint32_t
     units += u;
   }
   if (max_terms) *max_terms = mt;
-  return reserve_ws(ix, nq, units, caps);
+  return reserve_ws(ix, w, nq, units, caps);
 }
 
-static griffin_status read_status(griffin_index *ix) {
+static griffin_status read_status(griffin_index *ix, Workspace &w) {
   int status = 0;
-  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(&status, ix->ws.scal.as<unsigned long long>() + kScalStatus,
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(&status, w.scal.as<unsigned long long>() + kScalStatus,
                                    sizeof(int), cudaMemcpyDeviceToHost, ix->stream));
   GRIFFIN_CUDA_TRY(cudaStreamSynchronize(ix->stream));
   if (status) {
-    GRIFFIN_CUDA_TRY(cudaMemsetAsync(ix->ws.scal.as<unsigned long long>() + kScalStatus, 0, 8,
+    GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.scal.as<unsigned long long>() + kScalStatus, 0, 8,
                                      ix->stream));
     GRIFFIN_CUDA_TRY(cudaStreamSynchronize(ix->stream));
     if (status & kStatusOverflow) {
@@ -243,6 +244,8 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   return GRIFFIN_OK;
 }
 
+static void free_workspace(Workspace &w);
+
 void griffin_index_destroy(griffin_index *ix) {
   if (!ix) return;
   {
@@ -254,6 +257,11 @@ void griffin_index_destroy(griffin_index *ix) {
     cudaFree(ix->d_payload);
     cudaFree(ix->d_tfw);
     cudaFree(ix->d_norm);
+    for (Workspace *xw : ix->extra_ws) {
+      free_workspace(*xw);
+      delete xw;
+    }
+    ix->extra_ws.clear();
     Workspace &w = ix->ws;
     for (DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel, &w.qmode,
                       &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal,
@@ -296,7 +304,7 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
   uint32_t max_terms = 1;
-  griffin_status s = reserve_for(ix, nq, qoffs, terms, k, &max_terms);
+  griffin_status s = reserve_for(ix, ix->ws, nq, qoffs, terms, k, &max_terms);
   if (s) return s;
   Workspace &w = ix->ws;
   const uint64_t nt = qoffs[nq];
@@ -317,7 +325,7 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qoffs.p, hp, ((size_t)nq + 1) * 4, cudaMemcpyHostToDevice, st));
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qterms.p, hp + ((size_t)nq + 1) * 4, nt * 4,
                                    cudaMemcpyHostToDevice, st));
-  s = run_batch(ix, nq, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), max_terms, k,
+  s = run_batch(ix, ix->ws, nq, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), max_terms, k,
                 w.keys.as<uint64_t>(), w.counts.as<uint32_t>(), st, true, ix->mode);
   if (s) return s;
   if ((s = launch_keys_to_results(ix, nq, k, w.keys.as<uint64_t>(), w.counts.as<uint32_t>(),
@@ -327,7 +335,7 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho, w.docids.p, nk * 4, cudaMemcpyDeviceToHost, st));
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho + nk * 4, w.scores.p, nk * 4, cudaMemcpyDeviceToHost, st));
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho + nk * 8, w.counts.p, (size_t)nq * 4, cudaMemcpyDeviceToHost, st));
-  if ((s = read_status(ix))) return s;  // synchronises
+  if ((s = read_status(ix, ix->ws))) return s;  // synchronises
   std::memcpy(out_docids, ho, nk * 4);
   std::memcpy(out_scores, ho + nk * 4, nk * 4);
   std::memcpy(out_counts, ho + nk * 8, (size_t)nq * 4);
@@ -356,7 +364,7 @@ static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint
   const uint32_t offs[2] = {0, nterms};
   uint32_t mt = 1;
   // validation + bounds (same rules as the batch path)
-  griffin_status s = reserve_for(ix, 1, offs, terms, k, &mt);
+  griffin_status s = reserve_for(ix, ix->ws, 1, offs, terms, k, &mt);
   if (s) return s;
   if (!ix->single_ws) {
     uint64_t mx = 0, mb = 0;
@@ -364,9 +372,9 @@ static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint
       mx = std::max<uint64_t>(mx, t.df_local);
       mb = std::max<uint64_t>(mb, t.nblocks);
     }
-    if ((s = reserve_ws(ix, 1, 2 * mb + 1, mx + 1))) return s;
-    if ((s = reserve_topk(ix, 1, GRIFFIN_MAX_K))) return s;
-    if ((s = reserve_topk(ix, 1, 2048))) return s;   // the k with the most selection levels
+    if ((s = reserve_ws(ix, w, 1, 2 * mb + 1, mx + 1))) return s;
+    if ((s = reserve_topk(ix, w, 1, GRIFFIN_MAX_K))) return s;
+    if ((s = reserve_topk(ix, w, 1, 2048))) return s;   // the k with the most selection levels
     GRIFFIN_CUDA_TRY(w.qoffs.reserve(8));
     GRIFFIN_CUDA_TRY(w.qterms.reserve(GRIFFIN_MAX_TERMS * 4 * 4));
     GRIFFIN_CUDA_TRY(w.keys.reserve(GRIFFIN_MAX_K * 8));
@@ -395,7 +403,7 @@ static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint
     GRIFFIN_CUDA_TRY(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
     cudaMemcpyAsync(w.qoffs.p, h_off, 8, cudaMemcpyHostToDevice, st);
     cudaMemcpyAsync(w.qterms.p, h_terms, GRIFFIN_MAX_TERMS * 4 * 4, cudaMemcpyHostToDevice, st);
-    griffin_status rs = run_batch(ix, 1, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), mt, k,
+    griffin_status rs = run_batch(ix, ix->ws, 1, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), mt, k,
                                   w.keys.as<uint64_t>(), w.counts.as<uint32_t>(), st, true,
                                   ix->mode);
     if (!rs)
@@ -426,7 +434,7 @@ static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint
   GRIFFIN_CUDA_TRY(cudaGraphLaunch(exec, st));
   GRIFFIN_CUDA_TRY(cudaStreamSynchronize(st));
   if (*h_status) {
-    if ((s = read_status(ix))) return s;   // clears the device flag
+    if ((s = read_status(ix, ix->ws))) return s;   // clears the device flag
   }
   std::memcpy(out_docids, h_res, (size_t)k * 4);
   std::memcpy(out_scores, h_res + (size_t)k * 4, (size_t)k * 4);
@@ -453,7 +461,7 @@ griffin_status griffin_reserve(griffin_index *ix, uint32_t nq, const uint32_t *q
   if (!ix || (nq && (!qoffs || !terms))) return invalid("null argument");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
-  return reserve_for(ix, nq, qoffs, terms, k, nullptr);
+  return reserve_for(ix, ix->ws, nq, qoffs, terms, k, nullptr);
 }
 
 griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs,
@@ -466,7 +474,7 @@ griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq, const 
   if (nq == 0) return GRIFFIN_OK;
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
-  return run_batch(ix, nq, d_qoffs, d_terms, max_terms, k, d_out_keys, d_out_counts,
+  return run_batch(ix, ix->ws, nq, d_qoffs, d_terms, max_terms, k, d_out_keys, d_out_counts,
                    static_cast<cudaStream_t>(stream), true, ix->mode);
 }
 
@@ -476,7 +484,72 @@ griffin_status griffin_sync_status(griffin_index *ix) {
   DeviceGuard guard(ix->device);
   GRIFFIN_CUDA_TRY(cudaDeviceSynchronize());
   if (!ix->ws.scal.p) return GRIFFIN_OK;
-  return read_status(ix);
+  return read_status(ix, ix->ws);
+}
+
+griffin_status griffin_workspace_create(griffin_index *ix, griffin_workspace **out) {
+  if (!ix || !out) return invalid("null argument");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  Workspace *w = new Workspace();
+  ix->extra_ws.push_back(w);
+  *out = reinterpret_cast<griffin_workspace *>(w);
+  return GRIFFIN_OK;
+}
+
+static void free_workspace(Workspace &w) {
+  for (DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel, &w.qmode,
+                    &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.rbuf0,
+                    &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys, &w.counts,
+                    &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand, &w.tdec, &w.runs,
+                    &w.run_base, &w.vtmp, &w.arena})
+    b->release();
+  if (w.h_pinned) cudaFreeHost(w.h_pinned);
+  w.h_pinned = nullptr;
+}
+
+void griffin_workspace_destroy(griffin_index *ix, griffin_workspace *ws) {
+  if (!ix || !ws) return;
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  Workspace *w = reinterpret_cast<Workspace *>(ws);
+  cudaDeviceSynchronize();
+  free_workspace(*w);
+  for (size_t i = 0; i < ix->extra_ws.size(); ++i)
+    if (ix->extra_ws[i] == w) ix->extra_ws.erase(ix->extra_ws.begin() + i);
+  delete w;
+}
+
+griffin_status griffin_workspace_reserve(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
+                                         const uint32_t *qoffs, const uint32_t *terms,
+                                         uint32_t k) {
+  if (!ix || !ws || (nq && (!qoffs || !terms))) return invalid("null argument");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  return reserve_for(ix, *reinterpret_cast<Workspace *>(ws), nq, qoffs, terms, k, nullptr);
+}
+
+griffin_status griffin_query_batch_device_ws(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
+                                             const uint32_t *d_qoffs, const uint32_t *d_terms,
+                                             uint32_t max_terms, uint32_t k, uint64_t *d_out_keys,
+                                             uint32_t *d_out_counts, void *stream) {
+  if (!ix || !ws) return invalid("null argument");
+  if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
+  if (max_terms == 0 || max_terms > GRIFFIN_MAX_TERMS) return invalid("max_terms out of range");
+  if (nq == 0) return GRIFFIN_OK;
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  return run_batch(ix, *reinterpret_cast<Workspace *>(ws), nq, d_qoffs, d_terms, max_terms, k,
+                   d_out_keys, d_out_counts, static_cast<cudaStream_t>(stream), true, ix->mode);
+}
+
+griffin_status griffin_workspace_sync_status(griffin_index *ix, griffin_workspace *ws) {
+  if (!ix || !ws) return invalid("null argument");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  GRIFFIN_CUDA_TRY(cudaDeviceSynchronize());
+  Workspace &w = *reinterpret_cast<Workspace *>(ws);
+  if (!w.scal.p) return GRIFFIN_OK;
+  return read_status(ix, w);
 }
 
 griffin_status griffin_merge_topk_device(griffin_index *ix, uint32_t num_runs, uint32_t nq,
@@ -532,10 +605,13 @@ griffin_status griffin_reset_profile(griffin_index *ix) {
   ix->pending.clear();
   ix->ev_next = 0;
   ix->launch_count = 0;
-  if (ix->ws.scal.p) {
-    GRIFFIN_CUDA_TRY(cudaMemset(ix->ws.scal.p, 0, 4 * 8));
-    GRIFFIN_CUDA_TRY(cudaMemset(ix->ws.scal.as<unsigned long long>() + kScalDec, 0, 3 * 8));
-  }
+  std::vector<Workspace *> all(ix->extra_ws);
+  all.push_back(&ix->ws);
+  for (Workspace *w : all)
+    if (w->scal.p) {
+      GRIFFIN_CUDA_TRY(cudaMemset(w->scal.p, 0, 4 * 8));
+      GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDec, 0, 3 * 8));
+    }
   return GRIFFIN_OK;
 }
 
@@ -557,16 +633,21 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
   ix->ev_next = 0;
   *out = ix->prof;
   out->launches_total = ix->launch_count;
-  if (ix->ws.scal.p) {
+  std::vector<Workspace *> all(ix->extra_ws);
+  all.push_back(&ix->ws);
+  out->alg_bytes = out->payload_bytes = out->decoded_postings = out->survivors = 0;
+  out->dec_alg_bytes = out->dec_payload_bytes = out->dec_postings = 0;
+  for (Workspace *w : all) {
+    if (!w->scal.p) continue;
     unsigned long long c[kScalCount];
-    GRIFFIN_CUDA_TRY(cudaMemcpy(c, ix->ws.scal.p, sizeof(c), cudaMemcpyDeviceToHost));
-    out->alg_bytes = c[0];
-    out->payload_bytes = c[1];
-    out->decoded_postings = c[2];
-    out->survivors = c[3];
-    out->dec_alg_bytes = c[kScalDec + 0];
-    out->dec_payload_bytes = c[kScalDec + 1];
-    out->dec_postings = c[kScalDec + 2];
+    GRIFFIN_CUDA_TRY(cudaMemcpy(c, w->scal.p, sizeof(c), cudaMemcpyDeviceToHost));
+    out->alg_bytes += c[0];
+    out->payload_bytes += c[1];
+    out->decoded_postings += c[2];
+    out->survivors += c[3];
+    out->dec_alg_bytes += c[kScalDec + 0];
+    out->dec_payload_bytes += c[kScalDec + 1];
+    out->dec_postings += c[kScalDec + 2];
   }
   return GRIFFIN_OK;
 }
@@ -691,7 +772,7 @@ griffin_status griffin_debug_intersect(griffin_index *ix, const uint32_t *terms,
   DeviceGuard guard(ix->device);
   const uint32_t offs[2] = {0, nterms};
   uint32_t max_terms = 1;
-  griffin_status s = reserve_for(ix, 1, offs, terms, 1, &max_terms);
+  griffin_status s = reserve_for(ix, ix->ws, 1, offs, terms, 1, &max_terms);
   if (s) return s;
   Workspace &w = ix->ws;
   GRIFFIN_CUDA_TRY(w.qoffs.reserve(8));
@@ -699,10 +780,10 @@ griffin_status griffin_debug_intersect(griffin_index *ix, const uint32_t *terms,
   cudaStream_t st = ix->stream;
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qoffs.p, offs, 8, cudaMemcpyHostToDevice, st));
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qterms.p, terms, (size_t)nterms * 4, cudaMemcpyHostToDevice, st));
-  s = run_batch(ix, 1, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), max_terms, 1, nullptr,
+  s = run_batch(ix, ix->ws, 1, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), max_terms, 1, nullptr,
                 nullptr, st, false, mode);
   if (s) return s;
-  if ((s = read_status(ix))) return s;
+  if ((s = read_status(ix, ix->ws))) return s;
   return copy_final_docids(ix, out_docids, cap, count);
 }
 

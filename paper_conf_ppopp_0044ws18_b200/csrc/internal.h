@@ -124,6 +124,7 @@ struct griffin_index {
   std::vector<griffin::TermInfo> h_terms;
   // query state
   griffin::Workspace ws;
+  std::vector<griffin::Workspace *> extra_ws;  // griffin_workspace_create
   int mode = 0;
   int reuse = 2;
   // single-query CUDA graphs, keyed by (distinct terms, k, mode, workspace identity)
@@ -168,12 +169,13 @@ namespace griffin {
 griffin_status encode_index(griffin_index *ix, const uint32_t *h_docids_local,
                             const uint32_t *h_tfs, const std::vector<uint64_t> &post_off);
 // query.cu
-griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs,
+griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uint32_t *d_qoffs,
                          const uint32_t *d_terms, uint32_t max_terms, uint32_t k,
                          uint64_t *d_keys, uint32_t *d_counts, cudaStream_t st, bool final_topk,
                          int forced_mode);
-griffin_status reserve_ws(griffin_index *ix, uint32_t nq, uint64_t units, uint64_t entries);
-griffin_status reserve_topk(griffin_index *ix, uint32_t nq, uint32_t k);
+griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t units,
+                          uint64_t entries);
+griffin_status reserve_topk(griffin_index *ix, Workspace &w, uint32_t nq, uint32_t k);
 griffin_status launch_merge_topk(griffin_index *ix, uint32_t G, uint32_t nq, uint32_t k,
                                  const uint64_t *d_keys, const uint32_t *d_counts,
                                  uint64_t *d_out_keys, uint32_t *d_out_counts, cudaStream_t st);

@@ -1813,8 +1813,8 @@ static int num_sms(int dev) {
   return cache[dev];
 }
 
-griffin_status reserve_ws(griffin_index *ix, uint32_t nq, uint64_t units, uint64_t entries) {
-  Workspace &w = ix->ws;
+griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t units,
+                          uint64_t entries) {
   const size_t q = (size_t)nq + 1;
   GRIFFIN_CUDA_TRY(w.plan_terms.reserve(q * kMaxTerms * 4));
   GRIFFIN_CUDA_TRY(w.plan_m.reserve(q * 4));
@@ -1890,8 +1890,7 @@ static cudaError_t launch_intersect(griffin_index *ix, const RoundArgs &ra, cuda
 
 // Top-k candidate buffers for a batch of nq queries with this k (grow-only;
 // called before a CUDA-graph capture so no allocation happens inside it).
-griffin_status reserve_topk(griffin_index *ix, uint32_t nq, uint32_t k) {
-  Workspace &w = ix->ws;
+griffin_status reserve_topk(griffin_index *ix, Workspace &w, uint32_t nq, uint32_t k) {
   const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
   const int levels = k <= 64 ? 1 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
   GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8 * std::max(levels, 1)));
@@ -1899,10 +1898,9 @@ griffin_status reserve_topk(griffin_index *ix, uint32_t nq, uint32_t k) {
   return GRIFFIN_OK;
 }
 
-griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs,
+griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uint32_t *d_qoffs,
                          const uint32_t *d_terms, uint32_t max_terms, uint32_t k, uint64_t *d_keys,
                          uint32_t *d_counts, cudaStream_t st, bool final_topk, int forced_mode) {
-  Workspace &w = ix->ws;
   if (nq == 0) return GRIFFIN_OK;
   if (nq > w.nq_cap || !w.scal.p) {
     set_error("workspace not reserved for this batch (call griffin_reserve)");
@@ -2036,7 +2034,7 @@ griffin_status run_batch(griffin_index *ix, uint32_t nq, const uint32_t *d_qoffs
     // by kTopkSmem / k; small k needs 2 levels, large k up to kTopkMaxLevels)
     const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
     const int levels = k <= 64 ? 1 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
-    griffin_status rs_ = reserve_topk(ix, nq, k);
+    griffin_status rs_ = reserve_topk(ix, w, nq, k);
     if (rs_) return rs_;
     CandBufs cb{};
     for (int L = 1; L <= levels; ++L) cb.lv[L] = w.cand.as<uint64_t>() + (size_t)(L - 1) * cand_cap;

@@ -367,3 +367,37 @@ def test_single_query_graph_path_reuse_and_recapture(tiny):
                 assert_topk_equal(gd, gs, gc, od, os_, oc)
         # a batch grows buffers -> the next single queries must re-capture
         gx.griffin_query_batch(ql.offsets, ql.terms, 3000)
+
+
+def test_concurrent_workspaces_on_two_streams(tiny):
+    """Two batches in flight on two streams (default + extra workspace) give the
+    same, oracle-exact results as one at a time."""
+    import torch
+    c, ql, ox = tiny
+    gx = g.GriffinIndex(c, block_size=128)
+    ws = gx.griffin_workspace_create()
+    k = 25
+    nq = ql.num_queries
+    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    gx.griffin_reserve(ql.offsets, ql.terms, k)
+    ws.griffin_workspace_reserve(ql.offsets, ql.terms, k)
+    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
+    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
+    outs = [(torch.zeros(nq * k, dtype=torch.int64, device="cuda"),
+             torch.zeros(nq, dtype=torch.int32, device="cuda")) for _ in range(2)]
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    for _ in range(3):
+        gx.griffin_query_batch_device(d_off, d_t, mt, k, outs[0][0], outs[0][1], s1)
+        ws.griffin_query_batch_device_ws(d_off, d_t, mt, k, outs[1][0], outs[1][1], s2)
+    torch.cuda.synchronize()
+    gx.griffin_sync_status()
+    ws.griffin_workspace_sync_status()
+    assert torch.equal(outs[0][0], outs[1][0]) and torch.equal(outs[0][1], outs[1][1])
+    dd = torch.zeros(nq * k, dtype=torch.int32, device="cuda")
+    ds = torch.zeros(nq * k, dtype=torch.float32, device="cuda")
+    gx.griffin_keys_to_results_device(nq, k, outs[1][0], outs[1][1], dd, ds)
+    torch.cuda.synchronize()
+    od, os_, oc = ox.query_batch(ql, k)
+    assert_topk_equal(dd.cpu().numpy().view(np.uint32).reshape(nq, k), ds.cpu().numpy().reshape(nq, k),
+                      outs[1][1].cpu().numpy().view(np.uint32), od, os_, oc)
+    ws.close()
