@@ -129,17 +129,19 @@ def c5(nq=None):
                 "decode_sweep": {"ms": sw["ms"], "gbs": sw["bytes"] / (sw["ms"] / 1e3) / 1e9,
                                  "gpostings_per_s": sw["postings"] / (sw["ms"] / 1e3) / 1e9}}
         if B == 128:
-            run = dev_batch(ix, ql, k)
-            ix.griffin_reset_profile()
-            ix.griffin_set_profiling(True)
-            ms = time_dev(run, iters=3, warmup=2)
-            ix.griffin_set_profiling(False)
-            p = ix.griffin_get_profile()
-            line.update({"queries": ql.num_queries, "k": k, "ms_per_batch": ms,
-                         "qps": ql.num_queries / (ms / 1e3),
-                         "stage_ms": {kk: p[kk] / 5 for kk in ("ms_plan", "ms_decode",
-                                                                 "ms_intersect", "ms_compact",
-                                                                 "ms_topk")}})
+            for kq in (k, 10):   # C5 (top-1000) and the C4 per-shard workload at G = 1 (top-10)
+                run = dev_batch(ix, ql, kq)
+                ix.griffin_reset_profile()
+                ix.griffin_set_profiling(True)
+                ms = time_dev(run, iters=3, warmup=2)
+                ix.griffin_set_profiling(False)
+                p = ix.griffin_get_profile()
+                line[f"k{kq}"] = {"queries": ql.num_queries, "k": kq, "ms_per_batch": ms,
+                                  "qps": ql.num_queries / (ms / 1e3),
+                                  "intersect_alg_gbs": p["alg_bytes"] / (p["ms_intersect"] / 1e3) / 1e9,
+                                  "stage_ms": {kk: p[kk] / 5 for kk in (
+                                      "ms_plan", "ms_decode", "ms_intersect", "ms_compact",
+                                      "ms_topk")}}
         print(json.dumps(line), flush=True)
         ix.close()
 
