@@ -11,5 +11,5 @@ ix = g.GriffinIndex(c, block_size=128)
 run = dev_batch(ix, ql, cfg["k"])
 run(); torch.cuda.synchronize(); run(); torch.cuda.synchronize()
 PY
-timeout 1800 ncu --set full --clock-control none --import-source on -k regex:"intersect_kernel|decode_once" -s 5 -c 3 -o gpurun_out/prof_c5 -f python /tmp/c5one.py > gpurun_out/prof_c5.log 2>&1
+timeout 1800 ncu --set full --clock-control none --import-source on -k regex:"intersect_kernel|decode_once" -s 3 -c 3 -o gpurun_out/prof_c5 -f python /tmp/c5one.py > gpurun_out/prof_c5.log 2>&1
 tail -3 gpurun_out/prof_c5.log
