@@ -190,7 +190,8 @@ def run_gpu(args):
     import torch.distributed as dist
 
     import paper_conf_ppopp_0044ws18_b200 as g
-    from paper_conf_ppopp_0044ws18_b200.sharded import ShardedSearcher, gather_runs
+    from paper_conf_ppopp_0044ws18_b200.sharded import (ShardedSearcher, exchange_sliced,
+                                                        gather_runs)
     from synth import make_workload
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -205,8 +206,16 @@ def run_gpu(args):
     corpus, ql, cfg = make_workload(args.config)
     k, B = cfg["k"], cfg["block"]
     nq = ql.num_queries
+    # docid: rank r holds docID-range shard r and the per-shard top-k are exchanged
+    # (all-gather, or the query-sliced all-to-all); replicate: every rank holds the
+    # whole index and runs its own batch, no exchange
+    replicate = world > 1 and args.shard_mode == "replicate"
+    sharded = world > 1 and not replicate
     t0 = time.time()
-    ix = g.GriffinIndex(corpus, block_size=B, device=dev, shard_index=rank, num_shards=world)
+    if replicate:
+        ix = g.GriffinIndex(corpus, block_size=B, device=dev)
+    else:
+        ix = g.GriffinIndex(corpus, block_size=B, device=dev, shard_index=rank, num_shards=world)
     build_s = time.time() - t0
     st = ix.griffin_index_stats()
     ix.griffin_reserve(ql.offsets, ql.terms, k)
@@ -219,14 +228,14 @@ def run_gpu(args):
     # batches in flight: slot 0 = the index's own workspace on the current
     # stream, slots 1.. = extra workspaces on their own streams (serving engine
     # overlapping consecutive batches); each slot has its own outputs
-    nstreams = max(1, args.streams) if world == 1 else 1
+    nstreams = max(1, args.streams) if not sharded else 1
     slots = [(None, stream, keys, cnts)]
     for _ in range(nstreams - 1):
         w = ix.griffin_workspace_create()
         w.griffin_workspace_reserve(ql.offsets, ql.terms, k)
         slots.append((w, torch.cuda.Stream(), torch.zeros(nq * k, dtype=torch.int64, device="cuda"),
                       torch.zeros(nq, dtype=torch.int32, device="cuda")))
-    if world > 1:
+    if sharded:
         out_keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
         out_cnts = torch.zeros(nq, dtype=torch.int32, device="cuda")
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device="cuda")  # 256 MB > L2
@@ -240,9 +249,13 @@ def run_gpu(args):
 
     def step():
         ix.griffin_query_batch_device(d_off, d_terms, max_terms, k, keys, cnts, stream)
-        if world > 1:
+        if sharded and args.exchange == "allgather":
             ak, ac = gather_runs(keys, cnts)
             ix.griffin_merge_topk_device(world, nq, k, ak, ac, out_keys, out_cnts, stream)
+        elif sharded:
+            ak, ac, (lo, hi) = exchange_sliced(keys, cnts, k)
+            if hi > lo:
+                ix.griffin_merge_topk_device(world, hi - lo, k, ak, ac, out_keys, out_cnts, stream)
 
     for i in range(args.warmup):
         step_on(i)
@@ -292,7 +305,8 @@ def run_gpu(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     ms_per_step = total_ms / args.steps
-    qps = nq * args.steps / (total_ms / 1e3)
+    # replicate: every rank answered its own full batch (weak scaling)
+    qps = (world if replicate else 1) * nq * args.steps / (total_ms / 1e3)
     peak, peak_kind = _peaks()
     ms_x = prof["ms_intersect"]
     achieved = prof["alg_bytes"] / (ms_x / 1e3) / 1e9 if ms_x > 0 else 0.0
@@ -326,20 +340,24 @@ def run_gpu(args):
     # ---- e2e: the public host-buffer C-ABI call, H2D of the step's queries and
     # D2H of its results inside every timed step (wall clock, max over ranks)
     e2e_times = []
-    if world > 1:
+    if sharded:
         searcher = ShardedSearcher.from_index(ix)
+    if world > 1:
         h_off = torch.from_numpy(ql.offsets.astype(np.int32)).pin_memory()
         h_terms = torch.from_numpy(ql.terms.astype(np.int32)).pin_memory()
     for i in range(args.warmup + args.steps):
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
-        if world == 1:
+        if not sharded:
             dd, ss, cc = ix.griffin_query_batch(ql.offsets, ql.terms, k)
         else:
             e_off = h_off.to("cuda", non_blocking=True)
             e_terms = h_terms.to("cuda", non_blocking=True)
-            dd, ss, cc = searcher.search(e_off, e_terms, max_terms, k, stream)
+            if args.exchange == "allgather":
+                dd, ss, cc = searcher.search(e_off, e_terms, max_terms, k, stream)
+            else:
+                _, _, dd, ss, cc = searcher.search_sliced(e_off, e_terms, max_terms, k, stream)
             dd, ss, cc = dd.cpu(), ss.cpu(), cc.cpu()
         dt = time.perf_counter() - t0
         if i >= args.warmup:
@@ -351,6 +369,8 @@ def run_gpu(args):
         e2e_s = float(t.item())
     h2d = (nq + 1) * 4 + len(ql.terms) * 4
     d2h = nq * k * 8 + nq * 4
+    if sharded and args.exchange == "sliced":   # each rank reads back its own slice
+        d2h = -(-nq // world) * (k * 8 + 4)
 
     # ---- closed-loop single-query latency (griffin_query, one in flight)
     lat = []
@@ -369,8 +389,8 @@ def run_gpu(args):
     line = {
         "metric": "queries/sec", "value": qps, "unit": "queries/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/f32",
-        "data": "synthetic",
+        "higher_is_better": True, "scaling": "weak" if replicate else "strong",
+        "vs_baseline": None, "dtype": "u32/f32", "data": "synthetic",
         "config": {"workload": WORKLOAD_DESC[args.config], "num_docs": corpus.num_docs,
                    "num_terms": corpus.num_terms, "num_postings": corpus.num_postings,
                    "queries_per_step": nq, "k": k, "block_size": B,
@@ -378,7 +398,9 @@ def run_gpu(args):
                           "inputs larger than L2 (index %.0f MB, L2 126 MB); not flushed" %
                           ((st["payload_bytes"] + st["skip_bytes"] + st["tf_bytes"]) / 1e6)),
                    "batches_in_flight": len(slots),
-                   "parallelism": f"docid-range shards x{world}" if world > 1 else "1 shard",
+                   "parallelism": (f"docid-range shards x{world}, {args.exchange} exchange"
+                                   if sharded else f"replicated index x{world}, no exchange"
+                                   if replicate else "1 shard"),
                    "index_bytes_per_shard": st["payload_bytes"] + st["skip_bytes"] + st["tf_bytes"],
                    "index_build_s": build_s},
         "decoded_postings_per_s": decoded_ps * world,
@@ -394,7 +416,8 @@ def run_gpu(args):
                               ("ms_plan", "ms_decode", "ms_intersect", "ms_compact", "ms_topk",
                                "ms_merge")},
         "gpu_launches": int(prof["launches_total"]),
-        "e2e": {"value": nq * args.steps / e2e_s, "unit": "queries/s", "h2d_bytes_per_step": h2d,
+        "e2e": {"value": (world if replicate else 1) * nq * args.steps / e2e_s,
+                "unit": "queries/s", "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": d2h,
                 "how": "griffin_query_batch (host buffers; pinned staging, H2D queries, D2H results)"},
         "clocks": clk,
@@ -440,6 +463,10 @@ def main():
     ap.add_argument("--latency-queries", type=int, default=1000)
     ap.add_argument("--streams", type=int, default=2,
                     help="batches in flight on separate streams/workspaces (N=1 only)")
+    ap.add_argument("--shard-mode", default="docid", choices=["docid", "replicate"],
+                    help="N>1: docID-range shards + exchange, or a replicated index per rank")
+    ap.add_argument("--exchange", default="allgather", choices=["allgather", "sliced"],
+                    help="docid shards: all-gather of per-shard top-k, or query-sliced all-to-all")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()

@@ -24,7 +24,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, out_q):
+def _worker(rank, world, port, out_q, exchange="allgather"):
     import sys
     sys.path.insert(0, ROOT)
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -34,7 +34,8 @@ def _worker(rank, world, port, out_q):
     try:
         import oracle
         import paper_conf_ppopp_0044ws18_b200 as g
-        from paper_conf_ppopp_0044ws18_b200.sharded import gather_runs
+        from paper_conf_ppopp_0044ws18_b200.sharded import (exchange_sliced, gather_runs,
+                                                            query_slices)
         from synth import make_workload
         c, ql, cfg = make_workload("tiny")
         ox = oracle.OracleIndex(c)
@@ -54,15 +55,22 @@ def _worker(rank, world, port, out_q):
                 keys[q, i] = (np.uint64(sb) << np.uint64(32)) | np.uint64(0xFFFFFFFF - d)
         kt = torch.from_numpy(keys.view(np.int64).reshape(-1).copy())
         ct = torch.from_numpy(cnts)
-        all_k, all_c = gather_runs(kt, ct)
-        assert all_k.shape == (world, nq * k) and all_c.shape == (world, nq)
+        if exchange == "allgather":
+            all_k, all_c = gather_runs(kt, ct)
+            lo, hi = 0, nq
+        else:
+            all_k, all_c, (lo, hi) = exchange_sliced(kt, ct, k)
+            assert (lo, hi) == query_slices(nq, world)[rank]
+        m = hi - lo
+        assert all_k.shape == (world, m * k) and all_c.shape == (world, m)
         # reference k-way merge over the g-major runs
         ok = True
-        for q in range(nq):
+        for q in range(lo, hi):
             runs = []
             for r in range(world):
-                n = int(all_c[r, q])
-                runs += [int(x) & 0xFFFFFFFFFFFFFFFF for x in all_k[r, q * k:q * k + n].tolist()]
+                n = int(all_c[r, q - lo])
+                runs += [int(x) & 0xFFFFFFFFFFFFFFFF
+                         for x in all_k[r, (q - lo) * k:(q - lo) * k + n].tolist()]
             top = sorted(runs, reverse=True)[:k]
             want = [(int(S[q, i].view(np.uint32)) << 32) | (0xFFFFFFFF - int(D[q, i]))
                     for i in range(min(k, C[q]))]
@@ -72,12 +80,12 @@ def _worker(rank, world, port, out_q):
         dist.destroy_process_group()
 
 
-def test_gloo_world2_shard_exchange_and_merge_exact():
-    world = 2
+def _run(world, exchange):
     port = _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, exchange))
+             for r in range(world)]
     for p in procs:
         p.start()
     res = [q.get(timeout=240) for _ in range(world)]
@@ -85,3 +93,22 @@ def test_gloo_world2_shard_exchange_and_merge_exact():
         p.join(timeout=60)
         assert p.exitcode == 0
     assert all(ok for _, ok in res), res
+
+
+def test_gloo_world2_shard_exchange_and_merge_exact():
+    _run(2, "allgather")
+
+
+def test_gloo_world3_query_sliced_exchange_exact():
+    """NEXT-2: all-to-all of per-shard runs by query slice (uneven slices at G=3)."""
+    _run(3, "sliced")
+
+
+def test_query_slices_cover():
+    from paper_conf_ppopp_0044ws18_b200.sharded import query_slices
+    for nq in (0, 1, 2, 7, 1000):
+        for w in (1, 2, 3, 8):
+            sl = query_slices(nq, w)
+            assert len(sl) == w and sl[0][0] == 0 and sl[-1][1] == nq
+            assert all(a <= b for a, b in sl)
+            assert all(sl[i][1] == sl[i + 1][0] for i in range(w - 1))
