@@ -204,6 +204,12 @@ griffin_status griffin_set_profiling(griffin_index *ix, int on);
  * EF-decoded once per batch into an HBM arena (the paper's decompress-then-
  * intersect pipeline, Alg. 1 output `decmp_array`) and intersected from there. */
 griffin_status griffin_set_reuse(griffin_index *ix, int mode);
+/* Galloping into a compressed (not arena-decoded) list: 1 = EF NextGEQ (default;
+ * select0 over the staged block's unary high stream finds the bucket of the
+ * probe's high part, only that bucket's few elements are decoded — SURVEY
+ * §8(f) NEXT-1), 0 = decode every touched block (Para-EF) and binary-search it.
+ * Results are identical; only the work differs.  Invalid value -> INVALID_ARG. */
+griffin_status griffin_set_nextgeq(griffin_index *ix, int on);
 griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out); /* syncs */
 griffin_status griffin_reset_profile(griffin_index *ix);
 const char *griffin_last_error(void);

@@ -96,6 +96,7 @@ _SIGS = {
     "griffin_set_mode": [_vp, ctypes.c_int],
     "griffin_set_profiling": [_vp, ctypes.c_int],
     "griffin_set_reuse": [_vp, ctypes.c_int],
+    "griffin_set_nextgeq": [_vp, ctypes.c_int],
     "griffin_get_profile": [_vp, ctypes.POINTER(Profile)],
     "griffin_reset_profile": [_vp],
     "griffin_shard_range": [_u32, _u32, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u32)],
@@ -263,6 +264,10 @@ class GriffinIndex:
     def griffin_set_reuse(self, mode: int):
         """0 off (fused decode every round), 1 on (decode hot lists once per batch), 2 auto."""
         _check(load_library().griffin_set_reuse(self.h, mode))
+
+    def griffin_set_nextgeq(self, on: bool):
+        """Gallop into compressed lists by EF NextGEQ (True, default) or block decode."""
+        _check(load_library().griffin_set_nextgeq(self.h, int(on)))
 
     def griffin_set_profiling(self, on: bool):
         _check(load_library().griffin_set_profiling(self.h, int(on)))

@@ -589,6 +589,17 @@ griffin_status griffin_set_reuse(griffin_index *ix, int mode) {
   return GRIFFIN_OK;
 }
 
+griffin_status griffin_set_nextgeq(griffin_index *ix, int on) {
+  if (!ix || on < 0 || on > 1) return invalid("nextgeq must be 0 or 1");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  if (ix->nextgeq != on) {   // captured single-query graphs bake the option in
+    for (auto &g : ix->graphs) cudaGraphExecDestroy(g.exec);
+    ix->graphs.clear();
+  }
+  ix->nextgeq = on;
+  return GRIFFIN_OK;
+}
+
 griffin_status griffin_set_profiling(griffin_index *ix, int on) {
   if (!ix) return invalid("null index");
   std::lock_guard<std::mutex> lk(ix->mu);

@@ -269,6 +269,60 @@ __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ 
   __syncwarp();
 }
 
+// ---- EF NextGEQ inside one staged block -------------------
+// Index of the first element >= x of the block staged at stg (n if none) and
+// its value in `val`, without decoding the block: the elements whose high part
+// is >= h = (x - first) >> b start right after the h-th zero of the unary high
+// stream (each zero closes one high bucket), so a select0 over the
+// high words (popc per word, byte LUT in the word) gives their index
+// i0 = pos - h; only the few elements of bucket h (about u/n / 2^b <= 2 on
+// average) are then decoded and compared.  One lane per query element.
+__device__ __forceinline__ uint32_t ef_next_geq_staged(const uint32_t *__restrict__ stg,
+                                                       uint32_t first, uint32_t y, uint32_t x,
+                                                       const uint8_t *__restrict__ lut,
+                                                       uint32_t &val) {
+  const uint32_t b = meta_b(y), n = meta_n(y), hw = meta_hw(y);
+  const uint32_t *hs = stg + low_words(n, b);
+  val = first;
+  if (x <= first) return 0u;
+  const uint32_t h = (x - first) >> b;
+  uint32_t pos = 0;   // first bit of the one-scan
+  uint32_t w = 0, cur = 0;
+  if (h) {
+    uint32_t need = h;
+    for (;;) {
+      if (w >= hw) return n;   // fewer than h zeros: every high part is < h
+      cur = hs[w];
+      const uint32_t z = 32u - __popc(cur);
+      if (z >= need) break;
+      need -= z;
+      ++w;
+    }
+    pos = (w << 5) + select_in_word(~cur, need - 1u, lut) + 1u;
+  }
+  uint32_t i = pos - h;   // ones before pos = pos - (zeros before pos = h)
+  const uint32_t mask = b ? (0xFFFFFFFFu >> (32u - b)) : 0u;
+  w = pos >> 5;
+  cur = w < hw ? hs[w] & (0xFFFFFFFFu << (pos & 31u)) : 0u;
+  while (i < n) {
+    while (cur == 0u) {
+      if (++w >= hw) return n;
+      cur = hs[w];
+    }
+    const uint32_t p = (w << 5) + (__ffs(cur) - 1u);
+    cur &= cur - 1u;
+    const uint32_t bp = i * b;
+    const uint32_t lo = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp) & mask;
+    const uint32_t xv = first + (((p - i) << b) | lo);
+    if (xv >= x) {
+      val = xv;
+      return i;
+    }
+    ++i;
+  }
+  return n;
+}
+
 // payload size of a block in 16-B units
 __host__ __device__ inline uint32_t block_size16(uint32_t y) {
   return (low_words(meta_n(y), meta_b(y)) + meta_hw(y) + 3u) >> 2;

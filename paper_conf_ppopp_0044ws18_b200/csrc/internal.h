@@ -81,6 +81,7 @@ struct RoundArgs {
   uint32_t nq, round, D, T, Tdec;
   int forced_mode;
   int probe;
+  int nextgeq;   // gallop into compressed S by EF NextGEQ (no block decode)
   const uint32_t *plan_terms;
   const uint32_t *plan_m;
   const uint32_t *cap;
@@ -138,6 +139,7 @@ struct griffin_index {
   bool single_ws = false;
   int use_graphs = 1;
   int probe = 1;
+  int nextgeq = 1;
   bool profiling = false;
   griffin_profile prof{};
   std::vector<cudaEvent_t> ev_pool;

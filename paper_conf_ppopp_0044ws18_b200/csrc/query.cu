@@ -736,7 +736,7 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
         if (lane >= ng) sz = 0;
         if (lane < ng) sn[lane] = nn;
         const uint32_t pay = __reduce_add_sync(0xffffffffu, lane < ng ? sz * 16u : 0u);
-        const uint32_t pst = __reduce_add_sync(0xffffffffu, lane < ng ? nn : 0u);
+        const uint32_t pst = __reduce_add_sync(0xffffffffu, lane < ng && !a.nextgeq ? nn : 0u);
         if (lane == 0) {
           acc.pay += pay;
           acc.post += pst;
@@ -744,18 +744,31 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
         }
         const uint32_t soff = warp_incl_scan(sz) - sz;
         stage_blocks(ix, sm, ng, mm, soff, sz, false);
-        for (uint32_t i = 0; i < ng; ++i) {
-          const uint32_t y = __shfl_sync(0xffffffffu, mm.y, i);
-          const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
-          const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
-          warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+        if (!a.nextgeq) {
+          for (uint32_t i = 0; i < ng; ++i) {
+            const uint32_t y = __shfl_sync(0xffffffffu, mm.y, i);
+            const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
+            const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
+            warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+          }
         }
         __syncwarp();
         for (;;) {
           const uint32_t e = ep + lane;
           const uint32_t gi = e < n ? kidx[e] : kNone;
           const bool in = gi != kNone && gi < g0 + ng;
-          if (in) {
+          if (a.nextgeq) {
+            const uint32_t src = in ? gi - g0 : 0u;
+            const uint32_t y = __shfl_sync(0xffffffffu, mm.y, src);
+            const uint32_t fi = __shfl_sync(0xffffffffu, f, src);
+            const uint32_t so = __shfl_sync(0xffffffffu, soff, src);
+            if (in) {
+              const uint32_t x = tileR[e];
+              uint32_t v;
+              const uint32_t p = ef_next_geq_staged(sm.stg + so * 4u, fi, y, x, sm.lut, v);
+              if (p < meta_n(y) && v == x) match[e] = dblk[gi] * B + p;
+            }
+          } else if (in) {
             const uint32_t x = tileR[e];
             const uint32_t *seg = tileS + (gi - g0) * B;
             const uint32_t p = lower_bound_s(seg, 0, sn[gi - g0], x);
@@ -1208,7 +1221,8 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
         {
           const bool own = lane < ng && !(lu > 0 && blk == k_first);
           const uint32_t sp = __reduce_add_sync(0xffffffffu, (own && !sdec) ? sz * 16u : 0u);
-          const uint32_t spn = __reduce_add_sync(0xffffffffu, (own && !sdec) ? nn : 0u);
+          const uint32_t spn =
+              __reduce_add_sync(0xffffffffu, (own && !sdec && !a.nextgeq) ? nn : 0u);
           const uint32_t sa = __reduce_add_sync(
               0xffffffffu, own ? (sdec ? nn * 4u : sz * 16u + 8u) : 0u);
           if (lane == 0) {
@@ -1217,6 +1231,7 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
             acc.alg += sa;
           }
         }
+        uint32_t soff = 0;
         if (sdec) {
           // decoded arena: each touched block straight into its tileS slot
           const uint32_t by = lane < ng ? ((nn + 3u) & ~3u) * 4u : 0u;
@@ -1230,22 +1245,37 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
           mbar_wait(sm.mbar, sm.phase);
           sm.phase ^= 1u;
         } else {
-          const uint32_t soff = warp_incl_scan(sz) - sz;
+          soff = warp_incl_scan(sz) - sz;
           stage_blocks(ix, sm, ng, m, soff, sz, false);
-          for (uint32_t i = 0; i < ng; ++i) {
-            const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
-            const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
-            const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
-            warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+          if (!a.nextgeq) {
+            for (uint32_t i = 0; i < ng; ++i) {
+              const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
+              const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
+              const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
+              warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
+            }
           }
         }
         __syncwarp();
         // elements mapping to this group: contiguous from ep
+        const bool ngeq = !sdec && a.nextgeq;
         for (;;) {
           const uint32_t e = ep + lane;
           const uint32_t gi = e < n ? kidx[e] : kNone;
           const bool in = gi != kNone && gi < g0 + ng;
-          if (in) {
+          if (ngeq) {
+            // NextGEQ on the staged payload: no block decode (NEXT-1)
+            const uint32_t src = in ? gi - g0 : 0u;
+            const uint32_t y = __shfl_sync(0xffffffffu, m.y, src);
+            const uint32_t fi = __shfl_sync(0xffffffffu, f, src);
+            const uint32_t so = __shfl_sync(0xffffffffu, soff, src);
+            if (in) {
+              const uint32_t x = tileR[e];
+              uint32_t v;
+              const uint32_t p = ef_next_geq_staged(sm.stg + so * 4u, fi, y, x, sm.lut, v);
+              if (p < meta_n(y) && v == x) match[e] = dblk[gi] * B + p;
+            }
+          } else if (in) {
             const uint32_t x = tileR[e];
             const uint32_t *seg = tileS + (gi - g0) * B;
             const uint32_t p = lower_bound_s(seg, 0, sn[gi - g0], x);
@@ -1986,6 +2016,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
   }
   // multi-list probe replaces SvS rounds 2..m-1 (auto mode, B small enough for its smem)
   ra.probe = forced_mode == 0 && ix->probe && ix->D >= 5;
+  ra.nextgeq = ix->nextgeq;
   uint32_t rounds = std::max<uint32_t>(1, max_terms > 0 ? max_terms - 1 : 1);
   if (ra.probe) rounds = std::min<uint32_t>(rounds, 2);
   for (uint32_t r = 1; r <= rounds; ++r) {

@@ -401,3 +401,49 @@ def test_concurrent_workspaces_on_two_streams(tiny):
     assert_topk_equal(dd.cpu().numpy().view(np.uint32).reshape(nq, k), ds.cpu().numpy().reshape(nq, k),
                       outs[1][1].cpu().numpy().view(np.uint32), od, os_, oc)
     ws.close()
+
+
+# ---------------------------------------------------------------- EF NextGEQ gallop
+
+def _nextgeq_corpus(rng, N=3_000_000):
+    """Lists that stress the bucket search: a consecutive run (b = 0), a very
+    sparse list (large b, many empty buckets), a clustered list (bursts of
+    consecutive docIDs: full buckets next to long zero runs), and random lists
+    of several densities to probe them with."""
+    run = np.arange(1_000_000, 1_006_000)
+    sparse = np.sort(rng.choice(N, size=900, replace=False))
+    starts = np.sort(rng.choice(N - 64, size=400, replace=False))
+    clustered = np.unique(np.concatenate([s + np.arange(int(rng.integers(1, 60))) for s in starts]))
+    lists = [run, sparse, clustered] + [np.sort(rng.choice(N, size=n, replace=False))
+                                        for n in (300, 3_000, 30_000, 300_000, 1_500_000)]
+    tfs = [rng.integers(1, 9, size=len(x)) for x in lists]
+    return corpus_from_lists(N, lists, tfs, rng.integers(1, 3000, size=N))
+
+
+@pytest.mark.parametrize("B", [64, 128, 256, 512])
+def test_nextgeq_gallop_matches_block_decode_and_oracle(B):
+    """Galloping into compressed lists by EF NextGEQ (select0 on the unary stream,
+    only the probe's bucket decoded) gives the oracle's sets and bit-exact top-k;
+    so does the block-decode gallop it replaces (griffin_set_nextgeq(0))."""
+    rng = np.random.default_rng(900 + B)
+    c = _nextgeq_corpus(rng)
+    ox = oracle.OracleIndex(c)
+    gx = g.GriffinIndex(c, block_size=B)
+    gx.griffin_set_reuse(0)           # S stays compressed: the NextGEQ path
+    pairs = [[a, b] for a in range(8) for b in range(8) if a != b]
+    triples = [list(rng.choice(8, size=3, replace=False)) for _ in range(20)]
+    qs = pairs + triples
+    ql = QueryLog(offsets=np.cumsum([0] + [len(q) for q in qs]).astype(np.uint32),
+                  terms=np.concatenate(qs).astype(np.uint32))
+    for ng in (1, 0):
+        gx.griffin_set_nextgeq(ng)
+        for q in qs:
+            want = ox.intersect(q)
+            for mode in (g.MODE_GALLOP, g.MODE_AUTO):
+                assert np.array_equal(gx.griffin_debug_intersect(q, mode), want), (ng, q, mode)
+        for mode in (g.MODE_GALLOP, g.MODE_AUTO):
+            gx.griffin_set_mode(mode)
+            od, os_, oc = ox.query_batch(ql, 100)
+            gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 100)
+            assert_topk_equal(gd, gs, gc, od, os_, oc)
+        gx.griffin_set_mode(g.MODE_AUTO)

@@ -91,9 +91,13 @@ def c3():
                "S_len": int(c.df()[sub.query(0)[1]])}
         for reuse in (0, 1):
             ix.griffin_set_reuse(reuse)
-            for name, mode in (("merge", g.MODE_MERGE), ("gallop", g.MODE_GALLOP),
-                               ("auto", g.MODE_AUTO)):
+            for name, mode, ngeq in (("merge", g.MODE_MERGE, 1), ("gallop", g.MODE_GALLOP, 1),
+                                     ("gallop_blockdec", g.MODE_GALLOP, 0),
+                                     ("auto", g.MODE_AUTO, 1)):
+                if reuse and ngeq == 0:
+                    continue
                 ix.griffin_set_mode(mode)
+                ix.griffin_set_nextgeq(ngeq)
                 run = dev_batch(ix, sub, 10)
                 ix.griffin_reset_profile()
                 ix.griffin_set_profiling(True)
