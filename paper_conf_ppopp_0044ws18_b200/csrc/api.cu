@@ -262,13 +262,7 @@ void griffin_index_destroy(griffin_index *ix) {
       delete xw;
     }
     ix->extra_ws.clear();
-    Workspace &w = ix->ws;
-    for (DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel, &w.qmode,
-                      &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal,
-                      &w.keys, &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand,
-                      &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.arena})
-      b->release();
-    if (w.h_pinned) cudaFreeHost(w.h_pinned);
+    free_workspace(ix->ws);
     for (cudaEvent_t e : ix->ev_pool) cudaEventDestroy(e);
     for (auto &g : ix->graphs) cudaGraphExecDestroy(g.exec);
     if (ix->stream) cudaStreamDestroy(ix->stream);
@@ -348,7 +342,8 @@ static uint64_t ws_identity(const Workspace &w) {
   for (const DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel,
                           &w.qmode, &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec,
                           &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys,
-                          &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms})
+                          &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand,
+                          &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.run_term, &w.arena})
     h = (h ^ (uint64_t)(uintptr_t)b->p) * 1099511628211ull;
   return h ^ (uint64_t)(uintptr_t)w.h_pinned;
 }
@@ -501,7 +496,7 @@ static void free_workspace(Workspace &w) {
                     &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.rbuf0,
                     &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys, &w.counts,
                     &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand, &w.tdec, &w.runs,
-                    &w.run_base, &w.vtmp, &w.arena})
+                    &w.run_base, &w.vtmp, &w.run_term, &w.arena})
     b->release();
   if (w.h_pinned) cudaFreeHost(w.h_pinned);
   w.h_pinned = nullptr;

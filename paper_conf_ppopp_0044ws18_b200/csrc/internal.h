@@ -58,7 +58,7 @@ struct Workspace {
   DevBuf rbuf0, rbuf1, bump, cand, tkstate;                                 // per survivor
   DevBuf scal;       // scalars: counters, status, bump ctr, unit ctr
   DevBuf keys, counts, docids, scores, qoffs, qterms;  // host-API staging on device
-  DevBuf demand, tdec, runs, run_base, vtmp;           // per term (batch reuse)
+  DevBuf demand, tdec, runs, run_base, vtmp, run_term; // per term / run (batch reuse)
   DevBuf arena;                                        // decoded lists, nblocks * B u32
   size_t nq_cap = 0, unit_cap = 0, entry_cap = 0;
   // pinned host staging
@@ -76,6 +76,8 @@ enum : int {
   kScalDec = 10,      // 3 x u64: decode-once alg bytes, payload bytes, postings
   kScalCount = 13
 };
+
+constexpr uint32_t kBumpChunk = 256;   // bump-area entries grabbed per warp atomic
 
 struct RoundArgs {
   uint32_t nq, round, D, T, Tdec;
@@ -97,6 +99,7 @@ struct RoundArgs {
   uint2 *rnext;
   uint2 *bump;
   uint64_t entry_cap;
+  uint64_t bump_cap;      // entries of the bump area (entry_cap + per-warp chunk slack)
   unsigned long long *scal;
   uint4 *urec;            // per unit: {q, i0|lu, j0, lo docID} (partition stage)
   const uint32_t *dec;    // batch decoded arena (global block * B + i), or null

@@ -176,10 +176,30 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
 
 struct Acc {
   unsigned long long alg = 0, pay = 0, post = 0, surv = 0;
+  // this warp's bump chunk in warp smem: {next free entry (u64), entries left (u32)}
+  unsigned long long *boff = nullptr;
+  uint32_t *bleft = nullptr;
 };
 
+// Output space for a unit's survivors (lane 0): carved from a per-warp chunk of
+// the bump area, so the global counter sees one atomic per kBumpChunk entries
+// instead of one per unit (same-address atomics serialise in L2).  Unit outputs
+// are located by unit_off/unit_cnt, so chunk order and gaps do not matter.
+__device__ __forceinline__ unsigned long long bump_alloc(const RoundArgs &a, Acc &acc,
+                                                         uint32_t cnt) {
+  unsigned long long off = *acc.boff;
+  uint32_t left = *acc.bleft;
+  if (cnt > left) {
+    left = cnt > kBumpChunk ? cnt : kBumpChunk;
+    off = atomicAdd(a.scal + kScalBump, (unsigned long long)left);
+  }
+  *acc.boff = off + cnt;
+  *acc.bleft = left - cnt;
+  return off;
+}
+
 // Per-warp shared memory carve-up (u32 words):
-//   [mbar 4][cnt 64][aux B+32][stg SW][tile (D+2)*B]
+//   [mbar+bump state 8][cnt 64][aux B+32][stg SW][tile (D+2)*B]
 // stg holds TMA-staged EF payloads; after decoding, the merge path reuses it for
 // the per-R-element match array.  The gallop path carves tile into
 // tileR | kidx | match | tileS[G blocks].
@@ -190,7 +210,7 @@ __host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D) {
   return ((D + 2) * B / 2 + 64 + 3) & ~3u;
 }
 __host__ __device__ inline uint32_t warp_smem_words(uint32_t B, uint32_t D) {
-  return 4 + 64 + (B + 32) + stage_words(B, D) + (D + 2) * B;
+  return 8 + 64 + (B + 32) + stage_words(B, D) + (D + 2) * B;
 }
 constexpr uint32_t kLutBytes = 2048;
 
@@ -207,8 +227,8 @@ __device__ __forceinline__ WarpSmem carve_warp_smem(uint4 *smem4, uint32_t B, ui
   w.lut = base;
   uint32_t *wb = reinterpret_cast<uint32_t *>(base + kLutBytes) +
                  (threadIdx.x >> 5) * warp_smem_words(B, D);
-  w.mbar = reinterpret_cast<uint64_t *>(wb);
-  w.cnt = wb + 4;
+  w.mbar = reinterpret_cast<uint64_t *>(wb);   // words 0-1; 2: bump left; 4-5: bump offset
+  w.cnt = wb + 8;
   w.aux = w.cnt + 64;
   w.stg = w.aux + B + 32;
   w.tile = w.stg + stage_words(B, D);
@@ -315,9 +335,9 @@ __device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, co
     }
   }
   unsigned long long off = 0;
-  if (lane == 0 && cnt) off = atomicAdd(a.scal + kScalBump, (unsigned long long)cnt);
+  if (lane == 0 && cnt) off = bump_alloc(a, acc, cnt);
   off = __shfl_sync(0xffffffffu, off, 0);
-  if (off + cnt > a.entry_cap) {
+  if (off + cnt > a.bump_cap) {
     if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
     cnt = 0;
   }
@@ -368,9 +388,9 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
   const uint32_t incl = warp_incl_scan(c);
   uint32_t cnt = __shfl_sync(0xffffffffu, incl, 31);
   unsigned long long off = 0;
-  if (lane == 0 && cnt) off = atomicAdd(a.scal + kScalBump, (unsigned long long)cnt);
+  if (lane == 0 && cnt) off = bump_alloc(a, acc, cnt);
   off = __shfl_sync(0xffffffffu, off, 0);
-  if (off + cnt > a.entry_cap) {
+  if (off + cnt > a.bump_cap) {
     if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
     cnt = 0;
   }
@@ -810,9 +830,9 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
   // ---- emit the survivors ----
   unsigned long long off = 0;
   uint32_t cnt = n;
-  if (lane == 0 && cnt) off = atomicAdd(a.scal + kScalBump, (unsigned long long)cnt);
+  if (lane == 0 && cnt) off = bump_alloc(a, acc, cnt);
   off = __shfl_sync(0xffffffffu, off, 0);
-  if (off + cnt > a.entry_cap) {
+  if (off + cnt > a.bump_cap) {
     if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
     cnt = 0;
   }
@@ -837,6 +857,12 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
   const uint32_t G = min(D - 1u, 31u);   // gallop: S blocks staged per group
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   Acc acc;
+  acc.bleft = reinterpret_cast<uint32_t *>(sm.mbar) + 2;
+  acc.boff = reinterpret_cast<unsigned long long *>(sm.mbar) + 2;
+  if (lane == 0) {
+    *acc.bleft = 0;
+    *acc.boff = 0;
+  }
   // dynamic unit tickets (balances long gallop/probe units); the next ticket is
   // requested at the start of a unit so its latency overlaps the unit's work
   unsigned long long ticket = 0;
@@ -1012,11 +1038,13 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
       }
       __syncwarp();
       // ranges inside [lo, hi)
+      // lanes 0-3 search (R, lo), (R, hi), (S, lo), (S, hi) in one converged loop
       uint32_t r_lo = 0;
-      if (lane == 0) r_lo = lower_bound_s(sm.tile, 0, nRt, lo_v);
-      if (lane == 1) r_lo = lower_bound_s(sm.tile, 0, nRt, hi_v);
-      if (lane == 2) r_lo = lower_bound_s(tileS, 0, nSt, lo_v);
-      if (lane == 3) r_lo = lower_bound_s(tileS, 0, nSt, hi_v);
+      {
+        const uint32_t *arr = lane < 2 ? sm.tile : tileS;
+        const uint64_t key = (lane & 1) ? hi_v : lo_v;
+        r_lo = lower_bound_s(arr, 0, lane < 2 ? nRt : (lane < 4 ? nSt : 0u), key);
+      }
       const uint32_t ra = __shfl_sync(0xffffffffu, r_lo, 0), rb = __shfl_sync(0xffffffffu, r_lo, 1);
       const uint32_t sa = __shfl_sync(0xffffffffu, r_lo, 2), sb = __shfl_sync(0xffffffffu, r_lo, 3);
       const uint32_t nr = rb - ra, ns = sb - sa;
@@ -1040,19 +1068,35 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
           je = ns;
         }
         // branch-free serial merge: every step writes the candidate pair and
-        // keeps it only when x == y (no divergent branches in the hot loop)
+        // keeps it only when x == y (no divergent branches in the hot loop).
+        // Each step advances at least one side, so min(remaining A, remaining B)
+        // steps can run without bound checks; re-check only between such runs.
+        // 32-bit shared addresses keep the step at ~12 instructions.
         uint32_t key = (ra + is) | (js << 16);   // R tile index | S tile index << 16
-        const uint32_t *pa = A + is, *pb = Bv + js;
-        const uint32_t *const pae = A + ie, *const pbe = Bv + je;
-        while (pa < pae && pb < pbe) {
-          const uint32_t x = *pa, y = *pb;
-          ml[c] = key;
-          c += (x == y) ? 1u : 0u;
-          const uint32_t ia = (x <= y) ? 1u : 0u, ib = (y <= x) ? 1u : 0u;
-          pa += ia;
-          pb += ib;
-          key += ia + (ib << 16);
+        uint32_t pa = smem_u32(A + is), pb = smem_u32(Bv + js);
+        const uint32_t pm0 = smem_u32(ml);
+        uint32_t pm = pm0;
+        uint32_t ra_left = ie - is, rb_left = je - js;
+        for (;;) {
+          const uint32_t K = min(ra_left, rb_left);
+          if (K == 0) break;
+          const uint32_t pa0 = pa, pb0 = pb;
+#pragma unroll 4
+          for (uint32_t t = 0; t < K; ++t) {
+            uint32_t x, y;
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(pa));
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(y) : "r"(pb));
+            asm volatile("st.shared.u32 [%0], %1;" ::"r"(pm), "r"(key));
+            pm += (x == y) ? 4u : 0u;
+            const uint32_t da = (x <= y) ? 1u : 0u, db = (y <= x) ? 1u : 0u;
+            pa += da << 2;
+            pb += db << 2;
+            key += da + (db << 16);
+          }
+          ra_left -= (pa - pa0) >> 2;
+          rb_left -= (pb - pb0) >> 2;
         }
+        c = (pm - pm0) >> 2;
       }
       __syncwarp();
       if (RC)
@@ -1789,8 +1833,19 @@ __global__ void select_kernel(DevIndex ix, const uint32_t *demand, uint8_t *tdec
 // Para-EF decode of every block of the selected terms into the arena
 // (slot = global block * B + i): warp per run of <= D+2 consecutive blocks,
 // TMA-staged payloads, decoded tile written back with 128-bit stores.
+// run -> term map for decode_once (replaces a per-run binary search over run_base)
+__global__ void run_map_kernel(uint32_t V, const uint32_t *runs, const uint64_t *run_base,
+                               uint32_t *run_term) {
+  const uint32_t t = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;   // warp per term
+  if (t >= V) return;
+  const uint32_t nr = runs[t];
+  const uint64_t b = run_base[t];
+  for (uint32_t i = lane_id(); i < nr; i += 32) run_term[b + i] = t;
+}
+
 __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t D,
-                                                          const uint64_t *run_base, uint32_t *arena,
+                                                          const uint64_t *run_base,
+                                                          const uint32_t *run_term, uint32_t *arena,
                                                           unsigned long long *scal) {
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
@@ -1802,11 +1857,7 @@ __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t 
   unsigned long long alg = 0, pay = 0, post = 0;
   for (uint64_t r = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); r < total;
        r += nwarps) {
-    uint32_t lo = 0, hi = V;
-    while (hi - lo > 1) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if (run_base[mid] <= r) lo = mid; else hi = mid;
-    }
+    const uint32_t lo = run_term[r];
     const TermInfo t = ix.terms[lo];
     const uint32_t ri = (uint32_t)(r - run_base[lo]);
     const uint32_t k0 = ri * run, nb = min(run, t.nblocks - k0);
@@ -1860,7 +1911,9 @@ griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t
   GRIFFIN_CUDA_TRY(w.unit_dst.reserve((units + 2) * 8 + (units / kScanTile + 2) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf0.reserve((entries + 1) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf1.reserve((entries + 1) * 8));
-  GRIFFIN_CUDA_TRY(w.bump.reserve((entries + 1) * 8));
+  // per-warp bump chunks: at most one partly used chunk per resident warp
+  const size_t bump_slack = (size_t)num_sms(ix->device) * 64 * kBumpChunk;
+  GRIFFIN_CUDA_TRY(w.bump.reserve((entries + bump_slack + 1) * 8));
   if (!w.scal.p) {
     GRIFFIN_CUDA_TRY(w.scal.reserve(kScalCount * 8));
     GRIFFIN_CUDA_TRY(cudaMemset(w.scal.p, 0, w.scal.bytes));
@@ -1960,6 +2013,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
   ra.unit_cap = w.unit_cap;
   ra.bump = w.bump.as<uint2>();
   ra.entry_cap = w.entry_cap;
+  ra.bump_cap = w.bump.bytes / 8 - 1;
   ra.scal = scal;
   const unsigned qblocks = (nq + 255) / 256;
   {
@@ -1987,6 +2041,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     GRIFFIN_CUDA_TRY(w.runs.reserve((size_t)V * 4));
     GRIFFIN_CUDA_TRY(w.run_base.reserve(((size_t)V + 2) * 8));
     GRIFFIN_CUDA_TRY(w.vtmp.reserve(((size_t)V / kScanTile + 4) * 8));
+    GRIFFIN_CUDA_TRY(w.run_term.reserve((ix->nblocks / (ix->D + 2) + (size_t)V + 2) * 4));
     GRIFFIN_CUDA_TRY(w.arena.reserve((ix->nblocks * ix->B + 64) * 4));
     GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.demand.p, 0, (size_t)V * 4, st));
     ra.T = ix->T;
@@ -1996,6 +2051,9 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
                                                    ix->D + 2);
     GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(w.runs.as<uint32_t>(), w.run_base.as<uint64_t>(), V,
                                               w.vtmp.as<uint64_t>(), st, &ix->launch_count));
+    run_map_kernel<<<(uint32_t)(((uint64_t)V * 32 + 255) / 256), 256, 0, st>>>(V, w.runs.as<uint32_t>(),
+                                                    w.run_base.as<uint64_t>(),
+                                                    w.run_term.as<uint32_t>());
     const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * 8;
     static thread_local int cfg_dev = -1;
     static thread_local size_t cfg_smem = 0;
@@ -2008,9 +2066,10 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, decode_once_kernel, 256, smem);
     decode_once_kernel<<<num_sms(ix->device) * std::max(1, per_sm), 256, smem, st>>>(
-        di, ix->D, w.run_base.as<uint64_t>(), w.arena.as<uint32_t>(), scal);
+        di, ix->D, w.run_base.as<uint64_t>(), w.run_term.as<uint32_t>(), w.arena.as<uint32_t>(),
+        scal);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
-    ix->launch_count += 3;
+    ix->launch_count += 4;
     ra.dec = w.arena.as<uint32_t>();
     ra.tdec = w.tdec.as<uint8_t>();
   }
