@@ -21,6 +21,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.cpp")
+_SRCS = [_SRC, os.path.join(_HERE, "pfd.cpp")]
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
@@ -31,9 +32,10 @@ _f32p = ctypes.POINTER(ctypes.c_float)
 
 def build(force: bool = False) -> str:
     """Compile liboracle.so (plain g++, -ffp-contract=off, no fast-math)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    if force or not os.path.exists(_LIB) or any(os.path.getmtime(_LIB) < os.path.getmtime(f)
+                                                 for f in _SRCS):
         cmd = ["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-fno-fast-math", "-fPIC",
-               "-shared", "-pthread", _SRC, "-o", _LIB + ".tmp"]
+               "-shared", "-pthread", *_SRCS, "-o", _LIB + ".tmp"]
         subprocess.check_call(cmd)
         os.replace(_LIB + ".tmp", _LIB)
     return _LIB
@@ -69,6 +71,10 @@ def _load():
             getattr(lib, fn).argtypes = [ctypes.c_void_p, ctypes.c_uint32]
         lib.oracle_k1p1.restype = ctypes.c_float
         lib.oracle_k1p1.argtypes = [ctypes.c_void_p]
+        lib.oracle_pfd_encode.restype = ctypes.c_uint32
+        lib.oracle_pfd_encode.argtypes = [_u32p, ctypes.c_uint32, ctypes.c_int, _u32p,
+                                          ctypes.c_uint32, _u32p, _u32p]
+        lib.oracle_pfd_decode.argtypes = [_u32p, ctypes.c_uint32, ctypes.c_uint32, _u32p]
         lib.oracle_index_bytes.restype = ctypes.c_uint64
         lib.oracle_index_bytes.argtypes = [ctypes.c_void_p]
         _lib = lib
@@ -106,6 +112,41 @@ def ef_decode(low, high, n: int, b: int) -> np.ndarray:
     out = np.zeros(n, np.uint32)
     lib.oracle_ef_decode(_p(low, _u32p), _p(high, _u32p), n, b, _p(out, _u32p))
     return out
+
+
+def pfd_encode(x, b: Optional[int] = None):
+    """PforDelta block encode (pfd.cpp): returns (words, b, n_exceptions).  The
+    block's first docID x[0] is its skip entry and is not in the stream."""
+    lib = _load()
+    v = np.ascontiguousarray(x, dtype=np.uint32)
+    cap = 2 + 2 * len(v) + 8
+    out = np.zeros(cap, np.uint32)
+    bo, ne = ctypes.c_uint32(), ctypes.c_uint32()
+    nw = lib.oracle_pfd_encode(_p(v, _u32p), len(v), -1 if b is None else int(b), _p(out, _u32p),
+                               cap, ctypes.byref(bo), ctypes.byref(ne))
+    if nw == 0:
+        raise ValueError("oracle_pfd_encode rejected the input")
+    return out[:nw].copy(), bo.value, ne.value
+
+
+def pfd_decode(words, first: int, n: int) -> np.ndarray:
+    lib = _load()
+    w = np.ascontiguousarray(np.concatenate([np.asarray(words, np.uint32), np.zeros(2, np.uint32)]))
+    out = np.zeros(n, np.uint32)
+    if lib.oracle_pfd_decode(_p(w, _u32p), first, n, _p(out, _u32p)):
+        raise ValueError("oracle_pfd_decode: malformed stream")
+    return out
+
+
+def pfd_list_bytes(docids, block_size: int = 128) -> int:
+    """PforDelta size of one list in the same block layout as the EF index: per
+    block the stream (16-B padded) + an 8-B skip entry (first docID + offset)."""
+    x = np.asarray(docids, np.uint32)
+    tot = 0
+    for s in range(0, len(x), block_size):
+        w, _, _ = pfd_encode(x[s:s + block_size])
+        tot += ((len(w) * 4 + 15) // 16) * 16 + 8
+    return tot
 
 
 class OracleIndex:

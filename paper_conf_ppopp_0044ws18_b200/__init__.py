@@ -116,11 +116,19 @@ def load_library():
     """Load libgriffin.so (building it in-tree with nvcc if it is missing or stale)."""
     global _lib
     if _lib is None:
-        if not os.path.exists(LIB_PATH) or _build._stale():
-            _build.build()
-        lib = ctypes.CDLL(LIB_PATH)
+        alt = os.environ.get("GRIFFIN_LIBRARY")   # A/B runs: another build of the same ABI
+        if alt:
+            lib = ctypes.CDLL(alt)
+        else:
+            if not os.path.exists(LIB_PATH) or _build._stale():
+                _build.build()
+            lib = ctypes.CDLL(LIB_PATH)
         for name, args in _SIGS.items():
-            fn = getattr(lib, name)
+            fn = getattr(lib, name, None)
+            if fn is None and alt:   # an older A/B build may predate some entry points
+                continue
+            if fn is None:
+                raise GriffinError(f"libgriffin.so lacks {name}")
             fn.argtypes = args
             fn.restype = ctypes.c_int
         lib.griffin_index_destroy.restype = None
