@@ -247,6 +247,46 @@ griffin_status griffin_debug_intersect(griffin_index *ix, const uint32_t *terms,
                                        int mode, uint32_t *out_docids, uint64_t cap,
                                        uint64_t *count);
 
+/* ---- PforDelta comparator codec -------------------------
+ * The paper's comparison scheme (§2.1.1; Fig. 3), for
+ * bits/posting and decode-throughput comparisons with the EF index (Table 1,
+ * Fig. 12).  Not on the query path.  Same block layout rules as the
+ * EF index: blocks of block_size docIDs, per block an 8-B skip entry {first
+ * docID, payload offset / 16 B + packed n/words/b} and a 16-B aligned stream:
+ *   word 0: first exception position (n-1 if none) | n_exc << 10 | b << 20,
+ *   then n-1 d-gap slots of b bits (LSB-first; an exception's slot holds the
+ *   distance to the next exception minus one, the last 0), then the n_exc
+ *   exception gaps as u32, last exception first.  b = bits of the largest of the
+ *   ceil(0.9 (n-1)) smallest gaps; exceptions more than 2^b apart force one in
+ *   between (readings P1-P3).
+ * griffin_pfd_build validates like griffin_index_build (GRIFFIN_ERR_UNSORTED,
+ * INVALID_ARG) and encodes on `device` (-1 = current); the handle owns its
+ * device memory, freed by griffin_pfd_destroy.  Calls are synchronous. */
+typedef struct griffin_pfd griffin_pfd;
+typedef struct {
+  uint32_t block_size;
+  uint64_t num_blocks, num_postings;
+  uint64_t payload_bytes;   /* streams incl. 16-B padding */
+  uint64_t skip_bytes;      /* 8 B per block */
+  uint64_t exceptions;      /* exception slots, forced ones included */
+} griffin_pfd_stats_t;
+griffin_status griffin_pfd_build(const griffin_corpus *c, uint32_t block_size, int device,
+                                 griffin_pfd **out);
+void griffin_pfd_destroy(griffin_pfd *p);
+griffin_status griffin_pfd_stats(const griffin_pfd *p, griffin_pfd_stats_t *out);
+/* Logical stream words of block `block` of term `term` (host buffer of cap words). */
+griffin_status griffin_pfd_block_stream(griffin_pfd *p, uint32_t term, uint32_t block,
+                                        uint32_t *first, uint32_t *n, uint32_t *words,
+                                        uint32_t cap, uint32_t *nwords);
+/* Warp-per-block decode of term's whole list (host buffer of cap docIDs). */
+griffin_status griffin_pfd_decode_list(griffin_pfd *p, uint32_t term, uint32_t *out,
+                                       uint64_t cap, uint64_t *n);
+/* Decode-only sweep over every block (as griffin_debug_decode_all): mean device
+ * ms of `iters` timed sweeps after one warm-up, postings, bytes read (streams +
+ * skip entries) and the XOR of all decoded docIDs. */
+griffin_status griffin_pfd_decode_all(griffin_pfd *p, uint32_t iters, double *ms,
+                                      uint64_t *postings, uint64_t *bytes, uint64_t *checksum);
+
 #ifdef __cplusplus
 }
 #endif

@@ -97,6 +97,11 @@ _SIGS = {
     "griffin_set_profiling": [_vp, ctypes.c_int],
     "griffin_set_reuse": [_vp, ctypes.c_int],
     "griffin_set_nextgeq": [_vp, ctypes.c_int],
+    "griffin_pfd_build": [_vp, _u32, ctypes.c_int, _vp],
+    "griffin_pfd_stats": [_vp, _vp],
+    "griffin_pfd_block_stream": [_vp, _u32, _u32, _vp, _vp, _vp, _u32, _vp],
+    "griffin_pfd_decode_list": [_vp, _u32, _vp, _u64, _vp],
+    "griffin_pfd_decode_all": [_vp, _u32, _vp, _vp, _vp, _vp],
     "griffin_get_profile": [_vp, ctypes.POINTER(Profile)],
     "griffin_reset_profile": [_vp],
     "griffin_shard_range": [_u32, _u32, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u32)],
@@ -133,6 +138,9 @@ def load_library():
             fn.restype = ctypes.c_int
         lib.griffin_index_destroy.restype = None
         lib.griffin_workspace_destroy.restype = None
+        if hasattr(lib, "griffin_pfd_destroy"):
+            lib.griffin_pfd_destroy.restype = None
+            lib.griffin_pfd_destroy.argtypes = [_vp]
         lib.griffin_last_error.restype = ctypes.c_char_p
         lib.griffin_last_error.argtypes = []
         _lib = lib
@@ -364,6 +372,72 @@ class GriffinWorkspace:
         _check(load_library().griffin_workspace_sync_status(self.index.h, self.h))
 
 
-__all__ = ["GriffinIndex", "GriffinWorkspace", "GriffinError", "load_library", "griffin_last_error",
+class PfdStats(ctypes.Structure):
+    _fields_ = [("block_size", ctypes.c_uint32), ("num_blocks", ctypes.c_uint64),
+                ("num_postings", ctypes.c_uint64), ("payload_bytes", ctypes.c_uint64),
+                ("skip_bytes", ctypes.c_uint64), ("exceptions", ctypes.c_uint64)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class GriffinPfd:
+    """PforDelta-coded copy of a corpus' docID lists on the device (griffin_pfd_*,
+    the NEXT-3 comparator codec; not on the query path)."""
+
+    def __init__(self, corpus, block_size: int = 128, device: int = -1):
+        lib = load_library()
+        arrs = [np.ascontiguousarray(corpus.offsets, np.uint64),
+                np.ascontiguousarray(corpus.docids, np.uint32),
+                np.ascontiguousarray(corpus.tfs, np.uint32),
+                np.ascontiguousarray(corpus.doc_lengths, np.uint32)]
+        off, doc, tf, dl = arrs
+        c = _Corpus(corpus.num_docs, len(off) - 1, off.ctypes.data, doc.ctypes.data,
+                    tf.ctypes.data, dl.ctypes.data)
+        h = ctypes.c_void_p()
+        _check(lib.griffin_pfd_build(ctypes.byref(c), block_size, device, ctypes.byref(h)))
+        self.h = h
+        self.block_size = block_size
+
+    def close(self):
+        if getattr(self, "h", None) and _lib is not None:
+            _lib.griffin_pfd_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        self.close()
+
+    def griffin_pfd_stats(self) -> dict:
+        s = PfdStats()
+        _check(load_library().griffin_pfd_stats(self.h, ctypes.byref(s)))
+        return s.as_dict()
+
+    def griffin_pfd_block_stream(self, term: int, block: int):
+        """(first, n, stream words) of one block."""
+        cap = 4 * self.block_size + 16
+        w = np.zeros(cap, np.uint32)
+        f, n, nw = ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint32()
+        _check(load_library().griffin_pfd_block_stream(self.h, term, block, ctypes.byref(f),
+                                                       ctypes.byref(n), _ptr(w), cap,
+                                                       ctypes.byref(nw)))
+        return f.value, n.value, w[:nw.value].copy()
+
+    def griffin_pfd_decode_list(self, term: int, cap: int) -> np.ndarray:
+        out = np.zeros(max(cap, 1), np.uint32)
+        n = _u64()
+        _check(load_library().griffin_pfd_decode_list(self.h, term, _ptr(out), len(out),
+                                                      ctypes.byref(n)))
+        return out[:n.value]
+
+    def griffin_pfd_decode_all(self, iters: int = 3) -> dict:
+        ms = ctypes.c_double()
+        p, b, ck = _u64(), _u64(), _u64()
+        _check(load_library().griffin_pfd_decode_all(self.h, iters, ctypes.byref(ms),
+                                                     ctypes.byref(p), ctypes.byref(b),
+                                                     ctypes.byref(ck)))
+        return {"ms": ms.value, "postings": p.value, "bytes": b.value, "checksum": ck.value}
+
+
+__all__ = ["GriffinIndex", "GriffinWorkspace", "GriffinPfd", "GriffinError", "load_library", "griffin_last_error",
            "griffin_shard_range", "griffin_merge_path_split", "MODE_AUTO", "MODE_MERGE",
            "MODE_GALLOP", "LIB_PATH"]

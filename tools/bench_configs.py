@@ -5,6 +5,9 @@
                                           groups (Fig. 8 / Fig. 13 analog, GPU only)
   python tools/bench_configs.py c5 [nq]   10K-query top-1000 batch on the 50M-doc index +
                                           decode-only sweep over block sizes 64..512
+  python tools/bench_configs.py codecs [cfg]  EF vs PforDelta (NEXT-3): bits/posting and
+                                          decode-only sweep on the same lists (Table 1 /
+                                          Fig. 12 shape)
 
 Each prints JSON lines (one per measurement).  Timing: CUDA events on the
 launching stream for device-side numbers, perf_counter for host-API latency.
@@ -150,6 +153,34 @@ def c5(nq=None):
         ix.close()
 
 
+def codecs(cfg_name="c2"):
+    c, _, cfg = make_workload(cfg_name, num_queries=1)
+    for B in (128, 64, 256):
+        ix = g.GriffinIndex(c, block_size=B)
+        st = ix.griffin_index_stats()
+        ef_bytes = st["payload_bytes"] + st["skip_bytes"]
+        sw = ix.griffin_debug_decode_all(iters=5)
+        ix.close()
+        px = g.GriffinPfd(c, block_size=B)
+        ps = px.griffin_pfd_stats()
+        pf_bytes = ps["payload_bytes"] + ps["skip_bytes"]
+        pw = px.griffin_pfd_decode_all(iters=5)
+        px.close()
+        P = c.num_postings
+        line = {"config": cfg_name, "block_size": B, "postings": P,
+                "ef": {"bits_per_posting": 8 * ef_bytes / P, "compression_ratio": 32 * P / (8 * ef_bytes),
+                       "decode_ms": sw["ms"], "decode_gbs": sw["bytes"] / (sw["ms"] / 1e3) / 1e9,
+                       "gpostings_per_s": sw["postings"] / (sw["ms"] / 1e3) / 1e9},
+                "pfd": {"bits_per_posting": 8 * pf_bytes / P, "compression_ratio": 32 * P / (8 * pf_bytes),
+                        "exception_frac": ps["exceptions"] / max(1, P - ps["num_blocks"]),
+                        "decode_ms": pw["ms"], "decode_gbs": pw["bytes"] / (pw["ms"] / 1e3) / 1e9,
+                        "gpostings_per_s": pw["postings"] / (pw["ms"] / 1e3) / 1e9},
+                "paper_table1": {"pfd_ratio": 3.3, "ef_ratio": 4.6, "note": "ClueWeb12, CPU PforDelta"}}
+        line["ef_vs_pfd_size"] = pf_bytes / ef_bytes
+        line["ef_vs_pfd_decode_speed"] = pw["ms"] / sw["ms"]
+        print(json.dumps(line), flush=True)
+
+
 if __name__ == "__main__":
     which = sys.argv[1]
     if which == "c1":
@@ -158,3 +189,5 @@ if __name__ == "__main__":
         c3()
     elif which == "c5":
         c5(int(sys.argv[2]) if len(sys.argv) > 2 else None)
+    elif which == "codecs":
+        codecs(sys.argv[2] if len(sys.argv) > 2 else "c2")
