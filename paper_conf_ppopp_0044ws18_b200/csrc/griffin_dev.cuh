@@ -269,6 +269,117 @@ __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ 
   __syncwarp();
 }
 
+// ---- two blocks per warp (B = 128) ----------------------------------------------
+// The per-block fixed work of warp_decode_staged (prefix scan of the high words,
+// owner search, select) costs as much as its per-element work at B = 128; here
+// each half-warp runs the same algorithm on its own block with 16 lanes x 8
+// consecutive elements (width-16 shuffles), so one instruction stream decodes
+// two blocks.  Requires n <= 128 (hence hw <= 12 <= 16 high words) for both.
+// Block B is skipped when has_b is false.  dst pointers 16-B aligned.
+__device__ __forceinline__ void warp_decode_pair_staged(
+    const uint32_t *stg_a, uint32_t first_a, uint32_t y_a, uint32_t *dst_a,
+    const uint32_t *stg_b, uint32_t first_b, uint32_t y_b, uint32_t *dst_b, bool has_b,
+    uint32_t *__restrict__ cnt, const uint8_t *__restrict__ lut) {
+  const uint32_t lane = lane_id(), hf = lane >> 4, l = lane & 15u;
+  const bool act = hf == 0 || has_b;
+  const uint32_t *stg = hf ? stg_b : stg_a;
+  const uint32_t first = hf ? first_b : first_a;
+  const uint32_t y = hf ? y_b : y_a;
+  uint32_t *dst = hf ? dst_b : dst_a;
+  const uint32_t b = meta_b(y), n = act ? meta_n(y) : 0u, hw = act ? meta_hw(y) : 0u;
+  const uint32_t *hs = stg + low_words(n, b);
+  const uint32_t w0 = l < hw ? hs[l] : 0u;
+  const uint32_t c0 = __popc(w0);
+  uint32_t i0 = c0;
+#pragma unroll
+  for (int d = 1; d < 16; d <<= 1) {
+    const uint32_t t = __shfl_up_sync(0xffffffffu, i0, d, 16);
+    if (l >= (uint32_t)d) i0 += t;
+  }
+  // owner word of element k0 = 8l: mark + inclusive max-scan (as the E = 4 path)
+  const uint32_t ex0 = i0 - c0;
+  const uint32_t a = (ex0 + 7u) >> 3, bnd = (i0 + 7u) >> 3;
+  cnt[lane] = 0u;
+  __syncwarp();
+  if (l < hw && a < bnd && a < 16u) cnt[(hf << 4) + a] = l + 1u;
+  __syncwarp();
+  uint32_t v = cnt[lane];
+#pragma unroll
+  for (int d = 1; d < 16; d <<= 1) {
+    const uint32_t t = __shfl_up_sync(0xffffffffu, v, d, 16);
+    if (l >= (uint32_t)d) v = max(v, t);
+  }
+  const uint32_t w = v ? v - 1u : 0u;
+  const uint32_t src = (hf << 4) | (w & 15u);
+  const uint32_t x = __shfl_sync(0xffffffffu, w0, src);
+  const uint32_t ex = __shfl_sync(0xffffffffu, ex0, src);
+  uint32_t nx = __shfl_sync(0xffffffffu, w0, (src + 1u) & 31u);
+  if (w + 1u >= hw) nx = 0u;
+  const uint32_t k0 = l << 3;
+  if (k0 < n) {
+    const uint32_t ne = min(8u, n - k0);
+    const uint32_t pos = select_in_word(x, k0 - ex, lut);
+    const uint32_t p0 = (w << 5) + pos;
+    uint32_t win = __funnelshift_rc(x, nx, pos + 1u);
+    const uint32_t mask = b ? (0xFFFFFFFFu >> (32u - b)) : 0u;
+    if (ne == 8u && __popc(win) >= 7u) {
+      uint32_t hv[8];
+      hv[0] = p0 - k0;
+#pragma unroll
+      for (uint32_t j = 1; j < 8; ++j) {
+        const uint32_t t = __ffs(win);
+        win &= win - 1u;
+        hv[j] = p0 + t - (k0 + j);
+      }
+      uint32_t lv[8];
+      const uint32_t bp = k0 * b;
+      if (b <= 4u) {
+        const uint32_t lw32 = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp);
+#pragma unroll
+        for (uint32_t j = 0; j < 8; ++j) lv[j] = (lw32 >> (j * b)) & mask;
+      } else if (b <= 8u) {
+        const uint32_t q = bp + 4u * b;
+        const uint32_t w1 = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp);
+        const uint32_t w2 = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q);
+#pragma unroll
+        for (uint32_t j = 0; j < 4; ++j) {
+          lv[j] = (w1 >> (j * b)) & mask;
+          lv[j + 4] = (w2 >> (j * b)) & mask;
+        }
+      } else {
+#pragma unroll
+        for (uint32_t j = 0; j < 8; ++j) {
+          const uint32_t q = bp + j * b;
+          lv[j] = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
+        }
+      }
+      uint4 *o = reinterpret_cast<uint4 *>(dst + k0);
+      o[0] = make_uint4(first + ((hv[0] << b) | lv[0]), first + ((hv[1] << b) | lv[1]),
+                        first + ((hv[2] << b) | lv[2]), first + ((hv[3] << b) | lv[3]));
+      o[1] = make_uint4(first + ((hv[4] << b) | lv[4]), first + ((hv[5] << b) | lv[5]),
+                        first + ((hv[6] << b) | lv[6]), first + ((hv[7] << b) | lv[7]));
+    } else {
+      uint32_t wb = p0 + 1u;
+      uint32_t p = p0;
+      uint32_t bp = k0 * b;
+      for (uint32_t j = 0; j < ne; ++j) {
+        if (j) {
+          while (win == 0u) {
+            wb += 32u;
+            win = __funnelshift_r(hs[wb >> 5], hs[(wb >> 5) + 1], wb);
+          }
+          p = wb + (__ffs(win) - 1u);
+          win &= win - 1u;
+        }
+        const uint32_t lo_bits = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp) & mask;
+        dst[k0 + j] = first + (((p - (k0 + j)) << b) | lo_bits);
+        bp += b;
+      }
+    }
+  }
+  __syncwarp();
+}
+
 // ---- EF NextGEQ inside one staged block -------------------
 // Index of the first element >= x of the block staged at stg (n if none) and
 // its value in `val`, without decoding the block: the elements whose high part

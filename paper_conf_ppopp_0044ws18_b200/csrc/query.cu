@@ -270,6 +270,31 @@ __device__ __forceinline__ void stage_blocks(const DevIndex &ix, WarpSmem &w, ui
   w.phase ^= 1u;
 }
 
+// Decode the staged blocks whose (meta word y, first docID f, staged offset so in
+// 16-B units) sit in lanes [l0, l0+nb) into dst + i*B: two blocks per warp
+// instruction stream when B = 128 (warp_decode_pair_staged), else one.
+__device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t B, uint32_t l0,
+                                                    uint32_t nb, uint32_t y, uint32_t f,
+                                                    uint32_t so, uint32_t *dst) {
+  if (B == 128u) {
+    for (uint32_t i = 0; i < nb; i += 2) {
+      const uint32_t la = l0 + i, lb = (l0 + i + 1) & 31u;
+      const uint32_t ya = __shfl_sync(0xffffffffu, y, la), yb = __shfl_sync(0xffffffffu, y, lb);
+      const uint32_t fa = __shfl_sync(0xffffffffu, f, la), fb = __shfl_sync(0xffffffffu, f, lb);
+      const uint32_t sa = __shfl_sync(0xffffffffu, so, la), sb = __shfl_sync(0xffffffffu, so, lb);
+      warp_decode_pair_staged(w.stg + sa * 4u, fa, ya, dst + i * B, w.stg + sb * 4u, fb, yb,
+                              dst + (i + 1) * B, i + 1 < nb, w.cnt, w.lut);
+    }
+  } else {
+    for (uint32_t i = 0; i < nb; ++i) {
+      const uint32_t yi = __shfl_sync(0xffffffffu, y, l0 + i);
+      const uint32_t fi = __shfl_sync(0xffffffffu, f, l0 + i);
+      const uint32_t si = __shfl_sync(0xffffffffu, so, l0 + i);
+      warp_decode_staged(w.stg + si * 4u, fi, yi, dst + i * B, w.cnt, w.lut);
+    }
+  }
+}
+
 // EF-decode the consecutive blocks held by lanes [l0, l0+nb) (meta m, first f,
 // payload size sz in 16-B units; contiguous in the payload) into dst + i*B,
 // staging them with TMA bulk copies in batches that fit the staging area.
@@ -295,12 +320,7 @@ __device__ __forceinline__ void stage_decode_lanes(const DevIndex &ix, WarpSmem 
     }
     mbar_wait(w.mbar, w.phase);
     w.phase ^= 1u;
-    for (uint32_t k = 0; k < nbat; ++k) {
-      const uint32_t y = __shfl_sync(0xffffffffu, m.y, li + k);
-      const uint32_t fk = __shfl_sync(0xffffffffu, f, li + k);
-      const uint32_t so = __shfl_sync(0xffffffffu, m.x, li + k) - m0;
-      warp_decode_staged(w.stg + so * 4u, fk, y, dst + (i + k) * ix.B, w.cnt, w.lut);
-    }
+    decode_staged_lanes(w, ix.B, li, nbat, m.y, f, m.x - m0, dst + i * ix.B);
     i += nbat;
   }
 }
@@ -1016,22 +1036,8 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
       }
       // ---- EF-decode the compressed blocks into the smem tiles ----
       if (fit) {
-        if (rcomp) {
-          for (uint32_t i = 0; i < nRb; ++i) {
-            const uint32_t y = __shfl_sync(0xffffffffu, m.y, i);
-            const uint32_t fi = __shfl_sync(0xffffffffu, f, i);
-            const uint32_t so = __shfl_sync(0xffffffffu, soff, i);
-            warp_decode_staged(sm.stg + so * 4u, fi, y, sm.tile + i * B, sm.cnt, sm.lut);
-          }
-        }
-        if (!sdec) {
-          for (uint32_t i = 0; i < nSb; ++i) {
-            const uint32_t y = __shfl_sync(0xffffffffu, m.y, nRb + i);
-            const uint32_t fi = __shfl_sync(0xffffffffu, f, nRb + i);
-            const uint32_t so = __shfl_sync(0xffffffffu, soff, nRb + i);
-            warp_decode_staged(sm.stg + so * 4u, fi, y, tileS + i * B, sm.cnt, sm.lut);
-          }
-        }
+        if (rcomp) decode_staged_lanes(sm, B, 0, nRb, m.y, f, soff, sm.tile);
+        if (!sdec) decode_staged_lanes(sm, B, nRb, nSb, m.y, f, soff, tileS);
       } else {
         if (rcomp) stage_decode_lanes(ix, sm, cap16, 0, nRb, m, f, sz, sm.tile);
         if (!sdec) stage_decode_lanes(ix, sm, cap16, nRb, nSb, m, f, sz, tileS);
