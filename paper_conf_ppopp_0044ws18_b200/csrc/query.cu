@@ -209,8 +209,9 @@ __host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D) {
   // lists (<= 32*((D+2)*B/64+1) words) and always >= one worst-case block.
   return ((D + 2) * B / 2 + 64 + 3) & ~3u;
 }
-__host__ __device__ inline uint32_t warp_smem_words(uint32_t B, uint32_t D) {
-  return 8 + 64 + (B + 32) + stage_words(B, D) + (D + 2) * B;
+// with_tile = false: no decode tile (kernels that decode straight to HBM)
+__host__ __device__ inline uint32_t warp_smem_words(uint32_t B, uint32_t D, bool with_tile = true) {
+  return 8 + 64 + (B + 32) + stage_words(B, D) + (with_tile ? (D + 2) * B : 0u);
 }
 constexpr uint32_t kLutBytes = 2048;
 
@@ -221,17 +222,18 @@ struct WarpSmem {
   uint32_t phase;
 };
 
-__device__ __forceinline__ WarpSmem carve_warp_smem(uint4 *smem4, uint32_t B, uint32_t D) {
+__device__ __forceinline__ WarpSmem carve_warp_smem(uint4 *smem4, uint32_t B, uint32_t D,
+                                                    bool with_tile = true) {
   uint8_t *base = reinterpret_cast<uint8_t *>(smem4);
   WarpSmem w;
   w.lut = base;
   uint32_t *wb = reinterpret_cast<uint32_t *>(base + kLutBytes) +
-                 (threadIdx.x >> 5) * warp_smem_words(B, D);
+                 (threadIdx.x >> 5) * warp_smem_words(B, D, with_tile);
   w.mbar = reinterpret_cast<uint64_t *>(wb);   // words 0-1; 2: bump left; 4-5: bump offset
   w.cnt = wb + 8;
   w.aux = w.cnt + 64;
   w.stg = w.aux + B + 32;
-  w.tile = w.stg + stage_words(B, D);
+  w.tile = with_tile ? w.stg + stage_words(B, D) : nullptr;
   w.phase = 0;
   return w;
 }
@@ -1730,7 +1732,7 @@ __global__ void keys_to_results_kernel(uint32_t nq, uint32_t k, const uint64_t *
 // w.tile via one TMA bulk copy; returns total postings and payload bytes.
 __device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, uint32_t D,
                                                uint64_t k0, uint32_t nb, uint32_t *pay_bytes,
-                                               uint32_t *my_n = nullptr) {
+                                               uint32_t *my_n = nullptr, uint32_t *dst = nullptr) {
   const uint32_t lane = lane_id();
   uint2 m = make_uint2(0, 0);
   uint32_t f = 0, sz = 0;
@@ -1739,7 +1741,7 @@ __device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, 
     f = ix.first[k0 + lane];
     sz = block_size16(m.y);
   }
-  stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, w.tile);
+  stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, dst ? dst : w.tile);
   const uint32_t tot = __reduce_add_sync(0xffffffffu, lane < nb ? meta_n(m.y) : 0u);
   *pay_bytes = __reduce_add_sync(0xffffffffu, sz) * 16u;
   if (my_n) *my_n = lane < nb ? meta_n(m.y) : 0u;
@@ -1855,7 +1857,7 @@ __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t 
                                                           unsigned long long *scal) {
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
-  WarpSmem w = carve_warp_smem(smem4, ix.B, D);
+  WarpSmem w = carve_warp_smem(smem4, ix.B, D, false);
   cta_smem_init(smem4, w);
   const uint32_t V = ix.num_terms, run = D + 2, B = ix.B;
   const uint64_t total = run_base[V];
@@ -1869,11 +1871,8 @@ __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t 
     const uint32_t k0 = ri * run, nb = min(run, t.nblocks - k0);
     const uint64_t gb = (uint64_t)t.block0 + k0;
     uint32_t p;
-    const uint32_t n = decode_run(ix, w, D, gb, nb, &p);
-    const uint4 *src = reinterpret_cast<const uint4 *>(w.tile);
-    uint4 *dst = reinterpret_cast<uint4 *>(arena + gb * B);
-    for (uint32_t i = lane; i < nb * B / 4u; i += 32) dst[i] = src[i];
-    __syncwarp();
+    // decoded straight into the arena (128-bit stores, coalesced per half-warp)
+    const uint32_t n = decode_run(ix, w, D, gb, nb, &p, nullptr, arena + gb * B);
     if (lane == 0) {
       pay += p;
       post += n;
@@ -2060,7 +2059,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     run_map_kernel<<<(uint32_t)(((uint64_t)V * 32 + 255) / 256), 256, 0, st>>>(V, w.runs.as<uint32_t>(),
                                                     w.run_base.as<uint64_t>(),
                                                     w.run_term.as<uint32_t>());
-    const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * 8;
+    const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D, false) * 4 * 8;
     static thread_local int cfg_dev = -1;
     static thread_local size_t cfg_smem = 0;
     if (cfg_dev != ix->device || cfg_smem < smem) {
