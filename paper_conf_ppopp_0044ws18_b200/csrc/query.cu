@@ -278,17 +278,21 @@ __device__ __forceinline__ void stage_blocks(const DevIndex &ix, WarpSmem &w, ui
 __device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t B, uint32_t l0,
                                                     uint32_t nb, uint32_t y, uint32_t f,
                                                     uint32_t so, uint32_t *dst) {
-  if (B == 128u) {
-    for (uint32_t i = 0; i < nb; i += 2) {
+  uint32_t i0 = 0;
+  if (B == 128u) {   // pairs; an odd last block takes the single-block decoder
+    const uint32_t npair = nb & ~1u;
+    for (uint32_t i = 0; i < npair; i += 2) {
       const uint32_t la = l0 + i, lb = (l0 + i + 1) & 31u;
       const uint32_t ya = __shfl_sync(0xffffffffu, y, la), yb = __shfl_sync(0xffffffffu, y, lb);
       const uint32_t fa = __shfl_sync(0xffffffffu, f, la), fb = __shfl_sync(0xffffffffu, f, lb);
       const uint32_t sa = __shfl_sync(0xffffffffu, so, la), sb = __shfl_sync(0xffffffffu, so, lb);
       warp_decode_pair_staged(w.stg + sa * 4u, fa, ya, dst + i * B, w.stg + sb * 4u, fb, yb,
-                              dst + (i + 1) * B, i + 1 < nb, w.cnt, w.lut);
+                              dst + (i + 1) * B, true, w.cnt, w.lut);
     }
-  } else {
-    for (uint32_t i = 0; i < nb; ++i) {
+    i0 = npair;
+  }
+  {
+    for (uint32_t i = i0; i < nb; ++i) {
       const uint32_t yi = __shfl_sync(0xffffffffu, y, l0 + i);
       const uint32_t fi = __shfl_sync(0xffffffffu, f, l0 + i);
       const uint32_t si = __shfl_sync(0xffffffffu, so, l0 + i);
@@ -660,6 +664,93 @@ __device__ __forceinline__ void skip_blocks_sampled(const uint32_t *__restrict__
   __syncwarp();
 }
 
+// Arena probe (gallop / probe pass into a list decoded in the batch arena): each
+// R element x knows its S block kb (skip search: first[kb] <= x < first[kb+1]).
+// Docs are spread evenly enough inside a block that interpolation on the skip
+// range [first[kb], first[kb+1]) lands in or next to the right 8-key chunk (one
+// 32-B sector, 32-B aligned): load it, step one chunk left/right until x is
+// bracketed, then compare.  ~1-2 dependent sector loads per probe instead of
+// log2(B) for a binary search.  kEpl independent probes per lane run in
+// lockstep so their loads overlap.  Writes match[e] = kb*B + pos on a hit and
+// returns the number of chunks loaded.
+constexpr int kArenaEpl = 4;
+__device__ __forceinline__ uint32_t arena_probe_slice(const uint32_t *__restrict__ decS,
+                                                      const uint32_t *__restrict__ fS,
+                                                      uint32_t nblocksS, uint32_t dfS, uint32_t B,
+                                                      const uint32_t *tileR, const uint32_t *kidx,
+                                                      uint32_t *match, uint32_t base, uint32_t n) {
+  const uint32_t lane = lane_id();
+  uint32_t xv[kArenaEpl], kb[kArenaEpl], nb[kArenaEpl], c[kArenaEpl];
+  bool act[kArenaEpl];
+  uint32_t chunks = 0;
+#pragma unroll
+  for (int j = 0; j < kArenaEpl; ++j) {
+    const uint32_t e = base + lane + 32u * j;
+    act[j] = false;
+    kb[j] = kNone;
+    xv[j] = 0;
+    nb[j] = 0;
+    c[j] = 0;
+    if (e < n) {
+      kb[j] = kidx[e];
+      if (kb[j] != kNone) {
+        act[j] = true;
+        xv[j] = tileR[e];
+        nb[j] = min(B, dfS - kb[j] * B);
+      }
+    }
+  }
+  // interpolation estimate (the last block's upper end is its last element + 1)
+  uint32_t f0[kArenaEpl], f1[kArenaEpl];
+#pragma unroll
+  for (int j = 0; j < kArenaEpl; ++j) {
+    f0[j] = f1[j] = 0;
+    if (act[j]) {
+      f0[j] = __ldg(fS + kb[j]);
+      f1[j] = kb[j] + 1 < nblocksS ? __ldg(fS + kb[j] + 1)
+                                   : __ldg(decS + (size_t)kb[j] * B + nb[j] - 1) + 1u;
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < kArenaEpl; ++j) {
+    if (act[j]) {
+      const uint32_t span = f1[j] > f0[j] ? f1[j] - f0[j] : 1u;
+      uint32_t est = (uint32_t)(((uint64_t)(xv[j] - f0[j]) * nb[j]) / span);
+      est = min(est, nb[j] - 1u);
+      c[j] = est & ~7u;
+    }
+  }
+  for (;;) {
+    bool any = false;
+#pragma unroll
+    for (int j = 0; j < kArenaEpl; ++j) {
+      if (!act[j]) continue;
+      any = true;
+      ++chunks;
+      const uint4 *p = reinterpret_cast<const uint4 *>(decS + (size_t)kb[j] * B + c[j]);
+      const uint4 lo4 = __ldg(p), hi4 = __ldg(p + 1);
+      const uint32_t v[8] = {lo4.x, lo4.y, lo4.z, lo4.w, hi4.x, hi4.y, hi4.z, hi4.w};
+      const uint32_t valid = min(8u, nb[j] - c[j]);
+      uint32_t less = 0, eq = 0;
+#pragma unroll
+      for (uint32_t i = 0; i < 8; ++i) {
+        less += (i < valid && v[i] < xv[j]) ? 1u : 0u;
+        eq |= (i < valid && v[i] == xv[j]) ? 1u : 0u;
+      }
+      if (less == 0 && !eq && c[j] > 0) {
+        c[j] -= 8;                       // x lies before this chunk
+      } else if (less == valid && c[j] + 8u < nb[j]) {
+        c[j] += 8;                       // x lies after this chunk
+      } else {
+        if (eq) match[base + lane + 32u * j] = kb[j] * B + c[j] + less;
+        act[j] = false;
+      }
+    }
+    if (!__any_sync(0xffffffffu, any)) break;
+  }
+  return chunks;
+}
+
 // Multi-list probe (SvS rounds 2..m-1 in one pass): every round-1 survivor is
 // looked up in each remaining list in canonical order — skip-pointer search,
 // then an in-place binary search of the decoded-arena block or a staged EF
@@ -697,49 +788,13 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
     skip_blocks_sampled(fS, 0, tS.nblocks, tileR, n, kidx, match, sm.stg,
                         stage_words(B, D));
     if (sdec) {
-      // ---- decoded arena: in-place binary search of the touched block ----
+      // ---- decoded arena: interpolation probes of the touched block ----
       uint32_t probes = 0;
-      for (uint32_t base = 0; base < n; base += 128) {
-        uint32_t lo[4], hi[4], xv[4], kb[4], nb[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const uint32_t e = base + lane + 32u * j;
-          lo[j] = 0;
-          hi[j] = 0;
-          xv[j] = 0;
-          kb[j] = kNone;
-          nb[j] = 0;
-          if (e < n) {
-            kb[j] = kidx[e];
-            if (kb[j] != kNone) {
-              nb[j] = min(B, tS.df_local - kb[j] * B);
-              hi[j] = nb[j];
-              xv[j] = tileR[e];
-            }
-          }
-        }
-        for (;;) {
-          bool any = false;
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            if (lo[j] < hi[j]) {
-              const uint32_t mid = (lo[j] + hi[j]) >> 1;
-              if (__ldg(decS + (size_t)kb[j] * B + mid) < xv[j]) lo[j] = mid + 1; else hi[j] = mid;
-              any = true;
-              ++probes;
-            }
-          }
-          if (!__any_sync(0xffffffffu, any)) break;
-        }
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const uint32_t e = base + lane + 32u * j;
-          if (kb[j] != kNone && lo[j] < nb[j] && __ldg(decS + (size_t)kb[j] * B + lo[j]) == xv[j])
-            match[e] = kb[j] * B + lo[j];
-        }
-      }
+      for (uint32_t base = 0; base < n; base += 32u * kArenaEpl)
+        probes += arena_probe_slice(decS, fS, tS.nblocks, tS.df_local, B, tileR, kidx, match,
+                                    base, n);
       const uint32_t sp = __reduce_add_sync(0xffffffffu, probes);
-      if (lane == 0) acc.alg += sp * 4ull;
+      if (lane == 0) acc.alg += sp * 32ull;
     } else {
       // ---- compressed: distinct touched blocks, staged + decoded in groups ----
       uint32_t nd = 0, prev = kNone, e_first = n;
@@ -867,6 +922,7 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
   }
   __syncwarp();
 }
+
 
 template <bool RC>
 __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevIndex ix, RoundArgs a) {
@@ -1038,8 +1094,10 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
       }
       // ---- EF-decode the compressed blocks into the smem tiles ----
       if (fit) {
-        if (rcomp) decode_staged_lanes(sm, B, 0, nRb, m.y, f, soff, sm.tile);
-        if (!sdec) decode_staged_lanes(sm, B, nRb, nSb, m.y, f, soff, tileS);
+        // R and S tiles are contiguous: one pass over every compressed block
+        if (rcomp && !sdec) decode_staged_lanes(sm, B, 0, nRb + nSb, m.y, f, soff, sm.tile);
+        else if (rcomp) decode_staged_lanes(sm, B, 0, nRb, m.y, f, soff, sm.tile);
+        else if (!sdec) decode_staged_lanes(sm, B, nRb, nSb, m.y, f, soff, tileS);
       } else {
         if (rcomp) stage_decode_lanes(ix, sm, cap16, 0, nRb, m, f, sz, sm.tile);
         if (!sdec) stage_decode_lanes(ix, sm, cap16, nRb, nSb, m, f, sz, tileS);
@@ -1171,53 +1229,14 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
       }
       __syncwarp();
       if (sdec) {
-        // S decoded in the arena: each R element binary-searches its touched
-        // block in place (no staging); a lane's elements are independent chains,
-        // so their probes overlap (log2(B) dependent steps per unit).
-        constexpr int kEpl = 4;   // elements per lane per 128-element slice
+        // S decoded in the arena: interpolation probes of the touched block in
+        // place (no staging), kArenaEpl independent probes per lane in flight
         uint32_t probes = 0;
-        for (uint32_t base = 0; base < n; base += 128) {
-          uint32_t lo[kEpl], hi[kEpl], xv[kEpl], kb[kEpl];
-#pragma unroll
-          for (int j = 0; j < kEpl; ++j) {
-            const uint32_t e = base + lane + 32u * j;
-            lo[j] = 0;
-            hi[j] = 0;
-            xv[j] = 0;
-            kb[j] = kNone;
-            if (e < n) {
-              kb[j] = kidx[e];
-              if (kb[j] != kNone) {
-                hi[j] = min(B, tS.df_local - kb[j] * B);
-                xv[j] = tileR[e];
-              }
-            }
-          }
-          const uint32_t nb0 = hi[0], nb1 = hi[1], nb2 = hi[2], nb3 = hi[3];
-          for (;;) {
-            bool any = false;
-#pragma unroll
-            for (int j = 0; j < kEpl; ++j) {
-              if (lo[j] < hi[j]) {
-                const uint32_t mid = (lo[j] + hi[j]) >> 1;
-                if (__ldg(decS + (size_t)kb[j] * B + mid) < xv[j]) lo[j] = mid + 1; else hi[j] = mid;
-                any = true;
-                ++probes;
-              }
-            }
-            if (!__any_sync(0xffffffffu, any)) break;
-          }
-          const uint32_t nbs[kEpl] = {nb0, nb1, nb2, nb3};
-#pragma unroll
-          for (int j = 0; j < kEpl; ++j) {
-            const uint32_t e = base + lane + 32u * j;
-            if (kb[j] != kNone && lo[j] < nbs[j] &&
-                __ldg(decS + (size_t)kb[j] * B + lo[j]) == xv[j])
-              match[e] = kb[j] * B + lo[j];
-          }
-        }
+        for (uint32_t base = 0; base < n; base += 32u * kArenaEpl)
+          probes += arena_probe_slice(decS, fS, tS.nblocks, tS.df_local, B, tileR, kidx, match,
+                                      base, n);
         const uint32_t sp = __reduce_add_sync(0xffffffffu, probes);
-        if (lane == 0) acc.alg += sp * 4ull;
+        if (lane == 0) acc.alg += sp * 32ull;
         __syncwarp();
         if (RC)
           emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
