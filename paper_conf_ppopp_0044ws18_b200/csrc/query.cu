@@ -680,7 +680,7 @@ __device__ __forceinline__ uint32_t arena_probe_slice(const uint32_t *__restrict
                                                       const uint32_t *tileR, const uint32_t *kidx,
                                                       uint32_t *match, uint32_t base, uint32_t n) {
   const uint32_t lane = lane_id();
-  uint32_t xv[kArenaEpl], kb[kArenaEpl], nb[kArenaEpl], c[kArenaEpl];
+  uint32_t xv[kArenaEpl], kb[kArenaEpl], nb[kArenaEpl], c[kArenaEpl], dir[kArenaEpl];
   bool act[kArenaEpl];
   uint32_t chunks = 0;
 #pragma unroll
@@ -691,6 +691,7 @@ __device__ __forceinline__ uint32_t arena_probe_slice(const uint32_t *__restrict
     xv[j] = 0;
     nb[j] = 0;
     c[j] = 0;
+    dir[j] = 0;
     if (e < n) {
       kb[j] = kidx[e];
       if (kb[j] != kNone) {
@@ -737,10 +738,14 @@ __device__ __forceinline__ uint32_t arena_probe_slice(const uint32_t *__restrict
         less += (i < valid && v[i] < xv[j]) ? 1u : 0u;
         eq |= (i < valid && v[i] == xv[j]) ? 1u : 0u;
       }
-      if (less == 0 && !eq && c[j] > 0) {
+      // step toward x, never reversing: a reversal means x falls between two
+      // adjacent chunks, i.e. it is absent
+      if (less == 0 && !eq && c[j] > 0 && dir[j] != 2u) {
         c[j] -= 8;                       // x lies before this chunk
-      } else if (less == valid && c[j] + 8u < nb[j]) {
+        dir[j] = 1u;
+      } else if (less == valid && c[j] + 8u < nb[j] && dir[j] != 1u) {
         c[j] += 8;                       // x lies after this chunk
+        dir[j] = 2u;
       } else {
         if (eq) match[base + lane + 32u * j] = kb[j] * B + c[j] + less;
         act[j] = false;

@@ -2,7 +2,7 @@
 # GPU-box check: parity tests + bench; summaries printed at the end.
 TAG=${1:-x}
 mkdir -p gpurun_out
-timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/tests_$TAG.log 2>&1
+timeout 900 python -m pytest tests -m gpu -x -q -p no:cacheprovider --timeout 240 --timeout-method thread > gpurun_out/tests_$TAG.log 2>&1
 timeout 400 python bench.py --no-cpu-baseline > gpurun_out/bench_$TAG.json 2> gpurun_out/bench_$TAG.err
 echo "== tests: $(tail -1 gpurun_out/tests_$TAG.log)"
 grep -E "^(FAILED|E  )" gpurun_out/tests_$TAG.log | head -10
