@@ -140,6 +140,19 @@ __device__ __forceinline__ uint32_t select_in_word(uint32_t x, uint32_t r, const
   return sh + lut[((x >> sh) & 0xFFu) * 8u + (r - base)];
 }
 
+// ---- decoder output sinks -------------------------------------------------------
+// StoreSink writes decoded docIDs (smem tile or HBM arena); XorSink folds them
+// into a register checksum (the decode-only sweep: nothing is written back).
+struct StoreSink {
+  __device__ __forceinline__ void put4(uint32_t *p, uint4 v) { *reinterpret_cast<uint4 *>(p) = v; }
+  __device__ __forceinline__ void put(uint32_t *p, uint32_t v) { *p = v; }
+};
+struct XorSink {
+  uint32_t x = 0;
+  __device__ __forceinline__ void put4(uint32_t *, uint4 v) { x ^= v.x ^ v.y ^ v.z ^ v.w; }
+  __device__ __forceinline__ void put(uint32_t *, uint32_t v) { x ^= v; }
+};
+
 // ---- Elias-Fano block decode (Para-EF, §3.1.1 / Alg. 1) -------------
 // One warp decodes one block of n <= B postings, already staged in shared memory
 // (low stream: lw words, then high stream: hw words), into dst[0..n) as absolute
@@ -154,10 +167,11 @@ __device__ __forceinline__ uint32_t select_in_word(uint32_t x, uint32_t r, const
 //    find-first-set); h_k = p_k - k (the zeros before the k-th one);
 //    the b low bits are funnel-shifted out of the staged low stream.
 // `cnt` is per-warp smem scratch of >= 64 u32.
+template <class Sink>
 __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ stg, uint32_t first,
                                                    uint32_t y, uint32_t *__restrict__ dst,
                                                    uint32_t *__restrict__ cnt,
-                                                   const uint8_t *__restrict__ lut) {
+                                                   const uint8_t *__restrict__ lut, Sink &sink) {
   const uint32_t lane = lane_id();
   const uint32_t b = meta_b(y), n = meta_n(y), hw = meta_hw(y);
   const uint32_t lw = low_words(n, b);
@@ -243,9 +257,8 @@ __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ 
         q += b;
         l3 = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
       }
-      *reinterpret_cast<uint4 *>(dst + k0) =
-          make_uint4(first + ((h0 << b) | l0), first + ((h1 << b) | l1),
-                     first + ((h2 << b) | l2), first + ((h3 << b) | l3));
+      sink.put4(dst + k0, make_uint4(first + ((h0 << b) | l0), first + ((h1 << b) | l1),
+                                     first + ((h2 << b) | l2), first + ((h3 << b) | l3)));
     } else {
       // generic path: walk the ones with a 32-bit window, refilling when empty
       uint32_t wb = p0 + 1u;  // absolute bit position of win's bit 0
@@ -261,7 +274,7 @@ __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ 
           win &= win - 1u;
         }
         const uint32_t lo_bits = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp) & mask;
-        dst[k0 + j] = first + (((p - (k0 + j)) << b) | lo_bits);
+        sink.put(dst + k0 + j, first + (((p - (k0 + j)) << b) | lo_bits));
         bp += b;
       }
     }
@@ -276,10 +289,11 @@ __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ 
 // consecutive elements (width-16 shuffles), so one instruction stream decodes
 // two blocks.  Requires n <= 128 (hence hw <= 12 <= 16 high words) for both.
 // Block B is skipped when has_b is false.  dst pointers 16-B aligned.
+template <class Sink>
 __device__ __forceinline__ void warp_decode_pair_staged(
     const uint32_t *stg_a, uint32_t first_a, uint32_t y_a, uint32_t *dst_a,
     const uint32_t *stg_b, uint32_t first_b, uint32_t y_b, uint32_t *dst_b, bool has_b,
-    uint32_t *__restrict__ cnt, const uint8_t *__restrict__ lut) {
+    uint32_t *__restrict__ cnt, const uint8_t *__restrict__ lut, Sink &sink) {
   const uint32_t lane = lane_id(), hf = lane >> 4, l = lane & 15u;
   const bool act = hf == 0 || has_b;
   const uint32_t *stg = hf ? stg_b : stg_a;
@@ -353,11 +367,10 @@ __device__ __forceinline__ void warp_decode_pair_staged(
           lv[j] = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
         }
       }
-      uint4 *o = reinterpret_cast<uint4 *>(dst + k0);
-      o[0] = make_uint4(first + ((hv[0] << b) | lv[0]), first + ((hv[1] << b) | lv[1]),
-                        first + ((hv[2] << b) | lv[2]), first + ((hv[3] << b) | lv[3]));
-      o[1] = make_uint4(first + ((hv[4] << b) | lv[4]), first + ((hv[5] << b) | lv[5]),
-                        first + ((hv[6] << b) | lv[6]), first + ((hv[7] << b) | lv[7]));
+      sink.put4(dst + k0, make_uint4(first + ((hv[0] << b) | lv[0]), first + ((hv[1] << b) | lv[1]),
+                                     first + ((hv[2] << b) | lv[2]), first + ((hv[3] << b) | lv[3])));
+      sink.put4(dst + k0 + 4, make_uint4(first + ((hv[4] << b) | lv[4]), first + ((hv[5] << b) | lv[5]),
+                                         first + ((hv[6] << b) | lv[6]), first + ((hv[7] << b) | lv[7])));
     } else {
       uint32_t wb = p0 + 1u;
       uint32_t p = p0;
@@ -372,12 +385,20 @@ __device__ __forceinline__ void warp_decode_pair_staged(
           win &= win - 1u;
         }
         const uint32_t lo_bits = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp) & mask;
-        dst[k0 + j] = first + (((p - (k0 + j)) << b) | lo_bits);
+        sink.put(dst + k0 + j, first + (((p - (k0 + j)) << b) | lo_bits));
         bp += b;
       }
     }
   }
   __syncwarp();
+}
+
+__device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ stg, uint32_t first,
+                                                   uint32_t y, uint32_t *__restrict__ dst,
+                                                   uint32_t *__restrict__ cnt,
+                                                   const uint8_t *__restrict__ lut) {
+  StoreSink s;
+  warp_decode_staged(stg, first, y, dst, cnt, lut, s);
 }
 
 // ---- EF NextGEQ inside one staged block -------------------

@@ -275,9 +275,10 @@ __device__ __forceinline__ void stage_blocks(const DevIndex &ix, WarpSmem &w, ui
 // Decode the staged blocks whose (meta word y, first docID f, staged offset so in
 // 16-B units) sit in lanes [l0, l0+nb) into dst + i*B: two blocks per warp
 // instruction stream when B = 128 (warp_decode_pair_staged), else one.
+template <class Sink>
 __device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t B, uint32_t l0,
                                                     uint32_t nb, uint32_t y, uint32_t f,
-                                                    uint32_t so, uint32_t *dst) {
+                                                    uint32_t so, uint32_t *dst, Sink &sink) {
   uint32_t i0 = 0;
   if (B == 128u) {   // pairs; an odd last block takes the single-block decoder
     const uint32_t npair = nb & ~1u;
@@ -287,7 +288,7 @@ __device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t 
       const uint32_t fa = __shfl_sync(0xffffffffu, f, la), fb = __shfl_sync(0xffffffffu, f, lb);
       const uint32_t sa = __shfl_sync(0xffffffffu, so, la), sb = __shfl_sync(0xffffffffu, so, lb);
       warp_decode_pair_staged(w.stg + sa * 4u, fa, ya, dst + i * B, w.stg + sb * 4u, fb, yb,
-                              dst + (i + 1) * B, true, w.cnt, w.lut);
+                              dst + (i + 1) * B, true, w.cnt, w.lut, sink);
     }
     i0 = npair;
   }
@@ -296,17 +297,24 @@ __device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t 
       const uint32_t yi = __shfl_sync(0xffffffffu, y, l0 + i);
       const uint32_t fi = __shfl_sync(0xffffffffu, f, l0 + i);
       const uint32_t si = __shfl_sync(0xffffffffu, so, l0 + i);
-      warp_decode_staged(w.stg + si * 4u, fi, yi, dst + i * B, w.cnt, w.lut);
+      warp_decode_staged(w.stg + si * 4u, fi, yi, dst + i * B, w.cnt, w.lut, sink);
     }
   }
+}
+__device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t B, uint32_t l0,
+                                                    uint32_t nb, uint32_t y, uint32_t f,
+                                                    uint32_t so, uint32_t *dst) {
+  StoreSink s;
+  decode_staged_lanes(w, B, l0, nb, y, f, so, dst, s);
 }
 
 // EF-decode the consecutive blocks held by lanes [l0, l0+nb) (meta m, first f,
 // payload size sz in 16-B units; contiguous in the payload) into dst + i*B,
 // staging them with TMA bulk copies in batches that fit the staging area.
+template <class Sink>
 __device__ __forceinline__ void stage_decode_lanes(const DevIndex &ix, WarpSmem &w, uint32_t cap16,
                                                    uint32_t l0, uint32_t nb, uint2 m, uint32_t f,
-                                                   uint32_t sz, uint32_t *dst) {
+                                                   uint32_t sz, uint32_t *dst, Sink &sink) {
   const uint32_t lane = lane_id();
   const uint32_t incl = warp_incl_scan(lane >= l0 && lane < l0 + nb ? sz : 0u);
   uint32_t i = 0;
@@ -326,9 +334,15 @@ __device__ __forceinline__ void stage_decode_lanes(const DevIndex &ix, WarpSmem 
     }
     mbar_wait(w.mbar, w.phase);
     w.phase ^= 1u;
-    decode_staged_lanes(w, ix.B, li, nbat, m.y, f, m.x - m0, dst + i * ix.B);
+    decode_staged_lanes(w, ix.B, li, nbat, m.y, f, m.x - m0, dst + i * ix.B, sink);
     i += nbat;
   }
+}
+__device__ __forceinline__ void stage_decode_lanes(const DevIndex &ix, WarpSmem &w, uint32_t cap16,
+                                                   uint32_t l0, uint32_t nb, uint2 m, uint32_t f,
+                                                   uint32_t sz, uint32_t *dst) {
+  StoreSink s;
+  stage_decode_lanes(ix, w, cap16, l0, nb, m, f, sz, dst, s);
 }
 
 // Load R "block" k of an intermediate (chunk of B entries) into dst.
@@ -1754,9 +1768,11 @@ __global__ void keys_to_results_kernel(uint32_t nq, uint32_t k, const uint64_t *
 
 // Warp decodes the consecutive blocks [k0, k0+nb) (nb <= D+2) of the shard into
 // w.tile via one TMA bulk copy; returns total postings and payload bytes.
+template <class Sink = StoreSink>
 __device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, uint32_t D,
                                                uint64_t k0, uint32_t nb, uint32_t *pay_bytes,
-                                               uint32_t *my_n = nullptr, uint32_t *dst = nullptr) {
+                                               uint32_t *my_n = nullptr, uint32_t *dst = nullptr,
+                                               Sink *sink = nullptr) {
   const uint32_t lane = lane_id();
   uint2 m = make_uint2(0, 0);
   uint32_t f = 0, sz = 0;
@@ -1765,7 +1781,8 @@ __device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, 
     f = ix.first[k0 + lane];
     sz = block_size16(m.y);
   }
-  stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, dst ? dst : w.tile);
+  if (sink) stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, w.tile, *sink);
+  else stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, dst ? dst : w.tile);
   const uint32_t tot = __reduce_add_sync(0xffffffffu, lane < nb ? meta_n(m.y) : 0u);
   *pay_bytes = __reduce_add_sync(0xffffffffu, sz) * 16u;
   if (my_n) *my_n = lane < nb ? meta_n(m.y) : 0u;
@@ -1795,7 +1812,7 @@ __global__ void __launch_bounds__(256) decode_all_kernel(DevIndex ix, uint32_t D
                                                          unsigned long long *acc) {
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
-  WarpSmem w = carve_warp_smem(smem4, ix.B, D);
+  WarpSmem w = carve_warp_smem(smem4, ix.B, D, false);   // no tile: XorSink
   cta_smem_init(smem4, w);
   const uint32_t run = D + 2;
   const uint64_t nruns = (nblocks + run - 1) / run;
@@ -1807,15 +1824,11 @@ __global__ void __launch_bounds__(256) decode_all_kernel(DevIndex ix, uint32_t D
     const uint64_t k = r * run;
     const uint32_t nb = (uint32_t)((nblocks - k) < run ? (nblocks - k) : run);
     uint32_t p;
-    uint32_t mn;
-    const uint32_t n = decode_run(ix, w, D, k, nb, &p, &mn);
-    // blocks of a run may belong to different terms: only each term's last block
-    // is short, so XOR block by block
-    for (uint32_t bi = 0; bi < nb; ++bi) {
-      const uint32_t nbk = __shfl_sync(0xffffffffu, mn, bi);
-      for (uint32_t i = lane; i < nbk; i += 32) x ^= w.tile[bi * ix.B + i];
-    }
-    __syncwarp();
+    // decoded docIDs are folded into a register checksum by the decoder itself
+    // (XorSink): the sweep measures decoding, not a tile write + re-read
+    XorSink xs;
+    const uint32_t n = decode_run(ix, w, D, k, nb, &p, nullptr, nullptr, &xs);
+    x ^= xs.x;
     post += n;
     pay += p + 8u * nb;
   }
@@ -2223,7 +2236,7 @@ griffin_status launch_decode_list(griffin_index *ix, uint32_t term, uint32_t *d_
 
 griffin_status launch_decode_all(griffin_index *ix, unsigned long long *d_acc, cudaStream_t st) {
   if (!ix->nblocks) return GRIFFIN_OK;
-  const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * 8;
+  const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D, false) * 4 * 8;
   GRIFFIN_CUDA_TRY(cudaFuncSetAttribute(decode_all_kernel,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int per_sm = 0;

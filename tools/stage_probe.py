@@ -53,3 +53,7 @@ for name, setup in variants:
     print(json.dumps({"config": cfg_name, "variant": name,
                       "ms_per_batch": statistics.median(tot),
                       **{s: round(statistics.median(v), 4) for s, v in per.items()}}), flush=True)
+sw = ix.griffin_debug_decode_all(iters=5)
+print(json.dumps({"config": cfg_name, "decode_sweep_ms": sw["ms"],
+                  "gpostings_per_s": sw["postings"] / (sw["ms"] / 1e3) / 1e9,
+                  "gbs": sw["bytes"] / (sw["ms"] / 1e3) / 1e9}), flush=True)
