@@ -209,9 +209,12 @@ __host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D) {
   // lists (<= 32*((D+2)*B/64+1) words) and always >= one worst-case block.
   return ((D + 2) * B / 2 + 64 + 3) & ~3u;
 }
+// read slack after the tile: the uniform-trip merge loop may read up to L =
+// ceil((D+2)*B/32) words past a lane's segment (D <= 8 at B = 128 -> 40)
+constexpr uint32_t kTileSlack = 64;
 // with_tile = false: no decode tile (kernels that decode straight to HBM)
 __host__ __device__ inline uint32_t warp_smem_words(uint32_t B, uint32_t D, bool with_tile = true) {
-  return 8 + 64 + (B + 32) + stage_words(B, D) + (with_tile ? (D + 2) * B : 0u);
+  return 8 + 64 + (B + 32) + stage_words(B, D) + (with_tile ? (D + 2) * B + kTileSlack : 0u);
 }
 constexpr uint32_t kLutBytes = 2048;
 
@@ -416,14 +419,17 @@ __device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, co
 }
 
 // Ordered emission of per-lane match lists (merge units): lane l found c
-// matches, packed (R tile index | S tile index << 16) at ml[0..c); lanes are in
-// merge-path order, so a warp scan of the counts gives sorted output offsets.
+// matches, packed (R tile index | S tile index << 16) at ml0[l*cap ..+c); lanes
+// are in merge-path order, so the warp's j-th match overall is match
+// j - excl[s] of the lane s whose inclusive count first exceeds j.  The matches
+// are spread evenly over the lanes (4 per lane per pass, gathers issued
+// together so their latencies overlap) and written coalesced.
 // Round 1 (RC): s = w_R + w_S; later rounds: s = s_prev + w_S.
 template <bool RC>
 __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, const TermInfo &tR,
                            const TermInfo &tS, const uint2 *Rq, const uint32_t *tile,
-                           const uint32_t *ml, uint32_t c, uint32_t posR0, uint32_t posS0,
-                           Acc &acc) {
+                           const uint32_t *ml0, uint32_t cap, uint32_t c, uint32_t *scr,
+                           uint32_t posR0, uint32_t posS0, Acc &acc) {
   const uint32_t lane = lane_id();
   const uint32_t incl = warp_incl_scan(c);
   uint32_t cnt = __shfl_sync(0xffffffffu, incl, 31);
@@ -435,17 +441,22 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
     cnt = 0;
   }
   if (cnt) {
-    uint2 *dst = a.bump + off + (incl - c);
-    // gathers (norm, tf words, previous score) of up to 4 matches are issued
-    // together before any is consumed, so their latencies overlap
-    for (uint32_t j0 = 0; j0 < c; j0 += 4) {
+    scr[lane] = incl;
+    __syncwarp();
+    uint2 *dst = a.bump + off;
+    for (uint32_t j0 = 0; j0 < cnt; j0 += 128) {
       uint32_t doc[4], tS_[4], tR_[4], prev[4];
       float nrm[4];
 #pragma unroll
       for (int t = 0; t < 4; ++t) {
-        const uint32_t j = j0 + t;
-        if (j < c) {
-          const uint32_t e = ml[j];
+        const uint32_t j = j0 + 32u * t + lane;
+        if (j < cnt) {
+          uint32_t o = 0;   // owner lane: number of lanes with incl <= j
+#pragma unroll
+          for (uint32_t step = 16; step; step >>= 1)
+            if (scr[o + step - 1] <= j) o += step;
+          const uint32_t ex = o ? scr[o - 1] : 0u;
+          const uint32_t e = ml0[o * cap + (j - ex)];
           const uint32_t i = e & 0xFFFFu;
           doc[t] = tile[i];
           nrm[t] = __ldg(ix.norm + doc[t]);
@@ -456,8 +467,8 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
       }
 #pragma unroll
       for (int t = 0; t < 4; ++t) {
-        const uint32_t j = j0 + t;
-        if (j < c) {
+        const uint32_t j = j0 + 32u * t + lane;
+        if (j < cnt) {
           const float wS = bm25_w(tS.idf, tS_[t], nrm[t], ix.k1p1);
           float s;
           if (RC) {
@@ -470,6 +481,7 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
         }
       }
     }
+    __syncwarp();
   }
   if (lane == 0) {
     a.unit_off[u] = off;
@@ -1152,42 +1164,40 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
           ie = nr;
           je = ns;
         }
-        // branch-free serial merge: every step writes the candidate pair and
-        // keeps it only when x == y (no divergent branches in the hot loop).
-        // Each step advances at least one side, so min(remaining A, remaining B)
-        // steps can run without bound checks; re-check only between such runs.
-        // 32-bit shared addresses keep the step at ~12 instructions.
+        // branch-free serial merge with a warp-uniform trip count: every lane
+        // runs exactly L steps (its segment holds <= L merged elements and each
+        // step consumes >= 1, so the segment is covered).  Steps past the
+        // segment's end read the next lane's (still sorted) elements; a match
+        // counts only while the A index is inside the segment (pa < paE), and no
+        // in-segment element can equal an out-of-segment one (merge-path order +
+        // the A9 fix-up).  Every step writes the candidate pair and keeps it only
+        // on a match, so the loop has no divergent branch at all.
         uint32_t key = (ra + is) | (js << 16);   // R tile index | S tile index << 16
         uint32_t pa = smem_u32(A + is), pb = smem_u32(Bv + js);
+        const uint32_t paE = smem_u32(A + ie);
         const uint32_t pm0 = smem_u32(ml);
         uint32_t pm = pm0;
-        uint32_t ra_left = ie - is, rb_left = je - js;
-        for (;;) {
-          const uint32_t K = min(ra_left, rb_left);
-          if (K == 0) break;
-          const uint32_t pa0 = pa, pb0 = pb;
 #pragma unroll 4
-          for (uint32_t t = 0; t < K; ++t) {
-            uint32_t x, y;
-            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(pa));
-            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(y) : "r"(pb));
-            asm volatile("st.shared.u32 [%0], %1;" ::"r"(pm), "r"(key));
-            pm += (x == y) ? 4u : 0u;
-            const uint32_t da = (x <= y) ? 1u : 0u, db = (y <= x) ? 1u : 0u;
-            pa += da << 2;
-            pb += db << 2;
-            key += da + (db << 16);
-          }
-          ra_left -= (pa - pa0) >> 2;
-          rb_left -= (pb - pb0) >> 2;
+        for (uint32_t t = 0; t < L; ++t) {
+          uint32_t x, y;
+          asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(pa));
+          asm volatile("ld.shared.u32 %0, [%1];" : "=r"(y) : "r"(pb));
+          asm volatile("st.shared.u32 [%0], %1;" ::"r"(pm), "r"(key));
+          pm += (x == y && pa < paE) ? 4u : 0u;
+          const uint32_t da = (x <= y) ? 1u : 0u, db = (y <= x) ? 1u : 0u;
+          pa += da << 2;
+          pb += db << 2;
+          key += da + (db << 16);
         }
         c = (pm - pm0) >> 2;
       }
       __syncwarp();
       if (RC)
-        emit_lanes<true>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, ml, c, rb0 * B, sb0 * B + sa, acc);
+        emit_lanes<true>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, sm.stg, cap, c, sm.cnt, rb0 * B,
+                         sb0 * B + sa, acc);
       else
-        emit_lanes<false>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, ml, c, rb0 * B, sb0 * B + sa, acc);
+        emit_lanes<false>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, sm.stg, cap, c, sm.cnt, rb0 * B,
+                          sb0 * B + sa, acc);
       __syncwarp();
     } else {
       // ---- gallop: R chunk lu, skip-pointer search into S (Fig. 9) ----
