@@ -340,7 +340,7 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
 static uint64_t ws_identity(const Workspace &w) {
   uint64_t h = 1469598103934665603ull;
   for (const DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel,
-                          &w.qmode, &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec,
+                          &w.qmode, &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.uperm,
                           &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys,
                           &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand,
                           &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.run_term, &w.arena})
@@ -493,7 +493,7 @@ griffin_status griffin_workspace_create(griffin_index *ix, griffin_workspace **o
 
 static void free_workspace(Workspace &w) {
   for (DevBuf *b : {&w.plan_terms, &w.plan_m, &w.cap, &w.cap_off, &w.rcount, &w.rsel, &w.qmode,
-                    &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.rbuf0,
+                    &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.uperm, &w.rbuf0,
                     &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys, &w.counts,
                     &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand, &w.tdec, &w.runs,
                     &w.run_base, &w.vtmp, &w.run_term, &w.arena})

@@ -54,7 +54,7 @@ struct DevBuf {
 // Query workspace (all grow-only; sized by griffin_reserve / the host API).
 struct Workspace {
   DevBuf plan_terms, plan_m, cap, cap_off, rcount, rsel, qmode, unit_base;  // per query
-  DevBuf unit_off, unit_cnt, unit_dst, urec;                                // per unit
+  DevBuf unit_off, unit_cnt, unit_dst, urec, uperm;                         // per unit
   DevBuf rbuf0, rbuf1, bump, cand, tkstate;                                 // per survivor
   DevBuf scal;       // scalars: counters, status, bump ctr, unit ctr
   DevBuf keys, counts, docids, scores, qoffs, qterms;  // host-API staging on device
@@ -74,7 +74,8 @@ enum : int {
   kScalStatus = 6,    // int status
   kScalTotals = 7,    // u64 x2: sum cap, sum units (written by plan kernels)
   kScalDec = 10,      // 3 x u64: decode-once alg bytes, payload bytes, postings
-  kScalCount = 13
+  kScalPerm = 13,     // 2 x u64: unit order list head (merge units) / tail (the rest)
+  kScalCount = 15
 };
 
 constexpr uint32_t kBumpChunk = 256;   // bump-area entries grabbed per warp atomic
@@ -102,6 +103,7 @@ struct RoundArgs {
   uint64_t bump_cap;      // entries of the bump area (entry_cap + per-warp chunk slack)
   unsigned long long *scal;
   uint4 *urec;            // per unit: {q, i0|lu, j0, lo docID} (partition stage)
+  uint32_t *uperm;        // processing order of the units: merge units first, then the rest
   const uint32_t *dec;    // batch decoded arena (global block * B + i), or null
   const uint8_t *tdec;    // per term: 1 = decoded in the arena this batch
 };

@@ -127,6 +127,8 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
   if (q == 0) {
     a.scal[kScalBump] = 0;
     a.scal[kScalUnitCtr] = 0;
+    a.scal[kScalPerm] = 0;
+    a.scal[kScalPerm + 1] = 0;
     if (overflow) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
   }
   if (q >= a.nq) return;
@@ -539,6 +541,9 @@ __device__ __forceinline__ void warp_mp_search2(HR hR, uint32_t nbR, HS hS, uint
 // and the unit's first docID.  The merging stage reads {q, i0, j0, lo} of unit u
 // and of unit u+1 (its end), so no warp ever searches on the critical path.
 template <bool RC>
+__device__ __forceinline__ void unit_record(const DevIndex &ix, const RoundArgs &a, uint64_t u);
+
+template <bool RC>
 __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
   const uint64_t total = a.unit_base[a.nq];
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -547,6 +552,36 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
       a.urec[u] = make_uint4(kNone, 0, 0, 0);
       continue;
     }
+    unit_record<RC>(ix, a, u);
+  }
+  // Processing order: merge units first, then gallop/probe/single-term units,
+  // so that at any time the warps mostly run one unit kind's code (the kernel
+  // is instruction-cache bound).  Output placement depends only on unit ids,
+  // so the (atomic, unordered) list does not affect results.
+  for (uint64_t base = blockIdx.x * (uint64_t)blockDim.x; base < total; base += stride) {
+    const uint64_t u = base + threadIdx.x;
+    const bool valid = u < total;
+    uint32_t q = 0;
+    if (valid) q = a.urec[u].x;
+    const bool mg = valid && a.qmode[q] == kModeMerge;
+    const uint32_t bm = __ballot_sync(0xffffffffu, mg), bo = __ballot_sync(0xffffffffu, valid && !mg);
+    const uint32_t lane = threadIdx.x & 31u, lt = (1u << lane) - 1u;
+    unsigned long long hm = 0, ho = 0;
+    if (lane == 0) {
+      if (bm) hm = atomicAdd(a.scal + kScalPerm, (unsigned long long)__popc(bm));
+      if (bo) ho = atomicAdd(a.scal + kScalPerm + 1, (unsigned long long)__popc(bo));
+    }
+    hm = __shfl_sync(0xffffffffu, hm, 0);
+    ho = __shfl_sync(0xffffffffu, ho, 0);
+    if (mg) a.uperm[hm + __popc(bm & lt)] = (uint32_t)u;
+    else if (valid) a.uperm[total - 1 - (ho + __popc(bo & lt))] = (uint32_t)u;
+  }
+}
+
+// Partition-stage record of unit u (see partition_kernel).
+template <bool RC>
+__device__ __forceinline__ void unit_record(const DevIndex &ix, const RoundArgs &a, uint64_t u) {
+  {
     uint32_t lo = 0, hi = a.nq;
     while (hi - lo > 1) {
       const uint32_t mid = (lo + hi) >> 1;
@@ -978,9 +1013,10 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
   if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
   (void)nwarps;
   for (;;) {
-    const uint64_t u = __shfl_sync(0xffffffffu, ticket, 0);
-    if (u >= total) break;
+    const uint64_t tk = __shfl_sync(0xffffffffu, ticket, 0);
+    if (tk >= total) break;
     if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
+    const uint64_t u = a.uperm[tk];   // merge units first (see partition_kernel)
     const uint4 rec = a.urec[u];
     const uint4 nxt = a.urec[u + 1];
     const uint32_t q = rec.x;
@@ -1124,26 +1160,47 @@ __global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevInde
         }
       }
       // ---- EF-decode the compressed blocks into the smem tiles ----
+      // (one call site per decoder path: every inlined copy of the decoders
+      // costs ~5 KB of SASS, and the kernel is instruction-cache bound)
       if (fit) {
         // R and S tiles are contiguous: one pass over every compressed block
-        if (rcomp && !sdec) decode_staged_lanes(sm, B, 0, nRb + nSb, m.y, f, soff, sm.tile);
-        else if (rcomp) decode_staged_lanes(sm, B, 0, nRb, m.y, f, soff, sm.tile);
-        else if (!sdec) decode_staged_lanes(sm, B, nRb, nSb, m.y, f, soff, tileS);
+        const uint32_t l0 = rcomp ? 0u : nRb;
+        const uint32_t nbd = (rcomp ? nRb : 0u) + (sdec ? 0u : nSb);
+        if (nbd) decode_staged_lanes(sm, B, l0, nbd, m.y, f, soff, rcomp ? sm.tile : tileS);
       } else {
-        if (rcomp) stage_decode_lanes(ix, sm, cap16, 0, nRb, m, f, sz, sm.tile);
-        if (!sdec) stage_decode_lanes(ix, sm, cap16, nRb, nSb, m, f, sz, tileS);
+#pragma unroll 1
+        for (uint32_t jb = 0; jb < 2; ++jb) {
+          if (jb == 0 ? rcomp : !sdec)
+            stage_decode_lanes(ix, sm, cap16, jb ? nRb : 0u, jb ? nSb : nRb, m, f, sz,
+                               jb ? tileS : sm.tile);
+        }
       }
       __syncwarp();
-      // ranges inside [lo, hi)
-      // lanes 0-3 search (R, lo), (R, hi), (S, lo), (S, hi) in one converged loop
-      uint32_t r_lo = 0;
+      // ranges inside [lo, hi): four lower_bounds — (R, lo), (R, hi), (S, lo),
+      // (S, hi) — each by an 8-lane group doing an 8-ary search (7 probes per
+      // step, ballot + popc), ~log8 dependent smem loads instead of log2
+      uint32_t r_lo;
       {
-        const uint32_t *arr = lane < 2 ? sm.tile : tileS;
-        const uint64_t key = (lane & 1) ? hi_v : lo_v;
-        r_lo = lower_bound_s(arr, 0, lane < 2 ? nRt : (lane < 4 ? nSt : 0u), key);
+        const uint32_t g = lane >> 3, sub = lane & 7u;
+        const uint32_t *arr = g < 2 ? sm.tile : tileS;
+        const uint64_t key = (g & 1) ? hi_v : lo_v;
+        const uint32_t gmask = 0xFFu << (g * 8u);
+        uint32_t lo = 0, hi = g < 2 ? nRt : nSt;   // answer in [lo, hi]
+        while (__any_sync(0xffffffffu, lo < hi)) {
+          const uint32_t step = (hi - lo + 8u) >> 3;   // 8 steps cover the hi-lo+1 candidates
+          const uint32_t qp = lo + (sub + 1u) * step - 1u;
+          const bool pr = lo < hi && sub < 7u && qp < hi && (uint64_t)arr[qp] < key;
+          const uint32_t c = __popc(__ballot_sync(0xffffffffu, pr) & gmask);
+          if (lo < hi) {
+            const uint32_t nlo = lo + c * step;
+            hi = min(hi, lo + (c + 1u) * step - 1u);
+            lo = nlo;
+          }
+        }
+        r_lo = lo;
       }
-      const uint32_t ra = __shfl_sync(0xffffffffu, r_lo, 0), rb = __shfl_sync(0xffffffffu, r_lo, 1);
-      const uint32_t sa = __shfl_sync(0xffffffffu, r_lo, 2), sb = __shfl_sync(0xffffffffu, r_lo, 3);
+      const uint32_t ra = __shfl_sync(0xffffffffu, r_lo, 0), rb = __shfl_sync(0xffffffffu, r_lo, 8);
+      const uint32_t sa = __shfl_sync(0xffffffffu, r_lo, 16), sb = __shfl_sync(0xffffffffu, r_lo, 24);
       const uint32_t nr = rb - ra, ns = sb - sa;
       const uint32_t tot2 = nr + ns, L = (tot2 + 31) >> 5;
       const uint32_t cap = (L >> 1) + 2;           // matches per lane <= ceil(L/2), +1 slack write
@@ -1960,6 +2017,7 @@ griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t
   GRIFFIN_CUDA_TRY(w.unit_off.reserve((units + 1) * 8));
   GRIFFIN_CUDA_TRY(w.unit_cnt.reserve((units + 1) * 4));
   GRIFFIN_CUDA_TRY(w.urec.reserve((units + 2) * 16));
+  GRIFFIN_CUDA_TRY(w.uperm.reserve((units + 2) * 4));
   GRIFFIN_CUDA_TRY(w.unit_dst.reserve((units + 2) * 8 + (units / kScanTile + 2) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf0.reserve((entries + 1) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf1.reserve((entries + 1) * 8));
@@ -2062,6 +2120,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
   ra.unit_off = w.unit_off.as<uint64_t>();
   ra.unit_cnt = w.unit_cnt.as<uint32_t>();
   ra.urec = w.urec.as<uint4>();
+  ra.uperm = w.uperm.as<uint32_t>();
   ra.unit_cap = w.unit_cap;
   ra.bump = w.bump.as<uint2>();
   ra.entry_cap = w.entry_cap;
