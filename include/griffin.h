@@ -210,6 +210,12 @@ griffin_status griffin_set_reuse(griffin_index *ix, int mode);
  * §8(f) NEXT-1), 0 = decode every touched block (Para-EF) and binary-search it.
  * Results are identical; only the work differs.  Invalid value -> INVALID_ARG. */
 griffin_status griffin_set_nextgeq(griffin_index *ix, int on);
+/* Probe pass (SvS rounds 2..m-1, one multi-list pass over the round-1
+ * survivors): survivors per work unit, a multiple of 32 in [32, block_size];
+ * 0 restores the default (block_size / 2, at least 32).  Smaller chunks give more, shorter
+ * units (more parallelism when few survivors remain).  Results are identical.
+ * Invalid value -> INVALID_ARG. */
+griffin_status griffin_set_probe_chunk(griffin_index *ix, uint32_t chunk);
 griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out); /* syncs */
 griffin_status griffin_reset_profile(griffin_index *ix);
 const char *griffin_last_error(void);

@@ -97,6 +97,7 @@ _SIGS = {
     "griffin_set_profiling": [_vp, ctypes.c_int],
     "griffin_set_reuse": [_vp, ctypes.c_int],
     "griffin_set_nextgeq": [_vp, ctypes.c_int],
+    "griffin_set_probe_chunk": [_vp, _u32],
     "griffin_pfd_build": [_vp, _u32, ctypes.c_int, _vp],
     "griffin_pfd_stats": [_vp, _vp],
     "griffin_pfd_block_stream": [_vp, _u32, _u32, _vp, _vp, _vp, _u32, _vp],
@@ -284,6 +285,10 @@ class GriffinIndex:
     def griffin_set_nextgeq(self, on: bool):
         """Gallop into compressed lists by EF NextGEQ (True, default) or block decode."""
         _check(load_library().griffin_set_nextgeq(self.h, int(on)))
+
+    def griffin_set_probe_chunk(self, chunk: int):
+        """Probe-pass survivors per unit (multiple of 32 in [32, B]; 0 = B)."""
+        _check(load_library().griffin_set_probe_chunk(self.h, chunk))
 
     def griffin_set_profiling(self, on: bool):
         _check(load_library().griffin_set_profiling(self.h, int(on)))

@@ -595,6 +595,19 @@ griffin_status griffin_set_nextgeq(griffin_index *ix, int on) {
   return GRIFFIN_OK;
 }
 
+griffin_status griffin_set_probe_chunk(griffin_index *ix, uint32_t chunk) {
+  if (!ix) return invalid("null index");
+  if (chunk != 0 && (chunk < 32 || chunk > ix->B || chunk % 32 != 0))
+    return invalid("probe chunk must be 0 or a multiple of 32 in [32, block_size]");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  if (ix->P != chunk) {   // captured single-query graphs bake the option in
+    for (auto &g : ix->graphs) cudaGraphExecDestroy(g.exec);
+    ix->graphs.clear();
+  }
+  ix->P = chunk;
+  return GRIFFIN_OK;
+}
+
 griffin_status griffin_set_profiling(griffin_index *ix, int on) {
   if (!ix) return invalid("null index");
   std::lock_guard<std::mutex> lk(ix->mu);

@@ -97,10 +97,10 @@ __global__ void plan_queries_kernel(DevIndex ix, uint32_t nq, const uint32_t *__
   rsel[q] = 0;
 }
 
-// Σ cap and Σ unit bounds (bound = nblocks(t0) + max_r nblocks(t_r)), checked
-// against the reserved workspace before any round runs.
+// Σ cap and Σ unit bounds (bound = nblocks(t0) + max(max_r nblocks(t_r),
+// ceil(cap / P))), checked against the reserved workspace before any round runs.
 __global__ void plan_totals_kernel(DevIndex ix, uint32_t nq, const uint32_t *plan_terms,
-                                   const uint32_t *plan_m, const uint32_t *cap,
+                                   const uint32_t *plan_m, const uint32_t *cap, uint32_t P,
                                    unsigned long long *scal) {
   unsigned long long c = 0, u = 0;
   for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < nq; q += gridDim.x * blockDim.x) {
@@ -109,6 +109,7 @@ __global__ void plan_totals_kernel(DevIndex ix, uint32_t nq, const uint32_t *pla
     c += cap[q];
     uint32_t mx = 0;
     for (uint32_t i = 1; i < m; ++i) mx = max(mx, ix.terms[plan_terms[q * kMaxTerms + i]].nblocks);
+    if (m >= 3) mx = max(mx, (cap[q] + P - 1) / P);   // probe pass
     u += (unsigned long long)ix.terms[plan_terms[q * kMaxTerms]].nblocks + mx;
   }
   for (int d = 16; d; d >>= 1) {
@@ -153,7 +154,7 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
       nbR = (uint32_t)((nR + ix.B - 1) / ix.B);
       if (a.probe) {   // rounds 2..m-1 as one multi-list probe pass
         mode = kModeProbe;
-        units = nbR;
+        units = (uint32_t)((nR + a.pchunk - 1) / a.pchunk);
       } else {
         pair = true;
       }
@@ -835,8 +836,8 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
   uint32_t *tileR = sm.tile, *sc = sm.tile + B, *nrm = sm.tile + 2 * B, *kidx = sm.tile + 3 * B;
   uint32_t *match = sm.tile + 4 * B, *tileS = sm.tile + 5 * B;
   uint32_t *dblk = sm.aux, *sn = sm.aux + B;
-  const uint32_t s0 = lu * B;
-  uint32_t n = min(B, nR - s0);
+  const uint32_t s0 = lu * a.pchunk;
+  uint32_t n = min(a.pchunk, nR - s0);
   for (uint32_t e = lane; e < n; e += 32) {
     const uint2 v = Rq[s0 + e];
     tileR[e] = v.x;
@@ -851,7 +852,12 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
     const uint32_t *fS = ix.first + tS.block0;
     const bool sdec = a.tdec && a.tdec[sid];
     const uint32_t *decS = sdec ? a.dec + (size_t)tS.block0 * B : nullptr;
-    skip_blocks_sampled(fS, 0, tS.nblocks, tileR, n, kidx, match, sm.stg,
+    // skip pointers this chunk can touch: [ub(first survivor) - 1, ub(last)),
+    // found by a warp-cooperative 16-ary search; a chunk usually spans few
+    // enough of them to be searched from one coalesced smem window
+    uint32_t k0, k1;
+    warp_upper_bound2(fS, tS.nblocks, tileR[0], tileR[n - 1], &k0, &k1);
+    skip_blocks_sampled(fS, k0 ? k0 - 1u : 0u, k1, tileR, n, kidx, match, sm.stg,
                         stage_words(B, D));
     if (sdec) {
       // ---- decoded arena: interpolation probes of the touched block ----
@@ -2135,7 +2141,8 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
                                                  w.rcount.as<uint32_t>(), w.rsel.as<uint8_t>(), scal);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
     plan_totals_kernel<<<std::min<unsigned>(qblocks, 1024), 256, 0, st>>>(
-        di, nq, w.plan_terms.as<uint32_t>(), w.plan_m.as<uint32_t>(), w.cap.as<uint32_t>(), scal);
+        di, nq, w.plan_terms.as<uint32_t>(), w.plan_m.as<uint32_t>(), w.cap.as<uint32_t>(),
+        probe_chunk(ix), scal);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
     GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(w.cap.as<uint32_t>(), w.cap_off.as<uint64_t>(), nq,
                                               scan_tmp, st, &ix->launch_count));
@@ -2187,6 +2194,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
   // multi-list probe replaces SvS rounds 2..m-1 (auto mode, B small enough for its smem)
   ra.probe = forced_mode == 0 && ix->probe && ix->D >= 5;
   ra.nextgeq = ix->nextgeq;
+  ra.pchunk = probe_chunk(ix);
   uint32_t rounds = std::max<uint32_t>(1, max_terms > 0 ? max_terms - 1 : 1);
   if (ra.probe) rounds = std::min<uint32_t>(rounds, 2);
   for (uint32_t r = 1; r <= rounds; ++r) {
@@ -2365,6 +2373,8 @@ void host_query_bounds(const griffin_index *ix, const uint32_t *terms, uint32_t 
   *cap = std::min(t0.df_local, ix->h_terms[ts[1]].df_local);
   uint32_t mx = 0;
   for (size_t i = 1; i < ts.size(); ++i) mx = std::max(mx, ix->h_terms[ts[i]].nblocks);
+  const uint32_t P = probe_chunk(ix);   // probe-pass units: ceil(|R| / P), |R| <= cap
+  if (ts.size() >= 3) mx = std::max<uint32_t>(mx, (uint32_t)((*cap + P - 1) / P));
   *units = (uint64_t)t0.nblocks + mx;
 }
 

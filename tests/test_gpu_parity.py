@@ -139,6 +139,24 @@ def test_query_batch_forced_modes(tiny, mode):
     assert_topk_equal(gd, gs, gc, od, os_, oc)
 
 
+@pytest.mark.parametrize("chunk", [32, 64, 96])
+def test_probe_chunk_sizes(tiny, chunk):
+    """Probe-pass units of `chunk` survivors give the same results (incl. the
+    single-query graph path, whose capture bakes the option in)."""
+    c, ql, ox = tiny
+    gx = g.GriffinIndex(c, block_size=128)
+    gx.griffin_set_probe_chunk(chunk)
+    od, os_, oc = ox.query_batch(ql, 10)
+    gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 10)
+    assert_topk_equal(gd, gs, gc, od, os_, oc)
+    for q in range(min(ql.num_queries, 8)):
+        d1, s1, c1 = ox.query(ql.query(q), 10)
+        d2, s2, c2 = gx.griffin_query(ql.query(q), 10)
+        assert_topk_equal(d2, s2, c2, d1, s1, c1)
+    with pytest.raises(Exception):
+        gx.griffin_set_probe_chunk(48)
+
+
 def test_c1_single_query():
     c, ql, cfg = make_workload("c1")
     ox = oracle.OracleIndex(c, block_size=128)

@@ -28,7 +28,8 @@ stages = ("ms_plan", "ms_decode", "ms_intersect", "ms_compact", "ms_topk")
 variants = [("default", lambda: None)]
 for extra in sys.argv[2:]:
     name, val = extra.split("=")
-    variants.append((extra, lambda n=name, v=int(val): getattr(ix, "griffin_set_" + n)(v)))
+    variants.append((extra, lambda n=name, v=int(val): (getattr(ix, "griffin_set_" + n)(v),
+                                                        ix.griffin_reserve(ql.offsets, ql.terms, k))))
 for name, setup in variants:
     setup()
     for _ in range(5):
