@@ -1528,12 +1528,7 @@ __global__ void __launch_bounds__(256) compact_copy_kernel(RoundArgs a, const ui
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); u < total;
        u += nwarps) {
-    uint32_t lo = 0, hi = a.nq;
-    while (hi - lo > 1) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if (ubase[mid] <= u) lo = mid; else hi = mid;
-    }
-    const uint32_t q = lo;
+    const uint32_t q = a.urec[u].x;   // the partition stage's record
     const uint64_t base = udst[ubase[q]];
     const uint64_t my = udst[u];
     const uint32_t cnt = a.unit_cnt[u];
