@@ -11,14 +11,14 @@ rep, idx = sys.argv[1], int(sys.argv[2])
 out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass",
                       "--launch-skip", str(idx), "--launch-count", "1"], capture_output=True,
                      text=True).stdout
-REG = {'merge_loop': ('query.cu', 1153, 1195), 'fine_split': ('griffin_dev.cuh', 500, 516),
-       'emit_lanes': ('query.cu', 428, 496), 'emit_unit': ('query.cu', 359, 427),
-       'tf/bm25': ('griffin_dev.cuh', 458, 476), 'decoders': ('griffin_dev.cuh', 143, 410),
-       'nextgeq': ('griffin_dev.cuh', 411, 457),
-       'staging': ('query.cu', 250, 358), 'arena_probe': ('query.cu', 703, 790),
-       'skip_search': ('query.cu', 597, 702), 'probe_unit': ('query.cu', 791, 957),
-       'gallop_unit': ('query.cu', 1196, 1405), 'merge_unit_setup': ('query.cu', 1037, 1152),
-       'unit_head': ('query.cu', 959, 1036), 'lower_bound_s': ('griffin_dev.cuh', 477, 499),
+REG = {'merge_loop': ('query.cu', 1216, 1265), 'fine_split': ('griffin_dev.cuh', 515, 535),
+       'emit_lanes': ('query.cu', 432, 500), 'emit_unit': ('query.cu', 360, 431),
+       'tf/bm25': ('griffin_dev.cuh', 460, 480), 'decoders': ('griffin_dev.cuh', 143, 420),
+       'nextgeq': ('griffin_dev.cuh', 421, 459),
+       'staging': ('query.cu', 250, 359), 'arena_probe': ('query.cu', 739, 826),
+       'skip_search': ('query.cu', 641, 738), 'probe_unit': ('query.cu', 827, 999),
+       'gallop_unit': ('query.cu', 1266, 1468), 'merge_unit_setup': ('query.cu', 1079, 1215),
+       'unit_head': ('query.cu', 1000, 1078), 'lower_bound_s': ('griffin_dev.cuh', 481, 514),
        'carve': ('query.cu', 200, 249), 'scan82': ('griffin_dev.cuh', 76, 86)}
 rows = list(csv.reader(io.StringIO(out)))
 cur, hdr = None, None
