@@ -2,6 +2,7 @@
 // statistics, docID-range sharding, workspace management and the synchronous
 // host-buffer entry points.  Every step of the query path itself runs in the
 // kernels of encode.cu / query.cu; nothing here computes query results.
+#include <cstdlib>
 #include <algorithm>
 #include <cmath>
 #include <cstring>
@@ -181,6 +182,7 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   ix->T = opts.gallop_ratio ? opts.gallop_ratio : std::max<uint32_t>(4, B / 8);
   ix->Tdec = opts.gallop_ratio_decoded ? opts.gallop_ratio_decoded : std::max<uint32_t>(4, B / 8);
   ix->D = std::max<uint32_t>(2, 1024 / B);
+  if (const char *e = std::getenv("GRIFFIN_TUNE_D")) ix->D = std::max<uint32_t>(2, (uint32_t)std::atoi(e));  // A/B probes
   ix->k1 = k1;
   ix->bm25_b = bb;
   ix->N = N;

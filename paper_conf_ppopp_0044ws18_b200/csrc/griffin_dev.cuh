@@ -153,6 +153,103 @@ struct XorSink {
   __device__ __forceinline__ void put(uint32_t *, uint32_t v) { x ^= v; }
 };
 
+// ---- eight consecutive elements of a staged block (one lane) ----------------------
+// Elements k .. k+ne-1 (ne <= 8) given p = the high-stream position of element
+// k's one and `win` = the 32 high-stream bits after it.  The ones of elements
+// k+1..k+4 come from `win`; a fresh window read right after element k+4's one
+// gives k+5..k+7, so a run of zeros inside one 32-bit window (likely when the
+// high stream is sparse, u/2^b ~ 2n) does not force the slow path.  Low bits by
+// funnel shifts of the staged low stream (one window covers all eight when
+// b <= 4, two when b <= 8).  Falls back to a serial walk when a window lacks
+// ones (only near the end of a partial block).  Returns the position of the
+// last decoded element's one (valid when ne == 8 and the fast path ran).
+template <class Sink>
+__device__ __forceinline__ uint32_t decode8(const uint32_t *__restrict__ stg,
+                                            const uint32_t *__restrict__ hs, uint32_t first,
+                                            uint32_t b, uint32_t mask, uint32_t k, uint32_t ne,
+                                            uint32_t p, uint32_t win, uint32_t *dst, Sink &sink) {
+  uint32_t w1 = win;
+  const uint32_t t1 = __ffs(w1);
+  w1 &= w1 - 1u;
+  const uint32_t t2 = __ffs(w1);
+  w1 &= w1 - 1u;
+  const uint32_t t3 = __ffs(w1);
+  w1 &= w1 - 1u;
+  const uint32_t t4 = __ffs(w1);
+  const uint32_t p4 = p + t4;   // element k+4's one
+  const uint32_t wb = p4 + 1u;
+  const uint32_t win2 = __funnelshift_r(hs[wb >> 5], hs[(wb >> 5) + 1], wb);
+  uint32_t w2 = win2;
+  const uint32_t s1 = __ffs(w2);
+  w2 &= w2 - 1u;
+  const uint32_t s2 = __ffs(w2);
+  w2 &= w2 - 1u;
+  const uint32_t s3 = __ffs(w2);
+  const bool ok = (ne <= 1u || __popc(win) >= min(ne - 1u, 4u)) &&
+                  (ne <= 5u || __popc(win2) >= ne - 5u);
+  if (ok) {
+    uint32_t hv[8];
+    hv[0] = p - k;
+    hv[1] = p + t1 - (k + 1u);
+    hv[2] = p + t2 - (k + 2u);
+    hv[3] = p + t3 - (k + 3u);
+    hv[4] = p4 - (k + 4u);
+    hv[5] = p4 + s1 - (k + 5u);
+    hv[6] = p4 + s2 - (k + 6u);
+    hv[7] = p4 + s3 - (k + 7u);
+    uint32_t lv[8];
+    const uint32_t bp = k * b;
+    if (b <= 4u) {
+      const uint32_t lw32 = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp);
+#pragma unroll
+      for (uint32_t j = 0; j < 8; ++j) lv[j] = (lw32 >> (j * b)) & mask;
+    } else if (b <= 8u) {
+      const uint32_t q = bp + 4u * b;
+      const uint32_t x1 = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp);
+      const uint32_t x2 = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q);
+#pragma unroll
+      for (uint32_t j = 0; j < 4; ++j) {
+        lv[j] = (x1 >> (j * b)) & mask;
+        lv[j + 4] = (x2 >> (j * b)) & mask;
+      }
+    } else {
+#pragma unroll
+      for (uint32_t j = 0; j < 8; ++j) {
+        const uint32_t q = bp + j * b;
+        lv[j] = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
+      }
+    }
+    uint32_t v[8];
+#pragma unroll
+    for (uint32_t j = 0; j < 8; ++j) v[j] = first + ((hv[j] << b) | lv[j]);
+    if (ne == 8u) {
+      sink.put4(dst + k, make_uint4(v[0], v[1], v[2], v[3]));
+      sink.put4(dst + k + 4, make_uint4(v[4], v[5], v[6], v[7]));
+    } else {
+#pragma unroll
+      for (uint32_t j = 0; j < 8; ++j)
+        if (j < ne) sink.put(dst + k + j, v[j]);
+    }
+    return p4 + s3;
+  }
+  // serial walk with a refilled 32-bit window
+  uint32_t wbb = p + 1u, ww = win, pp = p, bp = k * b;
+  for (uint32_t j = 0; j < ne; ++j) {
+    if (j) {
+      while (ww == 0u) {
+        wbb += 32u;
+        ww = __funnelshift_r(hs[wbb >> 5], hs[(wbb >> 5) + 1], wbb);
+      }
+      pp = wbb + (__ffs(ww) - 1u);
+      ww &= ww - 1u;
+    }
+    const uint32_t lo_bits = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp) & mask;
+    sink.put(dst + k + j, first + (((pp - (k + j)) << b) | lo_bits));
+    bp += b;
+  }
+  return pp;
+}
+
 // ---- Elias-Fano block decode (Para-EF, §3.1.1 / Alg. 1) -------------
 // One warp decodes one block of n <= B postings, already staged in shared memory
 // (low stream: lw words, then high stream: hw words), into dst[0..n) as absolute
@@ -230,7 +327,20 @@ __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ 
     // the 32 bits following element k0's one (clamped funnel: pos+1 may be 32)
     uint32_t win = __funnelshift_rc(x, nx, pos + 1u);
     const uint32_t mask = b ? (0xFFFFFFFFu >> (32u - b)) : 0u;
-    if (E == 4 && ne == 4 && __popc(win) >= 3u) {
+    if (E == 8 || E == 16) {   // B = 256 / 512: runs of eight (decode8)
+      const uint32_t p7 = decode8(stg, hs, first, b, mask, k0, min(8u, ne), p0, win, dst, sink);
+      if (ne > 8u) {   // second run: element k0+8's one is the next one after p7
+        uint32_t wb = p7 + 1u;
+        uint32_t w8 = __funnelshift_r(hs[wb >> 5], hs[(wb >> 5) + 1], wb);
+        while (w8 == 0u) {
+          wb += 32u;
+          w8 = __funnelshift_r(hs[wb >> 5], hs[(wb >> 5) + 1], wb);
+        }
+        const uint32_t p8 = wb + (__ffs(w8) - 1u);
+        decode8(stg, hs, first, b, mask, k0 + 8u, ne - 8u, p8,
+                __funnelshift_r(hs[(p8 + 1u) >> 5], hs[((p8 + 1u) >> 5) + 1], p8 + 1u), dst, sink);
+      }
+    } else if (E == 4 && ne == 4 && __popc(win) >= 3u) {
       // fast path (B = 128): the next three ones are inside the window
       const uint32_t t1 = __ffs(win);
       win &= win - 1u;
@@ -331,64 +441,10 @@ __device__ __forceinline__ void warp_decode_pair_staged(
   if (w + 1u >= hw) nx = 0u;
   const uint32_t k0 = l << 3;
   if (k0 < n) {
-    const uint32_t ne = min(8u, n - k0);
     const uint32_t pos = select_in_word(x, k0 - ex, lut);
-    const uint32_t p0 = (w << 5) + pos;
-    uint32_t win = __funnelshift_rc(x, nx, pos + 1u);
     const uint32_t mask = b ? (0xFFFFFFFFu >> (32u - b)) : 0u;
-    if (ne == 8u && __popc(win) >= 7u) {
-      uint32_t hv[8];
-      hv[0] = p0 - k0;
-#pragma unroll
-      for (uint32_t j = 1; j < 8; ++j) {
-        const uint32_t t = __ffs(win);
-        win &= win - 1u;
-        hv[j] = p0 + t - (k0 + j);
-      }
-      uint32_t lv[8];
-      const uint32_t bp = k0 * b;
-      if (b <= 4u) {
-        const uint32_t lw32 = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp);
-#pragma unroll
-        for (uint32_t j = 0; j < 8; ++j) lv[j] = (lw32 >> (j * b)) & mask;
-      } else if (b <= 8u) {
-        const uint32_t q = bp + 4u * b;
-        const uint32_t w1 = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp);
-        const uint32_t w2 = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q);
-#pragma unroll
-        for (uint32_t j = 0; j < 4; ++j) {
-          lv[j] = (w1 >> (j * b)) & mask;
-          lv[j + 4] = (w2 >> (j * b)) & mask;
-        }
-      } else {
-#pragma unroll
-        for (uint32_t j = 0; j < 8; ++j) {
-          const uint32_t q = bp + j * b;
-          lv[j] = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q) & mask;
-        }
-      }
-      sink.put4(dst + k0, make_uint4(first + ((hv[0] << b) | lv[0]), first + ((hv[1] << b) | lv[1]),
-                                     first + ((hv[2] << b) | lv[2]), first + ((hv[3] << b) | lv[3])));
-      sink.put4(dst + k0 + 4, make_uint4(first + ((hv[4] << b) | lv[4]), first + ((hv[5] << b) | lv[5]),
-                                         first + ((hv[6] << b) | lv[6]), first + ((hv[7] << b) | lv[7])));
-    } else {
-      uint32_t wb = p0 + 1u;
-      uint32_t p = p0;
-      uint32_t bp = k0 * b;
-      for (uint32_t j = 0; j < ne; ++j) {
-        if (j) {
-          while (win == 0u) {
-            wb += 32u;
-            win = __funnelshift_r(hs[wb >> 5], hs[(wb >> 5) + 1], wb);
-          }
-          p = wb + (__ffs(win) - 1u);
-          win &= win - 1u;
-        }
-        const uint32_t lo_bits = __funnelshift_r(stg[bp >> 5], stg[(bp >> 5) + 1], bp) & mask;
-        sink.put(dst + k0 + j, first + (((p - (k0 + j)) << b) | lo_bits));
-        bp += b;
-      }
-    }
+    decode8(stg, hs, first, b, mask, k0, min(8u, n - k0), (w << 5) + pos,
+            __funnelshift_rc(x, nx, pos + 1u), dst, sink);
   }
   __syncwarp();
 }

@@ -215,9 +215,13 @@ __host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D) {
 // read slack after the tile: the uniform-trip merge loop may read up to L =
 // ceil((D+2)*B/32) words past a lane's segment (D <= 8 at B = 128 -> 40)
 constexpr uint32_t kTileSlack = 64;
+// read slack after the staging area: decoders read a word or two past a block's
+// high stream (look-ahead windows), also when it ends the staging area
+constexpr uint32_t kStgSlack = 4;
 // with_tile = false: no decode tile (kernels that decode straight to HBM)
 __host__ __device__ inline uint32_t warp_smem_words(uint32_t B, uint32_t D, bool with_tile = true) {
-  return 8 + 64 + (B + 32) + stage_words(B, D) + (with_tile ? (D + 2) * B + kTileSlack : 0u);
+  return 8 + 64 + (B + 32) + stage_words(B, D) + kStgSlack +
+         (with_tile ? (D + 2) * B + kTileSlack : 0u);
 }
 constexpr uint32_t kLutBytes = 2048;
 
@@ -239,7 +243,7 @@ __device__ __forceinline__ WarpSmem carve_warp_smem(uint4 *smem4, uint32_t B, ui
   w.cnt = wb + 8;
   w.aux = w.cnt + 64;
   w.stg = w.aux + B + 32;
-  w.tile = with_tile ? w.stg + stage_words(B, D) : nullptr;
+  w.tile = with_tile ? w.stg + stage_words(B, D) + kStgSlack : nullptr;
   w.phase = 0;
   return w;
 }
@@ -997,7 +1001,10 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
 
 
 template <bool RC>
-__global__ void __launch_bounds__(kIntersectThreads, 3) intersect_kernel(DevIndex ix, RoundArgs a) {
+#ifndef GRIFFIN_INTERSECT_MINB
+#define GRIFFIN_INTERSECT_MINB 3
+#endif
+__global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) intersect_kernel(DevIndex ix, RoundArgs a) {
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
   const uint32_t B = ix.B, D = a.D;

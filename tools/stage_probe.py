@@ -16,7 +16,7 @@ cfg_name = sys.argv[1] if len(sys.argv) > 1 else "c2"
 c, ql, cfg = make_workload(cfg_name)
 k = cfg["k"]
 nq = ql.num_queries
-ix = g.GriffinIndex(c, block_size=cfg["block"])
+ix = g.GriffinIndex(c, block_size=int(os.environ.get("PROBE_B", cfg["block"])))
 ix.griffin_reserve(ql.offsets, ql.terms, k)
 mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
 d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
