@@ -319,6 +319,91 @@ def test_c2_full_size_sampled():
         assert_topk_equal(gd[q], gs[q], gc[q], od, os_, oc)
 
 
+def _sub_corpus(c, terms):
+    """The corpus with every list outside `terms` emptied: N, doc lengths (so
+    avgdl and every norm) and the kept lists (so their df and idf) are unchanged,
+    hence the oracle scores the sampled queries exactly as on the full corpus."""
+    from synth import Corpus
+    keep = np.zeros(c.num_terms, bool)
+    keep[list(terms)] = True
+    df = np.where(keep, c.df(), 0)
+    off = np.zeros(c.num_terms + 1, np.uint64)
+    off[1:] = np.cumsum(df)
+    docs = np.concatenate([c.list(t) for t in sorted(terms)] or [np.zeros(0, np.uint32)])
+    tfs = np.concatenate([c.tf_list(t) for t in sorted(terms)] or [np.zeros(0, np.uint32)])
+    return Corpus(num_docs=c.num_docs, offsets=off, docids=docs.astype(np.uint32),
+                  tfs=tfs.astype(np.uint32), doc_lengths=c.doc_lengths)
+
+
+@pytest.mark.slow
+def test_c5_full_size_sampled():
+    """BASELINE configs[4] at full size (50M docs, ~1.86 B postings, 10K queries,
+    top-1000) in the launch configuration of the C5 batch (one batch of all
+    queries, device API, decode-once reuse on): invariants on every query and 12
+    sampled queries bit-exact against the oracle (built over the sampled
+    queries' complete lists with the full corpus' N and doc lengths)."""
+    import torch
+    c, ql, cfg = make_workload("c5")
+    k = cfg["k"]
+    nq = ql.num_queries
+    gx = g.GriffinIndex(c, block_size=128)
+    gx.griffin_reserve(ql.offsets, ql.terms, k)
+    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
+    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
+    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(nq, dtype=torch.int32, device="cuda")
+    gx.griffin_query_batch_device(d_off, d_t, mt, k, keys, cnt, torch.cuda.current_stream())
+    dd = torch.zeros(nq * k, dtype=torch.int32, device="cuda")
+    ds = torch.zeros(nq * k, dtype=torch.float32, device="cuda")
+    gx.griffin_keys_to_results_device(nq, k, keys, cnt, dd, ds)
+    torch.cuda.synchronize()
+    gx.griffin_sync_status()
+    del gx
+    gd = dd.cpu().numpy().view(np.uint32).reshape(nq, k)
+    gs = ds.cpu().numpy().reshape(nq, k)
+    gc = cnt.cpu().numpy().view(np.uint32)
+    assert gc.max() > 100, "the planted co-occurrences should give large results"
+    for q in range(nq):
+        n = gc[q]
+        s_, d_ = gs[q, :n], gd[q, :n]
+        assert np.all((s_[1:] < s_[:-1]) | ((s_[1:] == s_[:-1]) & (d_[1:] > d_[:-1])))
+        assert np.all(gd[q, n:] == 0xFFFFFFFF) and np.all(np.isneginf(gs[q, n:]))
+        for t in set(ql.query(q).tolist()):
+            lst = c.list(t)
+            pos = np.searchsorted(lst, d_)
+            assert np.all(lst[np.minimum(pos, len(lst) - 1)] == d_)
+    sample = np.random.default_rng(5).choice(nq, size=12, replace=False)
+    terms = set()
+    for q in sample:
+        terms |= set(ql.query(q).tolist())
+    ox = oracle.OracleIndex(_sub_corpus(c, terms), block_size=128)
+    for q in sample:
+        od, os_, oc = ox.query(ql.query(q), k)
+        assert_topk_equal(gd[q], gs[q], gc[q], od, os_, oc)
+
+
+@pytest.mark.slow
+def test_c3_full_size_ratio_pairs():
+    """BASELINE configs[2] shape at full size: 25M docs, |S| = 10M (G6 extended),
+    |R| = |S|/lambda for lambda from 1 to 1000: merge, gallop and
+    auto give the oracle's docID set, and the scored top-10 / top-1000 are
+    bit-exact (one batch of all pairs)."""
+    ratios = [1, 4, 16, 64, 128, 512, 1000]
+    c, ql = make_pair_workload(25_000_000, 10_000_000, ratios, seed=0x4752494646494E03)
+    ox = oracle.OracleIndex(c, block_size=128)
+    gx = g.GriffinIndex(c, block_size=128)
+    for q in range(ql.num_queries):
+        want = ox.intersect(ql.query(q))
+        assert len(want) > 0
+        for mode in (g.MODE_AUTO, g.MODE_MERGE, g.MODE_GALLOP):
+            assert np.array_equal(gx.griffin_debug_intersect(ql.query(q), mode), want)
+    for k in (10, 1000):
+        d, s, cn = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+        od, os_, oc = ox.query_batch(ql, k)
+        assert_topk_equal(d, s, cn, od, os_, oc)
+
+
 # ---------------------------------------------------------------- batch list reuse
 
 @pytest.mark.parametrize("reuse", [0, 1])
