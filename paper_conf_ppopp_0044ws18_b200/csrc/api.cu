@@ -183,6 +183,12 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   ix->Tdec = opts.gallop_ratio_decoded ? opts.gallop_ratio_decoded : std::max<uint32_t>(4, B / 8);
   ix->D = std::max<uint32_t>(2, 1024 / B);
   if (const char *e = std::getenv("GRIFFIN_TUNE_D")) ix->D = std::max<uint32_t>(2, (uint32_t)std::atoi(e));  // A/B probes
+  if (const char *e = std::getenv("GRIFFIN_TOPK_FILTER")) ix->topk_filter = std::atoi(e);  // A/B
+  if (const char *e = std::getenv("GRIFFIN_SORDER")) {   // A/B probes: 0 = off, else 1 + shift
+    const int v = std::atoi(e);
+    ix->sorder = v > 0;
+    if (v > 0) ix->sorder_shift = (uint32_t)(v - 1);
+  }
   ix->k1 = k1;
   ix->bm25_b = bb;
   ix->N = N;

@@ -56,10 +56,12 @@ struct Workspace {
   DevBuf plan_terms, plan_m, cap, cap_off, rcount, rsel, qmode, unit_base;  // per query
   DevBuf unit_off, unit_cnt, unit_dst, urec, uperm;                         // per unit
   DevBuf rbuf0, rbuf1, bump, cand, tkstate;                                 // per survivor
+  DevBuf flt, fstate;   // top-k sampled-threshold pre-filter: kept keys, per-query state
   DevBuf scal;       // scalars: counters, status, bump ctr, unit ctr
   DevBuf keys, counts, docids, scores, qoffs, qterms;  // host-API staging on device
   DevBuf demand, tdec, runs, run_base, vtmp, run_term; // per term / run (batch reuse)
   DevBuf arena;                                        // decoded lists, nblocks * B u32
+  DevBuf sbkt_cnt, sbkt_pos, sbkt_tmp;                 // S-locality unit order buckets
   size_t nq_cap = 0, unit_cap = 0, entry_cap = 0;
   // pinned host staging
   void *h_pinned = nullptr;
@@ -105,6 +107,9 @@ struct RoundArgs {
   unsigned long long *scal;
   uint4 *urec;            // per unit: {q, i0|lu, j0, lo docID} (partition stage)
   uint32_t *uperm;        // processing order of the units: merge units first, then the rest
+  uint32_t *sbkt_cnt;     // S-locality order: merge units per bucket of S blocks (or null)
+  unsigned long long *sbkt_pos;   // bucket cursors (exclusive scan of sbkt_cnt)
+  uint32_t sbkt_shift;    // bucket = global S block of the unit's start >> shift
   const uint32_t *dec;    // batch decoded arena (global block * B + i), or null
   const uint8_t *tdec;    // per term: 1 = decoded in the arena this batch
 };
@@ -146,6 +151,9 @@ struct griffin_index {
   int use_graphs = 1;
   int probe = 1;
   int nextgeq = 1;
+  int topk_filter = 1;   // sampled-threshold pre-filter for large candidate sets
+  int sorder = 1;   // merge units ordered by the S blocks they read (L2 reuse across queries)
+  uint32_t sorder_shift = 6;
   uint32_t P = 0;   // probe chunk (0 = B)
   bool profiling = false;
   griffin_profile prof{};

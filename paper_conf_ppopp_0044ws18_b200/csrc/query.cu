@@ -548,6 +548,14 @@ __device__ __forceinline__ void warp_mp_search2(HR hR, uint32_t nbR, HS hS, uint
 template <bool RC>
 __device__ __forceinline__ void unit_record(const DevIndex &ix, const RoundArgs &a, uint64_t u);
 
+// bucket of merge unit u for the S-locality order: global S block of its start
+__device__ __forceinline__ uint32_t merge_unit_bucket(const DevIndex &ix, const RoundArgs &a,
+                                                      uint64_t u) {
+  const uint4 rec = a.urec[u];
+  const uint32_t sid = a.plan_terms[(size_t)rec.x * kMaxTerms + a.round];
+  return (ix.terms[sid].block0 + rec.z) >> a.sbkt_shift;
+}
+
 template <bool RC>
 __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
   const uint64_t total = a.unit_base[a.nq];
@@ -578,8 +586,33 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
     }
     hm = __shfl_sync(0xffffffffu, hm, 0);
     ho = __shfl_sync(0xffffffffu, ho, 0);
-    if (mg) a.uperm[hm + __popc(bm & lt)] = (uint32_t)u;
-    else if (valid) a.uperm[total - 1 - (ho + __popc(bo & lt))] = (uint32_t)u;
+    if (mg) {
+      if (a.sbkt_cnt) atomicAdd(a.sbkt_cnt + merge_unit_bucket(ix, a, u), 1u);
+      else a.uperm[hm + __popc(bm & lt)] = (uint32_t)u;
+    } else if (valid) {
+      a.uperm[total - 1 - (ho + __popc(bo & lt))] = (uint32_t)u;
+    }
+  }
+}
+
+// S-locality order (after partition_kernel and a scan of the bucket counts):
+// used for batches of >= kSorderMinQueries queries (C5, 10K queries: intersect
+// 15.41 -> 14.76 ms; at C2's 1000 queries the extra scan + scatter cost more
+// than the reuse gains: 0.703 -> 0.722 ms, profiles/r01_configs.jsonl).
+// merge units are placed by the global S block their range starts at, so the
+// units of different queries that merge against the same S range are handed
+// out together and their S tiles come from L2 (a C2 batch merges 92M S
+// postings of 39M distinct ones, C5 2.66 B of 455M).  Order inside a bucket is
+// arbitrary; results do not depend on processing order.
+constexpr uint32_t kSorderMinQueries = 4096;
+__global__ void sorder_scatter_kernel(DevIndex ix, RoundArgs a) {
+  const uint64_t total = a.unit_base[a.nq];
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < total; u += stride) {
+    const uint32_t q = a.urec[u].x;
+    if (a.qmode[q] != kModeMerge) continue;
+    const unsigned long long slot = atomicAdd(a.sbkt_pos + merge_unit_bucket(ix, a, u), 1ull);
+    a.uperm[slot] = (uint32_t)u;
   }
 }
 
@@ -1189,6 +1222,12 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         }
       }
       __syncwarp();
+      // sentinel after the S tile's valid elements: the uniform-trip merge loop
+      // below may step B past them (a lane whose A elements outlast B), and
+      // stale shared memory there (e.g. another unit's R tile) could equal an
+      // in-segment A element and count as a false match
+      if (lane == 0) tileS[nSt] = kNone;
+      __syncwarp();
       // ranges inside [lo, hi): four lower_bounds — (R, lo), (R, hi), (S, lo),
       // (S, hi) — each by an 8-lane group doing an 8-ary search (7 probes per
       // step, ballot + popc), ~log8 dependent smem loads instead of log2
@@ -1659,7 +1698,24 @@ struct TopkState {
   uint8_t *qlev;
   uint64_t *qoff;
   uint32_t *qn;
+  // sampled-threshold pre-filter (queries with > kFiltMin candidates)
+  uint64_t *flt;     // slot s holds keys at flt[s * kFiltCap ..]
+  uint64_t *ftau;    // per query: threshold key
+  uint32_t *fslot;   // per query: slot or kNone
+  uint32_t *fcnt;    // per slot: keys >= threshold seen
+  uint32_t *fctr;    // slots handed out
+  uint32_t fmax;     // slots available (0 = pre-filter off)
 };
+constexpr uint8_t kLevFilt = 7;            // qlev: candidates are the query's filter slot
+constexpr uint32_t kFiltMin = 65536;       // pre-filter queries with more candidates than this
+constexpr uint32_t kFiltCap = 65536;       // keys kept per filtered query (else fall back)
+constexpr uint32_t kFiltSample = kTopkSmem;
+constexpr size_t kFiltSlots = 256;         // filtered queries per batch (the rest: no filter)
+
+__device__ __forceinline__ const uint64_t *cand_keys(const CandBufs &cb, const TopkState &ts,
+                                                     uint32_t lev, uint32_t q) {
+  return lev == kLevFilt ? ts.flt + ts.qoff[q] : cb.lv[lev] + ts.qoff[q];
+}
 
 __global__ void topk_init_kernel(uint32_t nq, const uint32_t *rcount, TopkState ts) {
   const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1667,6 +1723,101 @@ __global__ void topk_init_kernel(uint32_t nq, const uint32_t *rcount, TopkState 
     ts.qlev[q] = 0;
     ts.qoff[q] = 0;
     ts.qn[q] = rcount[q];
+    if (ts.fmax) ts.fslot[q] = kNone;
+  }
+  if (q == 0 && ts.fmax) *ts.fctr = 0;
+}
+
+// Pre-filter, step 1 (one CTA per query with n > kFiltMin candidates): a
+// systematic sample of kFiltSample keys; its r-th largest key becomes the
+// query's threshold tau, with r = mu + 4 sqrt(mu) + 2 for mu = k*s/n the
+// expected number of sampled keys among the true top k, so that with high
+// probability >= k keys are >= tau while only ~r*n/s survive the filter.
+// Exactness never depends on the sample: a query whose filtered count is < k
+// (or overflows kFiltCap) keeps its unfiltered candidates (topk_filter_update).
+__global__ void __launch_bounds__(kTopkThreads) topk_sample_kernel(
+    DevIndex ix, uint32_t nq, uint32_t k, const uint8_t *rsel, const uint64_t *cap_off,
+    const uint2 *rb0, const uint2 *rb1, TopkState ts) {
+  __shared__ uint64_t sk[kFiltSample];
+  __shared__ SelectSmem ss;
+  __shared__ uint32_t slot;
+  for (uint32_t q = blockIdx.x; q < nq; q += gridDim.x) {
+    const uint32_t n = ts.qn[q];
+    if (n <= kFiltMin) continue;   // block-uniform
+    const float mu = (float)k * (float)kFiltSample / (float)n;
+    const uint32_t r = (uint32_t)ceilf(mu + 4.f * sqrtf(mu) + 2.f);
+    if (r > kFiltSample / 8) continue;
+    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q];
+    for (uint32_t j = threadIdx.x; j < kFiltSample; j += blockDim.x)
+      sk[j] = make_key(R[(uint32_t)(((uint64_t)j * n) / kFiltSample)], ix.doc_base);
+    __syncthreads();
+    const uint64_t tau = cta_radix_select([&](uint32_t i) { return sk[i]; }, kFiltSample, r, ss);
+    if (threadIdx.x == 0) {
+      slot = atomicAdd(ts.fctr, 1u);
+      if (slot < ts.fmax) {
+        ts.ftau[q] = tau;
+        ts.fcnt[slot] = 0;
+        ts.fslot[q] = slot;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void topk_filter_plan_kernel(uint32_t nq, TopkState ts, uint32_t *nch) {
+  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q < nq) nch[q] = ts.fslot[q] != kNone ? (ts.qn[q] + kTopkSmem - 1) / kTopkSmem : 0u;
+}
+
+// Pre-filter, step 2: stream every candidate of the filtered queries (CTA per
+// chunk of kTopkSmem) and append the keys >= tau to the query's slot
+// (warp-aggregated atomics; order inside the slot is irrelevant).
+__global__ void __launch_bounds__(256) topk_filter_kernel(
+    DevIndex ix, uint32_t nq, const uint8_t *rsel, const uint64_t *cap_off, const uint2 *rb0,
+    const uint2 *rb1, TopkState ts, const uint64_t *cbase) {
+  const uint64_t total = cbase[nq];
+  const uint32_t lane = lane_id();
+  for (uint64_t c = blockIdx.x; c < total; c += gridDim.x) {
+    uint32_t lo = 0, hi = nq;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (cbase[mid] <= c) lo = mid; else hi = mid;
+    }
+    const uint32_t q = lo;
+    const uint32_t ci = (uint32_t)(c - cbase[q]);
+    const uint32_t len = min(kTopkSmem, ts.qn[q] - ci * kTopkSmem);
+    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q] + (size_t)ci * kTopkSmem;
+    const uint64_t tau = ts.ftau[q];
+    const uint32_t slot = ts.fslot[q];
+    uint64_t *out = ts.flt + (size_t)slot * kFiltCap;
+    for (uint32_t i0 = threadIdx.x - lane; i0 < len; i0 += blockDim.x) {
+      const uint32_t i = i0 + lane;
+      const uint64_t x = i < len ? make_key(R[i], ix.doc_base) : 0ull;
+      const bool keep = i < len && x >= tau;
+      const uint32_t bal = __ballot_sync(0xffffffffu, keep);
+      if (bal) {
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(ts.fcnt + slot, (uint32_t)__popc(bal));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        const uint32_t pos = base + __popc(bal & lanemask_lt());
+        if (keep && pos < kFiltCap) out[pos] = x;
+      }
+    }
+  }
+}
+
+// Pre-filter, step 3: a query whose slot holds >= min(k, n) keys (and did not
+// overflow) continues from its slot; otherwise from all its candidates.
+__global__ void topk_filter_update_kernel(uint32_t nq, uint32_t k, TopkState ts) {
+  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q >= nq) return;
+  const uint32_t slot = ts.fslot[q];
+  if (slot == kNone) return;
+  const uint32_t f = ts.fcnt[slot];
+  if (f >= min(k, ts.qn[q]) && f <= kFiltCap) {
+    ts.qlev[q] = kLevFilt;
+    ts.qoff[q] = (uint64_t)slot * kFiltCap;
+    ts.qn[q] = f;
   }
 }
 
@@ -1713,7 +1864,7 @@ __global__ void __launch_bounds__(kTopkThreads) topk_chunk_kernel(
       const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q] + (size_t)ci * kTopkSmem;
       for (uint32_t i = threadIdx.x; i < len; i += blockDim.x) sk[i] = make_key(R[i], ix.doc_base);
     } else {
-      const uint64_t *K = cb.lv[lev] + ts.qoff[q] + (size_t)ci * kTopkSmem;
+      const uint64_t *K = cand_keys(cb, ts, lev, q) + (size_t)ci * kTopkSmem;
       for (uint32_t i = threadIdx.x; i < len; i += blockDim.x) sk[i] = K[i];
     }
     __syncthreads();
@@ -1751,7 +1902,7 @@ __global__ void __launch_bounds__(kTopkThreads) topk_final_kernel(
     const uint32_t kk = min(k, c);
     const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q];
     const uint32_t lev = ts.qlev[q];
-    const uint64_t *C = lev ? cb.lv[lev] + ts.qoff[q] : nullptr;
+    const uint64_t *C = lev ? cand_keys(cb, ts, lev, q) : nullptr;
     const uint32_t n = ts.qn[q];
     auto key = [&](uint32_t i) -> uint64_t { return lev ? C[i] : make_key(R[i], ix.doc_base); };
     uint32_t nsel;
@@ -2027,6 +2178,12 @@ griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t
   GRIFFIN_CUDA_TRY(w.urec.reserve((units + 2) * 16));
   GRIFFIN_CUDA_TRY(w.uperm.reserve((units + 2) * 4));
   GRIFFIN_CUDA_TRY(w.unit_dst.reserve((units + 2) * 8 + (units / kScanTile + 2) * 8));
+  if (ix->sorder && nq >= kSorderMinQueries) {   // S-locality buckets (no allocation in run_batch)
+    const size_t nbkt = (ix->nblocks >> ix->sorder_shift) + 1;
+    GRIFFIN_CUDA_TRY(w.sbkt_cnt.reserve(nbkt * 4));
+    GRIFFIN_CUDA_TRY(w.sbkt_pos.reserve((nbkt + 1) * 8));
+    GRIFFIN_CUDA_TRY(w.sbkt_tmp.reserve((nbkt / kScanTile + 4) * 8));
+  }
   GRIFFIN_CUDA_TRY(w.rbuf0.reserve((entries + 1) * 8));
   GRIFFIN_CUDA_TRY(w.rbuf1.reserve((entries + 1) * 8));
   // per-warp bump chunks: at most one partly used chunk per resident warp
@@ -2096,6 +2253,11 @@ griffin_status reserve_topk(griffin_index *ix, Workspace &w, uint32_t nq, uint32
   const int levels = k <= 64 ? 1 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
   GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8 * std::max(levels, 1)));
   GRIFFIN_CUDA_TRY(w.tkstate.reserve(((size_t)nq + 1) * (1 + 8 + 4) + 64));
+  if (ix->topk_filter && k > 64 && w.entry_cap > kFiltMin && nq >= 2) {   // a query may exceed kFiltMin
+    const size_t slots = std::min<size_t>(nq, kFiltSlots);
+    GRIFFIN_CUDA_TRY(w.flt.reserve(slots * kFiltCap * 8));
+    GRIFFIN_CUDA_TRY(w.fstate.reserve(((size_t)nq + 1) * 12 + slots * 4 + 64));
+  }
   return GRIFFIN_OK;
 }
 
@@ -2214,13 +2376,27 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     {
       StageTimer t(ix, st, 1);
       const unsigned pgrid = num_sms(ix->device) * 8;
-      if (r == 1) {
-        partition_kernel<true><<<pgrid, 256, 0, st>>>(di, ra);
-        GRIFFIN_CUDA_TRY(launch_intersect<true>(ix, ra, st));
-      } else {
-        partition_kernel<false><<<pgrid, 256, 0, st>>>(di, ra);
-        GRIFFIN_CUDA_TRY(launch_intersect<false>(ix, ra, st));
+      ra.sbkt_cnt = nullptr;
+      ra.sbkt_pos = nullptr;
+      uint64_t nbkt = 0;
+      if (ix->sorder && nq >= kSorderMinQueries && (r == 1 || !ra.probe) && w.sbkt_cnt.p) {
+        ra.sbkt_shift = ix->sorder_shift;
+        nbkt = (ix->nblocks >> ra.sbkt_shift) + 1;   // buffers sized in reserve_ws
+        GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.sbkt_cnt.p, 0, nbkt * 4, st));
+        ra.sbkt_cnt = w.sbkt_cnt.as<uint32_t>();
+        ra.sbkt_pos = w.sbkt_pos.as<unsigned long long>();
       }
+      if (r == 1) partition_kernel<true><<<pgrid, 256, 0, st>>>(di, ra);
+      else partition_kernel<false><<<pgrid, 256, 0, st>>>(di, ra);
+      if (ra.sbkt_cnt) {
+        GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(ra.sbkt_cnt, w.sbkt_pos.as<uint64_t>(), nbkt,
+                                                  w.sbkt_tmp.as<uint64_t>(), st,
+                                                  &ix->launch_count));
+        sorder_scatter_kernel<<<pgrid, 256, 0, st>>>(di, ra);
+        ix->launch_count += 1;
+      }
+      if (r == 1) GRIFFIN_CUDA_TRY(launch_intersect<true>(ix, ra, st));
+      else GRIFFIN_CUDA_TRY(launch_intersect<false>(ix, ra, st));
       ix->launch_count += 1;
     }
     {
@@ -2253,10 +2429,34 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     ts.qoff = w.tkstate.as<uint64_t>();
     ts.qn = reinterpret_cast<uint32_t *>(ts.qoff + nq + 1);
     ts.qlev = reinterpret_cast<uint8_t *>(ts.qn + nq + 1);
+    ts.fmax = 0;
+    // for k > 64 (one chunk level keeps k of kTopkSmem keys, so large k needs
+    // up to 4 levels over shrinking-by-4x sets; C5 top-1000: 3.12 -> 1.29 ms);
+    // for k <= 64 one level already shrinks 64x and the extra launches cost more
+    if (ix->topk_filter && k > 64 && w.flt.p && w.fstate.p && nq >= 2) {
+      ts.fmax = (uint32_t)std::min<size_t>(w.flt.bytes / (kFiltCap * 8), kFiltSlots);
+      ts.flt = w.flt.as<uint64_t>();
+      ts.ftau = w.fstate.as<uint64_t>();
+      ts.fslot = reinterpret_cast<uint32_t *>(ts.ftau + nq + 1);
+      ts.fctr = ts.fslot + nq + 1;
+      ts.fcnt = ts.fctr + 1;
+      if ((size_t)(nq + 1) * 12 + 8 + (size_t)ts.fmax * 4 > w.fstate.bytes) ts.fmax = 0;
+    }
     const uint32_t *rc = w.rcount.as<uint32_t>();
     const uint8_t *rs = w.rsel.as<uint8_t>();
     topk_init_kernel<<<qblocks, 256, 0, st>>>(nq, rc, ts);
     ix->launch_count += 1;
+    if (ts.fmax) {
+      topk_sample_kernel<<<std::min<uint32_t>(nq, 148 * 4), kTopkThreads, 0, st>>>(
+          di, nq, k, rs, w.cap_off.as<uint64_t>(), w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), ts);
+      topk_filter_plan_kernel<<<qblocks, 256, 0, st>>>(nq, ts, nch);
+      GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(nch, cbase, nq, scan_tmp, st, &ix->launch_count));
+      topk_filter_kernel<<<num_sms(ix->device) * 8, 256, 0, st>>>(
+          di, nq, rs, w.cap_off.as<uint64_t>(), w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), ts, cbase);
+      topk_filter_update_kernel<<<qblocks, 256, 0, st>>>(nq, k, ts);
+      GRIFFIN_CUDA_TRY(cudaGetLastError());
+      ix->launch_count += 4;
+    }
     for (int L = 1; L <= levels; ++L) {
       topk_plan_kernel<<<qblocks, 256, 0, st>>>(nq, ts, nch);
       GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(nch, cbase, nq, scan_tmp, st, &ix->launch_count));

@@ -319,6 +319,17 @@ def test_c2_full_size_sampled():
         assert_topk_equal(gd[q], gs[q], gc[q], od, os_, oc)
 
 
+def test_large_batch_s_locality_order():
+    """Batches of >= 4096 queries hand out merge units in S-locality order
+    (sorder_scatter_kernel); the results must not depend on it."""
+    c, ql, cfg = make_workload("small", num_queries=5000)
+    gx = g.GriffinIndex(c, block_size=128)
+    ox = oracle.OracleIndex(c, block_size=128)
+    d, s, cn = gx.griffin_query_batch(ql.offsets, ql.terms, 10)
+    od, os_, oc = ox.query_batch(ql, 10, nthreads=4)
+    assert_topk_equal(d, s, cn, od, os_, oc)
+
+
 def _sub_corpus(c, terms):
     """The corpus with every list outside `terms` emptied: N, doc lengths (so
     avgdl and every norm) and the kept lists (so their df and idf) are unchanged,
@@ -456,6 +467,34 @@ def test_multilevel_topk_large_results(k):
     assert_topk_equal(gd, gs, gc, od, os_, oc)
 
 
+@pytest.mark.parametrize("k", [100, 1000])
+def test_topk_prefilter_on_off_identical(k, monkeypatch):
+    """Queries with > 65536 candidates go through the sampled-threshold
+    pre-filter (topk_sample/filter kernels, k > 64); with it disabled
+    (GRIFFIN_TOPK_FILTER=0 at build) the results are the same and equal the
+    oracle's.  Scores concentrated in a narrow docID band (long docs elsewhere)
+    make the systematic sample unrepresentative on purpose."""
+    rng = np.random.default_rng(900 + k)
+    N = 600_000
+    lists = [np.sort(rng.choice(N, size=n, replace=False)) for n in (500_000, 450_000, 200_000)]
+    tfs = [rng.integers(1, 40, size=len(l)) for l in lists]
+    dl = rng.integers(2000, 5000, size=N)
+    dl[300_000:300_050] = 1      # a band of very short docs: the top scores
+    c = corpus_from_lists(N, lists, tfs, dl)
+    qs = [[0, 1], [0], [1, 2], [0, 1, 2], [2]]
+    ql = QueryLog(offsets=np.cumsum([0] + [len(q) for q in qs]).astype(np.uint32),
+                  terms=np.concatenate(qs).astype(np.uint32))
+    od, os_, oc = oracle.OracleIndex(c).query_batch(ql, k)
+    res = []
+    for flag in ("1", "0"):
+        monkeypatch.setenv("GRIFFIN_TOPK_FILTER", flag)
+        gx = g.GriffinIndex(c)
+        res.append(gx.griffin_query_batch(ql.offsets, ql.terms, k))
+        del gx
+    for gd, gs, gc in res:
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
 def test_single_query_graph_path_reuse_and_recapture(tiny):
     """griffin_query replays cached CUDA graphs keyed by (distinct terms, k): many
     different queries, repeated, interleaved with a batch call that grows the
@@ -521,6 +560,25 @@ def _nextgeq_corpus(rng, N=3_000_000):
                                         for n in (300, 3_000, 30_000, 300_000, 1_500_000)]
     tfs = [rng.integers(1, 9, size=len(x)) for x in lists]
     return corpus_from_lists(N, lists, tfs, rng.integers(1, 3000, size=N))
+
+
+def test_merge_tile_tail_no_false_matches():
+    """Regression: the uniform-trip merge loop can step the S side past the
+    tile's valid elements; stale shared memory there once matched an R element
+    of an earlier unit (~1 in 400 calls at B = 512, D = 2; fixed by a sentinel).
+    Repeats the triggering merges (a consecutive-run S list, a short random R)
+    many times so stale tiles from earlier calls are around."""
+    rng = np.random.default_rng(900 + 512)
+    c = _nextgeq_corpus(rng)
+    ox = oracle.OracleIndex(c)
+    gx = g.GriffinIndex(c, block_size=512)
+    gx.griffin_set_reuse(0)
+    qs = ([0, 4], [4, 0], [0, 3], [0, 5], [0, 6], [0, 7])
+    want = [ox.intersect(q) for q in qs]
+    for _ in range(150):
+        for q, w in zip(qs, want):
+            for mode in (g.MODE_AUTO, g.MODE_MERGE):
+                assert np.array_equal(gx.griffin_debug_intersect(q, mode), w), (q, mode)
 
 
 @pytest.mark.parametrize("B", [64, 128, 256, 512])
