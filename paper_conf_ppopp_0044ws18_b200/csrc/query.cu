@@ -436,7 +436,8 @@ template <bool RC>
 __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, const TermInfo &tR,
                            const TermInfo &tS, const uint2 *Rq, const uint32_t *tile,
                            const uint32_t *ml0, uint32_t cap, uint32_t c, uint32_t *scr,
-                           uint32_t posR0, uint32_t posS0, Acc &acc) {
+                           uint32_t posR0, uint32_t posS0, uint32_t abase, uint32_t bbase,
+                           Acc &acc) {
   const uint32_t lane = lane_id();
   const uint32_t incl = warp_incl_scan(c);
   uint32_t cnt = __shfl_sync(0xffffffffu, incl, 31);
@@ -464,10 +465,11 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
             if (scr[o + step - 1] <= j) o += step;
           const uint32_t ex = o ? scr[o - 1] : 0u;
           const uint32_t e = ml0[o * cap + (j - ex)];
-          const uint32_t i = e & 0xFFFFu;
+          const uint32_t i = ((e - abase) & 0xFFFFu) >> 2;            // R tile index
+          const uint32_t js = (((e >> 16) - bbase) & 0xFFFFu) >> 2;   // S index from Bv
           doc[t] = tile[i];
           nrm[t] = __ldg(ix.norm + doc[t]);
-          tS_[t] = tf_lookup(ix, tS, posS0 + (e >> 16));
+          tS_[t] = tf_lookup(ix, tS, posS0 + js);
           if (RC) tR_[t] = tf_lookup(ix, tR, posR0 + i);
           else prev[t] = Rq[posR0 + i].y;
         }
@@ -1281,7 +1283,9 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         // in-segment element can equal an out-of-segment one (merge-path order +
         // the A9 fix-up).  Every step writes the candidate pair and keeps it only
         // on a match, so the loop has no divergent branch at all.
-        uint32_t key = (ra + is) | (js << 16);   // R tile index | S tile index << 16
+        // match key = low 16 bits of both smem addresses (one PRMT per step
+        // instead of maintaining a packed index pair; the tiles span < 64 KB,
+        // emit_lanes turns the halves back into tile indices)
         uint32_t pa = smem_u32(A + is), pb = smem_u32(Bv + js);
         const uint32_t paE = smem_u32(A + ie);
         const uint32_t pm0 = smem_u32(ml);
@@ -1291,22 +1295,22 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
           uint32_t x, y;
           asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(pa));
           asm volatile("ld.shared.u32 %0, [%1];" : "=r"(y) : "r"(pb));
-          asm volatile("st.shared.u32 [%0], %1;" ::"r"(pm), "r"(key));
+          asm volatile("st.shared.u32 [%0], %1;" ::"r"(pm), "r"(__byte_perm(pa, pb, 0x5410)));
           pm += (x == y && pa < paE) ? 4u : 0u;
-          const uint32_t da = (x <= y) ? 1u : 0u, db = (y <= x) ? 1u : 0u;
-          pa += da << 2;
-          pb += db << 2;
-          key += da + (db << 16);
+          pa += (x <= y) ? 4u : 0u;
+          pb += (y <= x) ? 4u : 0u;
         }
         c = (pm - pm0) >> 2;
       }
       __syncwarp();
       if (RC)
         emit_lanes<true>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, sm.stg, cap, c, sm.cnt, rb0 * B,
-                         sb0 * B + sa, acc);
+                         sb0 * B + sa, smem_u32(sm.tile) & 0xFFFFu,
+                         smem_u32(tileS + sa) & 0xFFFFu, acc);
       else
         emit_lanes<false>(ix, a, (uint32_t)u, tR, tS, Rq, sm.tile, sm.stg, cap, c, sm.cnt, rb0 * B,
-                          sb0 * B + sa, acc);
+                          sb0 * B + sa, smem_u32(sm.tile) & 0xFFFFu,
+                          smem_u32(tileS + sa) & 0xFFFFu, acc);
       __syncwarp();
     } else {
       // ---- gallop: R chunk lu, skip-pointer search into S (Fig. 9) ----

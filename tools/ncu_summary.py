@@ -55,17 +55,26 @@ for r in rows[2:]:
             except ValueError:
                 pass
     tot = sum(x for x, _ in stalls) or 1.0
+    # warp-execution efficiency = active threads per executed warp instruction / 32;
+    # divergence = branch targets reached by a divergent subset of a warp's threads
+    r = val(d, "smsp__thread_inst_executed_per_inst_executed.ratio")
+    wee = f"{100 * r / 32:.1f}%" if r is not None else "n/a"
+    dv = val(d, "smsp__sass_branch_targets_threads_divergent.sum")
+    br = val(d, "smsp__inst_executed_op_branch.sum")
+    div = (f"{dv:.3g} ({100 * dv / br:.1f}% of {br:.3g} branch instr)" if dv is not None and br
+           else "n/a")
     top = ", ".join(f"{h} {100 * x / tot:.0f}%" for x, h in sorted(stalls, reverse=True)[:4])
     lines.append(f"{name}: {t * 1e3:.3f} ms, DRAM read {rd / 1e6:.1f} MB write {wr / 1e6:.1f} MB "
                  f"({(rd + wr) / t / 1e9:.0f} GB/s), inst {val(d, 'smsp__inst_executed.sum'):.3g}, "
                  f"issue {d.get('smsp__issue_active.avg.pct_of_peak_sustained_active')}%, "
                  f"warps active {d.get('sm__warps_active.avg.pct_of_peak_sustained_active')}%, "
+                 f"warp-exec efficiency {wee}, divergent branch targets {div}, "
                  f"stalls: {top}")
 lines.append("")
 for idx in range(len(rows) - 2):
     name = rows[2 + idx][hdr.index("Kernel Name")]
     if "intersect" in name or "decode" in name:
-        src = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_lines.py"), rep,
+        src = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_lines2.py"), rep,
                               str(idx), "12"], capture_output=True, text=True).stdout
         lines.append(f"## top source lines, launch {idx}: {name.split('(')[0]}")
         lines += src.strip().splitlines()
