@@ -774,7 +774,10 @@ __device__ __forceinline__ void skip_blocks_sampled(const uint32_t *__restrict__
 // log2(B) for a binary search.  kEpl independent probes per lane run in
 // lockstep so their loads overlap.  Writes match[e] = kb*B + pos on a hit and
 // returns the number of chunks loaded.
-constexpr int kArenaEpl = 4;
+#ifndef GRIFFIN_ARENA_EPL
+#define GRIFFIN_ARENA_EPL 2
+#endif
+constexpr int kArenaEpl = GRIFFIN_ARENA_EPL;
 __device__ __forceinline__ uint32_t arena_probe_slice(const uint32_t *__restrict__ decS,
                                                       const uint32_t *__restrict__ fS,
                                                       uint32_t nblocksS, uint32_t dfS, uint32_t B,
@@ -1714,7 +1717,8 @@ constexpr uint8_t kLevFilt = 7;            // qlev: candidates are the query's f
 constexpr uint32_t kFiltMin = 65536;       // pre-filter queries with more candidates than this
 constexpr uint32_t kFiltCap = 65536;       // keys kept per filtered query (else fall back)
 constexpr uint32_t kFiltSample = kTopkSmem;
-constexpr size_t kFiltSlots = 256;         // filtered queries per batch (the rest: no filter)
+constexpr size_t kFiltSlots = 256;
+constexpr uint64_t kFiltBatchMin = 64ull << 20;   // see topk_filter_on         // filtered queries per batch (the rest: no filter)
 
 __device__ __forceinline__ const uint64_t *cand_keys(const CandBufs &cb, const TopkState &ts,
                                                      uint32_t lev, uint32_t q) {
@@ -2252,12 +2256,22 @@ static cudaError_t launch_intersect(griffin_index *ix, const RoundArgs &ra, cuda
 
 // Top-k candidate buffers for a batch of nq queries with this k (grow-only;
 // called before a CUDA-graph capture so no allocation happens inside it).
+// Pre-filter policy: always for k > 64 (one chunk level keeps k of kTopkSmem
+// keys, so a large k needs up to 4 levels over sets shrinking only ~4x); for
+// k <= 64 only when the batch may hold > kFiltBatchMin candidates (C4/C5-size
+// batches: one level over 10^8 keys costs more than sample + filter, while at
+// C2 the extra launches cost 0.03 ms).  topk_filter: 0 off, 1 auto, 2 always.
+static bool topk_filter_on(const griffin_index *ix, const Workspace &w, uint32_t k) {
+  if (ix->topk_filter == 2) return true;
+  return ix->topk_filter == 1 && (k > 64 || w.entry_cap > kFiltBatchMin);
+}
+
 griffin_status reserve_topk(griffin_index *ix, Workspace &w, uint32_t nq, uint32_t k) {
   const uint64_t cand_cap = (w.entry_cap / kTopkSmem + nq + 1) * (uint64_t)k;
   const int levels = k <= 64 ? 1 : (k <= 1024 ? 4 : (k <= 2048 ? kTopkMaxLevels : 0));
   GRIFFIN_CUDA_TRY(w.cand.reserve(cand_cap * 8 * std::max(levels, 1)));
   GRIFFIN_CUDA_TRY(w.tkstate.reserve(((size_t)nq + 1) * (1 + 8 + 4) + 64));
-  if (ix->topk_filter && k > 64 && w.entry_cap > kFiltMin && nq >= 2) {   // a query may exceed kFiltMin
+  if (topk_filter_on(ix, w, k) && w.entry_cap > kFiltMin && nq >= 2) {   // a query may exceed kFiltMin
     const size_t slots = std::min<size_t>(nq, kFiltSlots);
     GRIFFIN_CUDA_TRY(w.flt.reserve(slots * kFiltCap * 8));
     GRIFFIN_CUDA_TRY(w.fstate.reserve(((size_t)nq + 1) * 12 + slots * 4 + 64));
@@ -2437,7 +2451,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     // for k > 64 (one chunk level keeps k of kTopkSmem keys, so large k needs
     // up to 4 levels over shrinking-by-4x sets; C5 top-1000: 3.12 -> 1.29 ms);
     // for k <= 64 one level already shrinks 64x and the extra launches cost more
-    if (ix->topk_filter && k > 64 && w.flt.p && w.fstate.p && nq >= 2) {
+    if (topk_filter_on(ix, w, k) && w.flt.p && w.fstate.p && nq >= 2) {
       ts.fmax = (uint32_t)std::min<size_t>(w.flt.bytes / (kFiltCap * 8), kFiltSlots);
       ts.flt = w.flt.as<uint64_t>();
       ts.ftau = w.fstate.as<uint64_t>();
