@@ -33,6 +33,27 @@ namespace griffin {
 constexpr int kIntersectThreads = 256;
 constexpr int kWarpsPerCta = kIntersectThreads / 32;
 constexpr uint32_t kTopkSmem = 4096;
+#ifndef GRIFFIN_EMIT_DEPTH
+#define GRIFFIN_EMIT_DEPTH 1
+#endif
+#ifndef GRIFFIN_SKIP_DEPTH
+#define GRIFFIN_SKIP_DEPTH 2
+#endif
+// Work per lane kept in flight by the intersect kernel's inner loops.  The
+// kernel runs 3 CTAs x 8 warps per SM at the 80-register cap; deeper loops
+// spilled (C2 round-1+2 intersect, ms: emission depth 4 / 2 / 1 = 0.653 /
+// 0.626 / 0.607; arena probes 4 / 2 = 0.697 / 0.655; skip searches 4 / 2 =
+// 0.605 / 0.603 — profiles/r01_configs.jsonl, session 3).
+constexpr int kEmitDepth = GRIFFIN_EMIT_DEPTH;   // survivors per lane per emission pass (gathers in flight)
+constexpr int kSkipDepth = GRIFFIN_SKIP_DEPTH;   // interleaved skip-pointer searches per lane
+#ifndef GRIFFIN_MERGE_UNROLL
+#define GRIFFIN_MERGE_UNROLL 4
+#endif
+constexpr int kMergeUnroll = GRIFFIN_MERGE_UNROLL;
+#ifndef GRIFFIN_IK_PAIR
+#define GRIFFIN_IK_PAIR 1
+#endif
+constexpr bool kIkPair = GRIFFIN_IK_PAIR;   // intersect kernel: two-blocks-per-warp decoder at B = 128
 constexpr int kTopkThreads = 512;
 
 // ------------------------------------------------------------------- planning
@@ -285,12 +306,12 @@ __device__ __forceinline__ void stage_blocks(const DevIndex &ix, WarpSmem &w, ui
 // Decode the staged blocks whose (meta word y, first docID f, staged offset so in
 // 16-B units) sit in lanes [l0, l0+nb) into dst + i*B: two blocks per warp
 // instruction stream when B = 128 (warp_decode_pair_staged), else one.
-template <class Sink>
+template <class Sink, bool PAIR = true>
 __device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t B, uint32_t l0,
                                                     uint32_t nb, uint32_t y, uint32_t f,
                                                     uint32_t so, uint32_t *dst, Sink &sink) {
   uint32_t i0 = 0;
-  if (B == 128u) {   // pairs; an odd last block takes the single-block decoder
+  if (PAIR && B == 128u) {   // pairs; an odd last block takes the single-block decoder
     const uint32_t npair = nb & ~1u;
     for (uint32_t i = 0; i < npair; i += 2) {
       const uint32_t la = l0 + i, lb = (l0 + i + 1) & 31u;
@@ -311,17 +332,18 @@ __device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t 
     }
   }
 }
+template <bool PAIR = true>
 __device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t B, uint32_t l0,
                                                     uint32_t nb, uint32_t y, uint32_t f,
                                                     uint32_t so, uint32_t *dst) {
   StoreSink s;
-  decode_staged_lanes(w, B, l0, nb, y, f, so, dst, s);
+  decode_staged_lanes<StoreSink, PAIR>(w, B, l0, nb, y, f, so, dst, s);
 }
 
 // EF-decode the consecutive blocks held by lanes [l0, l0+nb) (meta m, first f,
 // payload size sz in 16-B units; contiguous in the payload) into dst + i*B,
 // staging them with TMA bulk copies in batches that fit the staging area.
-template <class Sink>
+template <class Sink, bool PAIR = true>
 __device__ __forceinline__ void stage_decode_lanes(const DevIndex &ix, WarpSmem &w, uint32_t cap16,
                                                    uint32_t l0, uint32_t nb, uint2 m, uint32_t f,
                                                    uint32_t sz, uint32_t *dst, Sink &sink) {
@@ -344,15 +366,16 @@ __device__ __forceinline__ void stage_decode_lanes(const DevIndex &ix, WarpSmem 
     }
     mbar_wait(w.mbar, w.phase);
     w.phase ^= 1u;
-    decode_staged_lanes(w, ix.B, li, nbat, m.y, f, m.x - m0, dst + i * ix.B, sink);
+    decode_staged_lanes<Sink, PAIR>(w, ix.B, li, nbat, m.y, f, m.x - m0, dst + i * ix.B, sink);
     i += nbat;
   }
 }
+template <bool PAIR = true>
 __device__ __forceinline__ void stage_decode_lanes(const DevIndex &ix, WarpSmem &w, uint32_t cap16,
                                                    uint32_t l0, uint32_t nb, uint2 m, uint32_t f,
                                                    uint32_t sz, uint32_t *dst) {
   StoreSink s;
-  stage_decode_lanes(ix, w, cap16, l0, nb, m, f, sz, dst, s);
+  stage_decode_lanes<StoreSink, PAIR>(ix, w, cap16, l0, nb, m, f, sz, dst, s);
 }
 
 // Load R "block" k of an intermediate (chunk of B entries) into dst.
@@ -452,11 +475,11 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
     scr[lane] = incl;
     __syncwarp();
     uint2 *dst = a.bump + off;
-    for (uint32_t j0 = 0; j0 < cnt; j0 += 128) {
-      uint32_t doc[4], tS_[4], tR_[4], prev[4];
-      float nrm[4];
+    for (uint32_t j0 = 0; j0 < cnt; j0 += 32u * kEmitDepth) {
+      uint32_t doc[kEmitDepth], tS_[kEmitDepth], tR_[kEmitDepth], prev[kEmitDepth];
+      float nrm[kEmitDepth];
 #pragma unroll
-      for (int t = 0; t < 4; ++t) {
+      for (int t = 0; t < kEmitDepth; ++t) {
         const uint32_t j = j0 + 32u * t + lane;
         if (j < cnt) {
           uint32_t o = 0;   // owner lane: number of lanes with incl <= j
@@ -475,7 +498,7 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
         }
       }
 #pragma unroll
-      for (int t = 0; t < 4; ++t) {
+      for (int t = 0; t < kEmitDepth; ++t) {
         const uint32_t j = j0 + 32u * t + lane;
         if (j < cnt) {
           const float wS = bm25_w(tS.idf, tS_[t], nrm[t], ix.k1p1);
@@ -714,7 +737,7 @@ __device__ __forceinline__ void warp_upper_bound2(const uint32_t *__restrict__ a
 // every `stride`-th skip pointer of [k_lo, k_hi) is sampled into shared memory
 // in one coalesced pass, each element binary-searches the sample there, and only
 // the last log2(stride) steps touch global memory, as interleaved independent
-// chains (4 elements per lane).  Also resets match[].
+// chains (kSkipDepth elements per lane).  Also resets match[].
 __device__ __forceinline__ void skip_blocks_sampled(const uint32_t *__restrict__ fS, uint32_t k_lo,
                                                     uint32_t k_hi, const uint32_t *tileR,
                                                     uint32_t n, uint32_t *kidx, uint32_t *match,
@@ -726,10 +749,10 @@ __device__ __forceinline__ void skip_blocks_sampled(const uint32_t *__restrict__
   const uint32_t ns = (span + stride - 1) / stride;
   for (uint32_t i = lane; i < ns; i += 32) samp[i] = __ldg(fS + k_lo + i * stride);
   __syncwarp();
-  for (uint32_t base = 0; base < n; base += 128) {
-    uint32_t lo[4], hi[4], xv[4];
+  for (uint32_t base = 0; base < n; base += 32u * kSkipDepth) {
+    uint32_t lo[kSkipDepth], hi[kSkipDepth], xv[kSkipDepth];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
+    for (int j = 0; j < kSkipDepth; ++j) {
       const uint32_t e = base + lane + 32u * j;
       xv[j] = e < n ? tileR[e] : 0u;
       // sample interval: t = #samples <= x; the answer lies in (k_lo+(t-1)*stride, k_lo+t*stride]
@@ -744,7 +767,7 @@ __device__ __forceinline__ void skip_blocks_sampled(const uint32_t *__restrict__
     for (;;) {
       bool any = false;
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
+      for (int j = 0; j < kSkipDepth; ++j) {
         if (lo[j] < hi[j]) {
           const uint32_t mid = (lo[j] + hi[j]) >> 1;
           if (__ldg(fS + mid) <= xv[j]) lo[j] = mid + 1; else hi[j] = mid;
@@ -754,7 +777,7 @@ __device__ __forceinline__ void skip_blocks_sampled(const uint32_t *__restrict__
       if (!__any_sync(0xffffffffu, any)) break;
     }
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
+    for (int j = 0; j < kSkipDepth; ++j) {
       const uint32_t e = base + lane + 32u * j;
       if (e < n) {
         kidx[e] = lo[j] - 1u;   // kNone (0 - 1) when x < fS[k_lo] and k_lo == 0
@@ -771,7 +794,7 @@ __device__ __forceinline__ void skip_blocks_sampled(const uint32_t *__restrict__
 // range [first[kb], first[kb+1]) lands in or next to the right 8-key chunk (one
 // 32-B sector, 32-B aligned): load it, step one chunk left/right until x is
 // bracketed, then compare.  ~1-2 dependent sector loads per probe instead of
-// log2(B) for a binary search.  kEpl independent probes per lane run in
+// log2(B) for a binary search.  kArenaEpl independent probes per lane run in
 // lockstep so their loads overlap.  Writes match[e] = kb*B + pos on a hit and
 // returns the number of chunks loaded.
 #ifndef GRIFFIN_ARENA_EPL
@@ -1217,12 +1240,12 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         // R and S tiles are contiguous: one pass over every compressed block
         const uint32_t l0 = rcomp ? 0u : nRb;
         const uint32_t nbd = (rcomp ? nRb : 0u) + (sdec ? 0u : nSb);
-        if (nbd) decode_staged_lanes(sm, B, l0, nbd, m.y, f, soff, rcomp ? sm.tile : tileS);
+        if (nbd) decode_staged_lanes<kIkPair>(sm, B, l0, nbd, m.y, f, soff, rcomp ? sm.tile : tileS);
       } else {
 #pragma unroll 1
         for (uint32_t jb = 0; jb < 2; ++jb) {
           if (jb == 0 ? rcomp : !sdec)
-            stage_decode_lanes(ix, sm, cap16, jb ? nRb : 0u, jb ? nSb : nRb, m, f, sz,
+            stage_decode_lanes<kIkPair>(ix, sm, cap16, jb ? nRb : 0u, jb ? nSb : nRb, m, f, sz,
                                jb ? tileS : sm.tile);
         }
       }
@@ -1293,7 +1316,7 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         const uint32_t paE = smem_u32(A + ie);
         const uint32_t pm0 = smem_u32(ml);
         uint32_t pm = pm0;
-#pragma unroll 4
+#pragma unroll kMergeUnroll
         for (uint32_t t = 0; t < L; ++t) {
           uint32_t x, y;
           asm volatile("ld.shared.u32 %0, [%1];" : "=r"(x) : "r"(pa));
