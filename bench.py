@@ -461,7 +461,7 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(WORKLOAD_DESC))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--latency-queries", type=int, default=1000)
-    ap.add_argument("--streams", type=int, default=2,
+    ap.add_argument("--streams", type=int, default=3,
                     help="batches in flight on separate streams/workspaces (N=1 only)")
     ap.add_argument("--shard-mode", default="docid", choices=["docid", "replicate"],
                     help="N>1: docID-range shards + exchange, or a replicated index per rank")
