@@ -212,6 +212,17 @@ __device__ __forceinline__ uint32_t decode8(const uint32_t *__restrict__ stg,
         lv[j] = (x1 >> (j * b)) & mask;
         lv[j + 4] = (x2 >> (j * b)) & mask;
       }
+    } else if (b <= 16u) {
+      // two low fields per 32-bit window (most postings of the C2/C5 indexes
+      // have b in 9..16): half the shared loads and address math of one
+      // window per element
+#pragma unroll
+      for (uint32_t j = 0; j < 8; j += 2) {
+        const uint32_t q = bp + j * b;
+        const uint32_t x = __funnelshift_r(stg[q >> 5], stg[(q >> 5) + 1], q);
+        lv[j] = x & mask;
+        lv[j + 1] = (x >> b) & mask;
+      }
     } else {
 #pragma unroll
       for (uint32_t j = 0; j < 8; ++j) {
