@@ -34,8 +34,7 @@ static griffin_status invalid(const std::string &m) {
   return GRIFFIN_ERR_INVALID_ARG;
 }
 
-static griffin_status ensure_pinned(griffin_index *ix, size_t bytes) {
-  Workspace &w = ix->ws;
+static griffin_status ensure_pinned_ws(Workspace &w, size_t bytes) {
   if (w.h_pinned_bytes >= bytes) return GRIFFIN_OK;
   if (w.h_pinned) cudaFreeHost(w.h_pinned);
   w.h_pinned = nullptr;
@@ -44,6 +43,9 @@ static griffin_status ensure_pinned(griffin_index *ix, size_t bytes) {
   GRIFFIN_CUDA_TRY(cudaMallocHost(&w.h_pinned, nb));
   w.h_pinned_bytes = nb;
   return GRIFFIN_OK;
+}
+static griffin_status ensure_pinned(griffin_index *ix, size_t bytes) {
+  return ensure_pinned_ws(ix->ws, bytes);
 }
 
 // Host validation of one batch's query terms + workspace reservation.
@@ -57,15 +59,21 @@ static griffin_status reserve_for(griffin_index *ix, Workspace &w, uint32_t nq,
     if (qoffs[q + 1] < qoffs[q]) return invalid("query_offsets must be non-decreasing");
     const uint32_t n = qoffs[q + 1] - qoffs[q];
     if (n == 0) return invalid("a query has no terms");
-    std::vector<uint32_t> ts(terms + qoffs[q], terms + qoffs[q + 1]);
-    for (uint32_t t : ts)
+    // distinct terms without heap allocation (<= GRIFFIN_MAX_TERMS are valid)
+    uint32_t ts[GRIFFIN_MAX_TERMS];
+    uint32_t nd = 0;
+    for (const uint32_t *p = terms + qoffs[q], *e = terms + qoffs[q + 1]; p < e; ++p) {
+      const uint32_t t = *p;
       if (t >= ix->V) return invalid("query term >= num_terms");
-    std::sort(ts.begin(), ts.end());
-    ts.erase(std::unique(ts.begin(), ts.end()), ts.end());
-    if (ts.size() > (size_t)GRIFFIN_MAX_TERMS) return invalid("more than GRIFFIN_MAX_TERMS distinct terms");
-    mt = std::max<uint32_t>(mt, (uint32_t)ts.size());
+      bool dup = false;
+      for (uint32_t i = 0; i < nd; ++i) dup |= ts[i] == t;
+      if (dup) continue;
+      if (nd == GRIFFIN_MAX_TERMS) return invalid("more than GRIFFIN_MAX_TERMS distinct terms");
+      ts[nd++] = t;
+    }
+    mt = std::max<uint32_t>(mt, nd);
     uint64_t c, u;
-    host_query_bounds(ix, terms + qoffs[q], n, &c, &u);
+    host_query_bounds(ix, ts, nd, &c, &u);
     caps += c;
     units += u;
   }
@@ -73,15 +81,15 @@ static griffin_status reserve_for(griffin_index *ix, Workspace &w, uint32_t nq,
   return reserve_ws(ix, w, nq, units, caps);
 }
 
-static griffin_status read_status(griffin_index *ix, Workspace &w) {
+static griffin_status read_status(griffin_index *ix, Workspace &w, cudaStream_t st = nullptr) {
+  if (!st) st = ix->stream;
   int status = 0;
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(&status, w.scal.as<unsigned long long>() + kScalStatus,
-                                   sizeof(int), cudaMemcpyDeviceToHost, ix->stream));
-  GRIFFIN_CUDA_TRY(cudaStreamSynchronize(ix->stream));
+                                   sizeof(int), cudaMemcpyDeviceToHost, st));
+  GRIFFIN_CUDA_TRY(cudaStreamSynchronize(st));
   if (status) {
-    GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.scal.as<unsigned long long>() + kScalStatus, 0, 8,
-                                     ix->stream));
-    GRIFFIN_CUDA_TRY(cudaStreamSynchronize(ix->stream));
+    GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.scal.as<unsigned long long>() + kScalStatus, 0, 8, st));
+    GRIFFIN_CUDA_TRY(cudaStreamSynchronize(st));
     if (status & kStatusOverflow) {
       set_error("query workspace overflow (reserve more with griffin_reserve)");
       return GRIFFIN_ERR_OOM;
@@ -504,7 +512,8 @@ static void free_workspace(Workspace &w) {
                     &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.uperm, &w.rbuf0,
                     &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys, &w.counts,
                     &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand, &w.tdec, &w.runs,
-                    &w.run_base, &w.vtmp, &w.run_term, &w.arena})
+                    &w.run_base, &w.vtmp, &w.run_term, &w.arena, &w.sbkt_cnt, &w.sbkt_pos,
+                    &w.sbkt_tmp, &w.flt, &w.fstate})
     b->release();
   if (w.h_pinned) cudaFreeHost(w.h_pinned);
   w.h_pinned = nullptr;

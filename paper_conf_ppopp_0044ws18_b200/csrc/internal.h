@@ -210,7 +210,7 @@ griffin_status copy_final_docids(griffin_index *ix, uint32_t *h_out, uint64_t ca
 inline uint32_t probe_chunk(const griffin_index *ix) {
   return ix->P ? ix->P : (ix->B / 2 >= 32 ? ix->B / 2 : 32u);
 }
-void host_query_bounds(const griffin_index *ix, const uint32_t *terms, uint32_t nterms,
-                       uint64_t *cap, uint64_t *units);
+void host_query_bounds(const griffin_index *ix, uint32_t *ts, uint32_t n, uint64_t *cap,
+                       uint64_t *units);
 
 }  // namespace griffin

@@ -2591,33 +2591,36 @@ griffin_status copy_final_docids(griffin_index *ix, uint32_t *h_out, uint64_t ca
   return GRIFFIN_OK;
 }
 
-void host_query_bounds(const griffin_index *ix, const uint32_t *terms, uint32_t nterms,
-                       uint64_t *cap, uint64_t *units) {
-  std::vector<uint32_t> ts(terms, terms + nterms);
-  std::sort(ts.begin(), ts.end());
-  ts.erase(std::unique(ts.begin(), ts.end()), ts.end());
+// Workspace bounds of one query (host): cap = entries of its round-1 region,
+// units = an upper bound of its units in any round.  `ts` = its distinct terms
+// (any order, all < V, 1..kMaxTerms of them); sorted here into SvS order.
+void host_query_bounds(const griffin_index *ix, uint32_t *ts, uint32_t n, uint64_t *cap,
+                       uint64_t *units) {
   *cap = 0;
   *units = 0;
-  for (uint32_t t : ts)
-    if (t >= ix->V) return;
-  if (ts.empty() || ts.size() > (size_t)kMaxTerms) return;
-  std::sort(ts.begin(), ts.end(), [&](uint32_t a, uint32_t b) {
+  auto less = [&](uint32_t a, uint32_t b) {
     const uint32_t da = ix->h_terms[a].df_global, db = ix->h_terms[b].df_global;
     return da != db ? da < db : a < b;
-  });
-  for (uint32_t t : ts)
-    if (ix->h_terms[t].df_local == 0) return;
+  };
+  for (uint32_t i = 1; i < n; ++i) {   // insertion sort: n <= kMaxTerms
+    const uint32_t x = ts[i];
+    uint32_t j = i;
+    for (; j > 0 && less(x, ts[j - 1]); --j) ts[j] = ts[j - 1];
+    ts[j] = x;
+  }
+  for (uint32_t i = 0; i < n; ++i)
+    if (ix->h_terms[ts[i]].df_local == 0) return;
   const TermInfo &t0 = ix->h_terms[ts[0]];
-  if (ts.size() == 1) {
+  if (n == 1) {
     *cap = t0.df_local;
     *units = t0.nblocks;
     return;
   }
   *cap = std::min(t0.df_local, ix->h_terms[ts[1]].df_local);
   uint32_t mx = 0;
-  for (size_t i = 1; i < ts.size(); ++i) mx = std::max(mx, ix->h_terms[ts[i]].nblocks);
+  for (uint32_t i = 1; i < n; ++i) mx = std::max(mx, ix->h_terms[ts[i]].nblocks);
   const uint32_t P = probe_chunk(ix);   // probe-pass units: ceil(|R| / P), |R| <= cap
-  if (ts.size() >= 3) mx = std::max<uint32_t>(mx, (uint32_t)((*cap + P - 1) / P));
+  if (n >= 3) mx = std::max<uint32_t>(mx, (uint32_t)((*cap + P - 1) / P));
   *units = (uint64_t)t0.nblocks + mx;
 }
 

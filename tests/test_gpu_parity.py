@@ -322,12 +322,27 @@ def test_c2_full_size_sampled():
 def test_large_batch_s_locality_order():
     """Batches of >= 4096 queries hand out merge units in S-locality order
     (sorder_scatter_kernel); the results must not depend on it."""
+    import torch
     c, ql, cfg = make_workload("small", num_queries=5000)
     gx = g.GriffinIndex(c, block_size=128)
     ox = oracle.OracleIndex(c, block_size=128)
-    d, s, cn = gx.griffin_query_batch(ql.offsets, ql.terms, 10)
-    od, os_, oc = ox.query_batch(ql, 10, nthreads=4)
-    assert_topk_equal(d, s, cn, od, os_, oc)
+    k, nq = 10, ql.num_queries
+    # device API: one batch of all 5000 queries (the host API would slice it)
+    gx.griffin_reserve(ql.offsets, ql.terms, k)
+    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
+    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
+    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(nq, dtype=torch.int32, device="cuda")
+    gx.griffin_query_batch_device(d_off, d_t, mt, k, keys, cnt, torch.cuda.current_stream())
+    dd = torch.zeros(nq * k, dtype=torch.int32, device="cuda")
+    ds = torch.zeros(nq * k, dtype=torch.float32, device="cuda")
+    gx.griffin_keys_to_results_device(nq, k, keys, cnt, dd, ds)
+    torch.cuda.synchronize()
+    gx.griffin_sync_status()
+    od, os_, oc = ox.query_batch(ql, k, nthreads=4)
+    assert_topk_equal(dd.cpu().numpy().view(np.uint32).reshape(nq, k), ds.cpu().numpy().reshape(nq, k),
+                      cnt.cpu().numpy().view(np.uint32), od, os_, oc)
 
 
 def _sub_corpus(c, terms):
