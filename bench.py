@@ -345,20 +345,42 @@ def run_gpu(args):
     if world > 1:
         h_off = torch.from_numpy(ql.offsets.astype(np.int32)).pin_memory()
         h_terms = torch.from_numpy(ql.terms.astype(np.int32)).pin_memory()
-    for i in range(args.warmup + args.steps):
+    if not sharded:
+        # griffin_query_batch split into submit/collect over the slots'
+        # workspaces: the same host-buffer call with len(slots) batches in
+        # flight (H2D of the queries, the path, D2H of the results per batch)
+        e2e_ws = [sl[0] for sl in slots[1:]] + [ix.griffin_workspace_create()]
+        e2e_st = [sl[1] for sl in slots[1:]] + [stream]
+        for w in e2e_ws[len(slots) - 1:]:
+            w.griffin_workspace_reserve(ql.offsets, ql.terms, k)
+
+        def e2e_run(n):
+            nw = len(e2e_ws)
+            for i in range(n):
+                w = e2e_ws[i % nw]
+                if i >= nw:
+                    w.griffin_query_batch_collect()
+                w.griffin_query_batch_submit(ql.offsets, ql.terms, k, e2e_st[i % nw])
+            for i in range(max(0, n - nw), n):
+                e2e_ws[i % nw].griffin_query_batch_collect()
+
+        e2e_run(args.warmup)
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
-        if not sharded:
-            dd, ss, cc = ix.griffin_query_batch(ql.offsets, ql.terms, k)
+        e2e_run(args.steps)
+        e2e_times.append(time.perf_counter() - t0)
+    for i in range(args.warmup + args.steps if sharded else 0):
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        e_off = h_off.to("cuda", non_blocking=True)
+        e_terms = h_terms.to("cuda", non_blocking=True)
+        if args.exchange == "allgather":
+            dd, ss, cc = searcher.search(e_off, e_terms, max_terms, k, stream)
         else:
-            e_off = h_off.to("cuda", non_blocking=True)
-            e_terms = h_terms.to("cuda", non_blocking=True)
-            if args.exchange == "allgather":
-                dd, ss, cc = searcher.search(e_off, e_terms, max_terms, k, stream)
-            else:
-                _, _, dd, ss, cc = searcher.search_sliced(e_off, e_terms, max_terms, k, stream)
-            dd, ss, cc = dd.cpu(), ss.cpu(), cc.cpu()
+            _, _, dd, ss, cc = searcher.search_sliced(e_off, e_terms, max_terms, k, stream)
+        dd, ss, cc = dd.cpu(), ss.cpu(), cc.cpu()
         dt = time.perf_counter() - t0
         if i >= args.warmup:
             e2e_times.append(dt)
@@ -419,7 +441,9 @@ def run_gpu(args):
         "e2e": {"value": (world if replicate else 1) * nq * args.steps / e2e_s,
                 "unit": "queries/s", "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": d2h,
-                "how": "griffin_query_batch (host buffers; pinned staging, H2D queries, D2H results)"},
+                "how": ("griffin_query_batch_submit/collect (host buffers; pinned staging, H2D queries, "
+                        "D2H results), batches_in_flight workspaces" if not sharded else
+                        "ShardedSearcher.search (pinned H2D queries, D2H results)")},
         "clocks": clk,
     }
     # decode-only sweep over every block of the shard (SURVEY §8(d) C5 sweep row)

@@ -182,6 +182,24 @@ griffin_status griffin_query_batch_device_ws(griffin_index *ix, griffin_workspac
                                              uint32_t *d_out_counts, void *stream);
 griffin_status griffin_workspace_sync_status(griffin_index *ix, griffin_workspace *ws);
 
+/* griffin_query_batch (host buffers, same arguments, validation and results)
+ * split into an enqueue and a wait on one workspace, so a caller holding several
+ * workspaces keeps several batches — H2D of the queries, the whole path, D2H of
+ * the results — in flight on different streams.  submit validates the batch on
+ * the host, copies query_offsets/terms into the workspace's pinned staging
+ * (the caller's arrays may be reused as soon as it returns) and enqueues
+ * everything on `stream` (NULL: the index's stream); it fails with
+ * GRIFFIN_ERR_INVALID_ARG if the workspace still holds an uncollected batch.
+ * collect waits for that batch and writes [nq*k] docIDs, [nq*k] scores and
+ * [nq] counts exactly as griffin_query_batch does; a device-detected error
+ * (workspace overflow, bad term) is returned here. */
+griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
+                                          const uint32_t *query_offsets, const uint32_t *terms,
+                                          uint32_t k, void *stream);
+griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace *ws,
+                                           uint32_t *out_docids, float *out_scores,
+                                           uint32_t *out_counts);
+
 /* Shard merge: given G per-shard sorted key runs
  * d_keys[g][nq*k] and counts d_counts[g][nq] (laid out contiguously, g-major, as
  * an all-gather produces them), write the global top-k keys and counts.  Exact:

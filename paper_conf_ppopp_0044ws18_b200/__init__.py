@@ -91,6 +91,8 @@ _SIGS = {
     "griffin_workspace_reserve": [_vp, _vp, _u32, _vp, _vp, _u32],
     "griffin_query_batch_device_ws": [_vp, _vp, _u32, _vp, _vp, _u32, _u32, _vp, _vp, _vp],
     "griffin_workspace_sync_status": [_vp, _vp],
+    "griffin_query_batch_submit": [_vp, _vp, _u32, _vp, _vp, _u32, _vp],
+    "griffin_query_batch_collect": [_vp, _vp, _vp, _vp, _vp],
     "griffin_merge_topk_device": [_vp, _u32, _u32, _u32, _vp, _vp, _vp, _vp, _vp],
     "griffin_keys_to_results_device": [_vp, _u32, _u32, _vp, _vp, _vp, _vp, _vp],
     "griffin_set_mode": [_vp, ctypes.c_int],
@@ -375,6 +377,25 @@ class GriffinWorkspace:
 
     def griffin_workspace_sync_status(self):
         _check(load_library().griffin_workspace_sync_status(self.index.h, self.h))
+
+    # -- pipelined host-buffer batch (griffin_query_batch_submit / _collect)
+    def griffin_query_batch_submit(self, offsets, terms, k: int, stream=None):
+        off = np.ascontiguousarray(offsets, np.uint32)
+        t = np.ascontiguousarray(terms, np.uint32)
+        st = ctypes.c_void_p(stream.cuda_stream if stream is not None else 0)
+        _check(load_library().griffin_query_batch_submit(self.index.h, self.h, len(off) - 1,
+                                                         _ptr(off), _ptr(t), k, st))
+        self._pend = (len(off) - 1, k)
+
+    def griffin_query_batch_collect(self):
+        nq, k = getattr(self, "_pend", (0, 1))
+        d = np.zeros(max(nq * k, 1), np.uint32)
+        s = np.zeros(max(nq * k, 1), np.float32)
+        c = np.zeros(max(nq, 1), np.uint32)
+        _check(load_library().griffin_query_batch_collect(self.index.h, self.h, _ptr(d), _ptr(s),
+                                                          _ptr(c)))
+        self._pend = (0, 1)
+        return d[:nq * k].reshape(nq, k), s[:nq * k].reshape(nq, k), c[:nq]
 
 
 class PfdStats(ctypes.Structure):

@@ -517,6 +517,10 @@ static void free_workspace(Workspace &w) {
     b->release();
   if (w.h_pinned) cudaFreeHost(w.h_pinned);
   w.h_pinned = nullptr;
+  w.h_pinned_bytes = 0;
+  if (w.done) cudaEventDestroy(w.done);
+  w.done = nullptr;
+  w.pending = false;
 }
 
 void griffin_workspace_destroy(griffin_index *ix, griffin_workspace *ws) {
@@ -562,6 +566,97 @@ griffin_status griffin_workspace_sync_status(griffin_index *ix, griffin_workspac
   Workspace &w = *reinterpret_cast<Workspace *>(ws);
   if (!w.scal.p) return GRIFFIN_OK;
   return read_status(ix, w);
+}
+
+// Host-buffer batch split into an enqueue and a wait, so a caller with several
+// workspaces keeps several batches (H2D of the queries, the path, D2H of the
+// results) in flight: the same staging as griffin_query_batch, but into the
+// workspace's own pinned buffer, plus the status word, then an event.
+griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
+                                          const uint32_t *qoffs, const uint32_t *terms,
+                                          uint32_t k, void *stream) {
+  if (!ix || !ws) return invalid("null argument");
+  if (nq && (!qoffs || !terms)) return invalid("null argument");
+  Workspace &w = *reinterpret_cast<Workspace *>(ws);
+  if (w.pending) return invalid("workspace has a submitted batch not yet collected");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  DeviceGuard guard(ix->device);
+  cudaStream_t st = stream ? static_cast<cudaStream_t>(stream) : ix->stream;
+  uint32_t max_terms = 1;
+  griffin_status s = GRIFFIN_OK;
+  if (nq && (s = reserve_for(ix, w, nq, qoffs, terms, k, &max_terms))) return s;
+  if (!nq && (k == 0 || k > GRIFFIN_MAX_K)) return invalid("k must be in [1, 4096]");
+  const uint64_t nt = nq ? qoffs[nq] : 0;
+  const size_t nk = (size_t)nq * k;
+  // pinned staging: [qoffs | terms | docids | scores | counts | status]
+  const size_t b_in = nq ? ((size_t)nq + 1 + nt) * 4 : 0;
+  const size_t b_out = nk * 8 + (size_t)nq * 4;
+  if ((s = ensure_pinned_ws(w, b_in + b_out + 8))) return s;
+  if (!w.done) GRIFFIN_CUDA_TRY(cudaEventCreateWithFlags(&w.done, cudaEventDisableTiming));
+  uint8_t *hp = static_cast<uint8_t *>(w.h_pinned);
+  int *h_status = reinterpret_cast<int *>(hp + b_in + b_out);
+  *h_status = 0;
+  if (nq) {
+    GRIFFIN_CUDA_TRY(w.qoffs.reserve(((size_t)nq + 1) * 4));
+    GRIFFIN_CUDA_TRY(w.qterms.reserve(std::max<uint64_t>(nt, 1) * 4));
+    GRIFFIN_CUDA_TRY(w.keys.reserve(nk * 8));
+    GRIFFIN_CUDA_TRY(w.counts.reserve((size_t)nq * 4));
+    GRIFFIN_CUDA_TRY(w.docids.reserve(nk * 4));
+    GRIFFIN_CUDA_TRY(w.scores.reserve(nk * 4));
+    std::memcpy(hp, qoffs, ((size_t)nq + 1) * 4);
+    std::memcpy(hp + ((size_t)nq + 1) * 4, terms, nt * 4);
+    GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qoffs.p, hp, ((size_t)nq + 1) * 4, cudaMemcpyHostToDevice, st));
+    GRIFFIN_CUDA_TRY(cudaMemcpyAsync(w.qterms.p, hp + ((size_t)nq + 1) * 4, nt * 4,
+                                     cudaMemcpyHostToDevice, st));
+    if ((s = run_batch(ix, w, nq, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), max_terms, k,
+                       w.keys.as<uint64_t>(), w.counts.as<uint32_t>(), st, true, ix->mode)))
+      return s;
+    if ((s = launch_keys_to_results(ix, nq, k, w.keys.as<uint64_t>(), w.counts.as<uint32_t>(),
+                                    w.docids.as<uint32_t>(), w.scores.as<float>(), st)))
+      return s;
+    uint8_t *ho = hp + b_in;
+    GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho, w.docids.p, nk * 4, cudaMemcpyDeviceToHost, st));
+    GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho + nk * 4, w.scores.p, nk * 4, cudaMemcpyDeviceToHost, st));
+    GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho + nk * 8, w.counts.p, (size_t)nq * 4,
+                                     cudaMemcpyDeviceToHost, st));
+    GRIFFIN_CUDA_TRY(cudaMemcpyAsync(h_status, w.scal.as<unsigned long long>() + kScalStatus,
+                                     sizeof(int), cudaMemcpyDeviceToHost, st));
+  }
+  GRIFFIN_CUDA_TRY(cudaEventRecord(w.done, st));
+  w.pend_stream = st;
+  w.pend_nq = nq;
+  w.pend_k = k;
+  w.pend_out = b_in;
+  w.pending = true;
+  return GRIFFIN_OK;
+}
+
+griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace *ws,
+                                           uint32_t *out_docids, float *out_scores,
+                                           uint32_t *out_counts) {
+  if (!ix || !ws) return invalid("null argument");
+  Workspace &w = *reinterpret_cast<Workspace *>(ws);
+  if (!w.pending) return invalid("no submitted batch on this workspace");
+  const size_t nk = (size_t)w.pend_nq * w.pend_k;
+  if (w.pend_nq && (!out_docids || !out_scores || !out_counts)) return invalid("null argument");
+  {
+    DeviceGuard guard(ix->device);
+    w.pending = false;
+    GRIFFIN_CUDA_TRY(cudaEventSynchronize(w.done));   // without the index lock: others submit
+  }
+  const uint8_t *ho = static_cast<const uint8_t *>(w.h_pinned) + w.pend_out;
+  if (*reinterpret_cast<const int *>(ho + nk * 8 + (size_t)w.pend_nq * 4)) {
+    std::lock_guard<std::mutex> lk(ix->mu);
+    DeviceGuard guard(ix->device);
+    griffin_status s = read_status(ix, w, w.pend_stream);   // clears the device flag
+    if (s) return s;
+  }
+  if (w.pend_nq) {
+    std::memcpy(out_docids, ho, nk * 4);
+    std::memcpy(out_scores, ho + nk * 4, nk * 4);
+    std::memcpy(out_counts, ho + nk * 8, (size_t)w.pend_nq * 4);
+  }
+  return GRIFFIN_OK;
 }
 
 griffin_status griffin_merge_topk_device(griffin_index *ix, uint32_t num_runs, uint32_t nq,

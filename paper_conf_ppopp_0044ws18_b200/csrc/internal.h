@@ -66,6 +66,12 @@ struct Workspace {
   // pinned host staging
   void *h_pinned = nullptr;
   size_t h_pinned_bytes = 0;
+  // griffin_query_batch_submit/collect: the batch in flight on this workspace
+  cudaEvent_t done = nullptr;
+  cudaStream_t pend_stream = nullptr;
+  uint32_t pend_nq = 0, pend_k = 0;
+  size_t pend_out = 0;   // byte offset of the results in h_pinned
+  bool pending = false;
 };
 
 // Offsets of the scalar block (u64 slots).

@@ -560,6 +560,49 @@ def test_concurrent_workspaces_on_two_streams(tiny):
     ws.close()
 
 
+def test_submit_collect_pipelined_workspaces(tiny):
+    """griffin_query_batch_submit/collect with three workspaces in flight on
+    three streams (bench.py's e2e loop): every collected batch is oracle-exact;
+    different batches (varying k and query subsets) do not mix; misuse and a bad
+    term are reported, and the workspace stays usable afterwards."""
+    import torch
+    c, ql, ox = tiny
+    gx = g.GriffinIndex(c, block_size=128)
+    wss = [gx.griffin_workspace_create() for _ in range(3)]
+    sts = [torch.cuda.Stream() for _ in range(3)]
+    nq = ql.num_queries
+    subsets = [(0, nq, 10), (0, nq // 2, 25), (nq // 3, nq, 7), (1, 5, 1), (0, nq, 100)]
+    expect = []
+    for lo, hi, k in subsets:
+        sub = ql.slice(lo, hi)
+        expect.append((sub, k, ox.query_batch(sub, k)))
+    got = [None] * len(expect)
+    for i, (sub, k, _) in enumerate(expect * 2):
+        w = wss[i % 3]
+        if i >= 3:
+            got[(i - 3) % len(expect)] = w.griffin_query_batch_collect()
+        w.griffin_query_batch_submit(sub.offsets, sub.terms, k, sts[i % 3])
+    for i in range(2 * len(expect) - 3, 2 * len(expect)):
+        got[i % len(expect)] = wss[i % 3].griffin_query_batch_collect()
+    for (sub, k, (od, os_, oc)), (gd, gs, gc) in zip(expect, got):
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+    w = wss[0]
+    with pytest.raises(g.GriffinError):
+        w.griffin_query_batch_collect()             # nothing submitted
+    sub, k, (od, os_, oc) = expect[0]
+    w.griffin_query_batch_submit(sub.offsets, sub.terms, k)
+    with pytest.raises(g.GriffinError):
+        w.griffin_query_batch_submit(sub.offsets, sub.terms, k)   # not yet collected
+    assert_topk_equal(*w.griffin_query_batch_collect(), od, os_, oc)
+    with pytest.raises(g.GriffinError):
+        w.griffin_query_batch_submit(np.array([0, 1], np.uint32),
+                                     np.array([c.num_terms], np.uint32), 10)
+    w.griffin_query_batch_submit(sub.offsets, sub.terms, k)
+    assert_topk_equal(*w.griffin_query_batch_collect(), od, os_, oc)
+    for w in wss:
+        w.close()
+
+
 # ---------------------------------------------------------------- EF NextGEQ gallop
 
 def _nextgeq_corpus(rng, N=3_000_000):
