@@ -349,10 +349,9 @@ def run_gpu(args):
         # griffin_query_batch split into submit/collect over the slots'
         # workspaces: the same host-buffer call with len(slots) batches in
         # flight (H2D of the queries, the path, D2H of the results per batch)
-        e2e_ws = [sl[0] for sl in slots[1:]] + [ix.griffin_workspace_create()]
-        e2e_st = [sl[1] for sl in slots[1:]] + [stream]
-        for w in e2e_ws[len(slots) - 1:]:
-            w.griffin_workspace_reserve(ql.offsets, ql.terms, k)
+        # (slot 0 = the index's own workspace; no extra device memory)
+        e2e_ws = [ix] + [sl[0] for sl in slots[1:]]
+        e2e_st = [sl[1] for sl in slots]
 
         def e2e_run(n):
             nw = len(e2e_ws)
@@ -485,8 +484,10 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(WORKLOAD_DESC))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--latency-queries", type=int, default=1000)
-    ap.add_argument("--streams", type=int, default=3,
-                    help="batches in flight on separate streams/workspaces (N=1 only)")
+    ap.add_argument("--streams", type=int, default=None,
+                    help="batches in flight on separate streams/workspaces (N=1 only); default "
+                         "3 for the 1K-query configs, 1 for the 10K-query top-1000 batches "
+                         "(one already fills the GPU; three workspaces of it exceed HBM)")
     ap.add_argument("--shard-mode", default="docid", choices=["docid", "replicate"],
                     help="N>1: docID-range shards + exchange, or a replicated index per rank")
     ap.add_argument("--exchange", default="allgather", choices=["allgather", "sliced"],
@@ -494,6 +495,8 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
+    if args.streams is None:
+        args.streams = 1 if args.config in ("c4", "c5") else 3
     if args.impl == "reference":
         run_reference(args)
     else:

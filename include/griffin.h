@@ -192,7 +192,10 @@ griffin_status griffin_workspace_sync_status(griffin_index *ix, griffin_workspac
  * GRIFFIN_ERR_INVALID_ARG if the workspace still holds an uncollected batch.
  * collect waits for that batch and writes [nq*k] docIDs, [nq*k] scores and
  * [nq] counts exactly as griffin_query_batch does; a device-detected error
- * (workspace overflow, bad term) is returned here. */
+ * (workspace overflow, bad term) is returned here.  ws = NULL: the index's own
+ * workspace (while it holds an uncollected batch, griffin_query,
+ * griffin_query_batch and griffin_query_batch_device fail with
+ * GRIFFIN_ERR_INVALID_ARG). */
 griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
                                           const uint32_t *query_offsets, const uint32_t *terms,
                                           uint32_t k, void *stream);

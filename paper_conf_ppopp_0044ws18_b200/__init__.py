@@ -163,6 +163,24 @@ def _ptr(a: np.ndarray):
     return ctypes.c_void_p(a.ctypes.data)
 
 
+def _submit(ih, wh, offsets, terms, k, stream):
+    off = np.ascontiguousarray(offsets, np.uint32)
+    t = np.ascontiguousarray(terms, np.uint32)
+    st = ctypes.c_void_p(stream.cuda_stream if stream is not None else 0)
+    _check(load_library().griffin_query_batch_submit(ih, wh, len(off) - 1, _ptr(off), _ptr(t), k,
+                                                     st))
+    return (len(off) - 1, k)
+
+
+def _collect(ih, wh, pend):
+    nq, k = pend
+    d = np.zeros(max(nq * k, 1), np.uint32)
+    s = np.zeros(max(nq * k, 1), np.float32)
+    c = np.zeros(max(nq, 1), np.uint32)
+    _check(load_library().griffin_query_batch_collect(ih, wh, _ptr(d), _ptr(s), _ptr(c)))
+    return d[:nq * k].reshape(nq, k), s[:nq * k].reshape(nq, k), c[:nq]
+
+
 def _dptr(t) -> ctypes.c_void_p:
     """device pointer of a torch tensor (plumbing only)"""
     return ctypes.c_void_p(t.data_ptr())
@@ -261,6 +279,15 @@ class GriffinIndex:
 
     def griffin_workspace_create(self) -> "GriffinWorkspace":
         return GriffinWorkspace(self)
+
+    # -- pipelined host-buffer batch on the index's own workspace (ws = NULL)
+    def griffin_query_batch_submit(self, offsets, terms, k: int, stream=None):
+        self._pend = _submit(self.h, None, offsets, terms, k, stream)
+
+    def griffin_query_batch_collect(self):
+        out = _collect(self.h, None, getattr(self, "_pend", (0, 1)))
+        self._pend = (0, 1)
+        return out
 
     def griffin_merge_topk_device(self, num_runs: int, nq: int, k: int, d_keys, d_counts,
                                   d_out_keys, d_out_counts, stream=None):
@@ -380,22 +407,12 @@ class GriffinWorkspace:
 
     # -- pipelined host-buffer batch (griffin_query_batch_submit / _collect)
     def griffin_query_batch_submit(self, offsets, terms, k: int, stream=None):
-        off = np.ascontiguousarray(offsets, np.uint32)
-        t = np.ascontiguousarray(terms, np.uint32)
-        st = ctypes.c_void_p(stream.cuda_stream if stream is not None else 0)
-        _check(load_library().griffin_query_batch_submit(self.index.h, self.h, len(off) - 1,
-                                                         _ptr(off), _ptr(t), k, st))
-        self._pend = (len(off) - 1, k)
+        self._pend = _submit(self.index.h, self.h, offsets, terms, k, stream)
 
     def griffin_query_batch_collect(self):
-        nq, k = getattr(self, "_pend", (0, 1))
-        d = np.zeros(max(nq * k, 1), np.uint32)
-        s = np.zeros(max(nq * k, 1), np.float32)
-        c = np.zeros(max(nq, 1), np.uint32)
-        _check(load_library().griffin_query_batch_collect(self.index.h, self.h, _ptr(d), _ptr(s),
-                                                          _ptr(c)))
+        out = _collect(self.index.h, self.h, getattr(self, "_pend", (0, 1)))
         self._pend = (0, 1)
-        return d[:nq * k].reshape(nq, k), s[:nq * k].reshape(nq, k), c[:nq]
+        return out
 
 
 class PfdStats(ctypes.Structure):

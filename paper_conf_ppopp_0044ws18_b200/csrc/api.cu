@@ -311,6 +311,7 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
   if (!ix) return invalid("null index");
   if (nq == 0) return GRIFFIN_OK;
   if (!qoffs || !terms || !out_docids || !out_scores || !out_counts) return invalid("null argument");
+  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
   uint32_t max_terms = 1;
@@ -457,6 +458,7 @@ griffin_status griffin_query(griffin_index *ix, const uint32_t *terms, uint32_t 
                              uint32_t *out_docids, float *out_scores, uint32_t *out_count) {
   if (nterms == 0) return invalid("nterms must be > 0");
   if (!ix || !terms || !out_docids || !out_scores || !out_count) return invalid("null argument");
+  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
   if (ix->use_graphs && !ix->profiling) {
     std::lock_guard<std::mutex> lk(ix->mu);
     DeviceGuard guard(ix->device);
@@ -483,6 +485,7 @@ griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq, const 
   if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
   if (max_terms == 0 || max_terms > GRIFFIN_MAX_TERMS) return invalid("max_terms out of range");
   if (nq == 0) return GRIFFIN_OK;
+  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
   return run_batch(ix, ix->ws, nq, d_qoffs, d_terms, max_terms, k, d_out_keys, d_out_counts,
@@ -575,9 +578,9 @@ griffin_status griffin_workspace_sync_status(griffin_index *ix, griffin_workspac
 griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
                                           const uint32_t *qoffs, const uint32_t *terms,
                                           uint32_t k, void *stream) {
-  if (!ix || !ws) return invalid("null argument");
+  if (!ix) return invalid("null index");
   if (nq && (!qoffs || !terms)) return invalid("null argument");
-  Workspace &w = *reinterpret_cast<Workspace *>(ws);
+  Workspace &w = ws ? *reinterpret_cast<Workspace *>(ws) : ix->ws;
   if (w.pending) return invalid("workspace has a submitted batch not yet collected");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -634,8 +637,8 @@ griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *
 griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace *ws,
                                            uint32_t *out_docids, float *out_scores,
                                            uint32_t *out_counts) {
-  if (!ix || !ws) return invalid("null argument");
-  Workspace &w = *reinterpret_cast<Workspace *>(ws);
+  if (!ix) return invalid("null index");
+  Workspace &w = ws ? *reinterpret_cast<Workspace *>(ws) : ix->ws;
   if (!w.pending) return invalid("no submitted batch on this workspace");
   const size_t nk = (size_t)w.pend_nq * w.pend_k;
   if (w.pend_nq && (!out_docids || !out_scores || !out_counts)) return invalid("null argument");

@@ -599,6 +599,13 @@ def test_submit_collect_pipelined_workspaces(tiny):
                                      np.array([c.num_terms], np.uint32), 10)
     w.griffin_query_batch_submit(sub.offsets, sub.terms, k)
     assert_topk_equal(*w.griffin_query_batch_collect(), od, os_, oc)
+    # the index's own workspace (ws = NULL) blocks the synchronous calls while
+    # it holds a batch
+    gx.griffin_query_batch_submit(sub.offsets, sub.terms, k)
+    with pytest.raises(g.GriffinError):
+        gx.griffin_query_batch(sub.offsets, sub.terms, k)
+    assert_topk_equal(*gx.griffin_query_batch_collect(), od, os_, oc)
+    assert_topk_equal(*gx.griffin_query_batch(sub.offsets, sub.terms, k), od, os_, oc)
     for w in wss:
         w.close()
 
