@@ -353,15 +353,19 @@ def run_gpu(args):
         e2e_ws = [ix] + [sl[0] for sl in slots[1:]]
         e2e_st = [sl[1] for sl in slots]
 
+        # host result arrays per in-flight slot, reused across batches
+        e2e_out = [(np.empty(nq * k, np.uint32), np.empty(nq * k, np.float32),
+                    np.empty(nq, np.uint32)) for _ in e2e_ws]
+
         def e2e_run(n):
             nw = len(e2e_ws)
             for i in range(n):
                 w = e2e_ws[i % nw]
                 if i >= nw:
-                    w.griffin_query_batch_collect()
+                    w.griffin_query_batch_collect(e2e_out[i % nw])
                 w.griffin_query_batch_submit(ql.offsets, ql.terms, k, e2e_st[i % nw])
             for i in range(max(0, n - nw), n):
-                e2e_ws[i % nw].griffin_query_batch_collect()
+                e2e_ws[i % nw].griffin_query_batch_collect(e2e_out[i % nw])
 
         e2e_run(args.warmup)
         if world > 1:

@@ -172,11 +172,22 @@ def _submit(ih, wh, offsets, terms, k, stream):
     return (len(off) - 1, k)
 
 
-def _collect(ih, wh, pend):
+def _collect(ih, wh, pend, out=None):
+    """out: optional (docids u32 >= nq*k, scores f32 >= nq*k, counts u32 >= nq)
+    arrays to fill (a serving loop reuses them instead of faulting in fresh
+    pages every batch)."""
     nq, k = pend
-    d = np.zeros(max(nq * k, 1), np.uint32)
-    s = np.zeros(max(nq * k, 1), np.float32)
-    c = np.zeros(max(nq, 1), np.uint32)
+    if out is None:
+        d = np.zeros(max(nq * k, 1), np.uint32)
+        s = np.zeros(max(nq * k, 1), np.float32)
+        c = np.zeros(max(nq, 1), np.uint32)
+    else:
+        d, s, c = out
+        if (d.dtype != np.uint32 or s.dtype != np.float32 or c.dtype != np.uint32
+                or d.size < nq * k or s.size < nq * k or c.size < nq
+                or not (d.flags.c_contiguous and s.flags.c_contiguous and c.flags.c_contiguous)):
+            raise ValueError("out arrays: contiguous u32[nq*k], f32[nq*k], u32[nq] required")
+        d, s, c = d.reshape(-1), s.reshape(-1), c.reshape(-1)
     _check(load_library().griffin_query_batch_collect(ih, wh, _ptr(d), _ptr(s), _ptr(c)))
     return d[:nq * k].reshape(nq, k), s[:nq * k].reshape(nq, k), c[:nq]
 
@@ -284,8 +295,8 @@ class GriffinIndex:
     def griffin_query_batch_submit(self, offsets, terms, k: int, stream=None):
         self._pend = _submit(self.h, None, offsets, terms, k, stream)
 
-    def griffin_query_batch_collect(self):
-        out = _collect(self.h, None, getattr(self, "_pend", (0, 1)))
+    def griffin_query_batch_collect(self, out=None):
+        out = _collect(self.h, None, getattr(self, "_pend", (0, 1)), out)
         self._pend = (0, 1)
         return out
 
@@ -409,8 +420,8 @@ class GriffinWorkspace:
     def griffin_query_batch_submit(self, offsets, terms, k: int, stream=None):
         self._pend = _submit(self.index.h, self.h, offsets, terms, k, stream)
 
-    def griffin_query_batch_collect(self):
-        out = _collect(self.index.h, self.h, getattr(self, "_pend", (0, 1)))
+    def griffin_query_batch_collect(self, out=None):
+        out = _collect(self.index.h, self.h, getattr(self, "_pend", (0, 1)), out)
         self._pend = (0, 1)
         return out
 

@@ -604,7 +604,11 @@ def test_submit_collect_pipelined_workspaces(tiny):
     gx.griffin_query_batch_submit(sub.offsets, sub.terms, k)
     with pytest.raises(g.GriffinError):
         gx.griffin_query_batch(sub.offsets, sub.terms, k)
-    assert_topk_equal(*gx.griffin_query_batch_collect(), od, os_, oc)
+    nqs = sub.num_queries
+    out = (np.full(nqs * k, 7, np.uint32), np.zeros(nqs * k, np.float32), np.zeros(nqs, np.uint32))
+    gd, gs, gc = gx.griffin_query_batch_collect(out)
+    assert gd.base is out[0] or gd is out[0] or np.shares_memory(gd, out[0])
+    assert_topk_equal(gd, gs, gc, od, os_, oc)
     assert_topk_equal(*gx.griffin_query_batch(sub.offsets, sub.terms, k), od, os_, oc)
     for w in wss:
         w.close()
