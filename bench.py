@@ -490,8 +490,8 @@ def main():
     ap.add_argument("--latency-queries", type=int, default=1000)
     ap.add_argument("--streams", type=int, default=None,
                     help="batches in flight on separate streams/workspaces (N=1 only); default "
-                         "3 for the 1K-query configs, 1 for the 10K-query top-1000 batches "
-                         "(one already fills the GPU; three workspaces of it exceed HBM)")
+                         "3 for the 1K-query configs, 2 for the 10K-query top-1000 batches "
+                         "(three workspaces of those exceed HBM)")
     ap.add_argument("--shard-mode", default="docid", choices=["docid", "replicate"],
                     help="N>1: docID-range shards + exchange, or a replicated index per rank")
     ap.add_argument("--exchange", default="allgather", choices=["allgather", "sliced"],
@@ -500,7 +500,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.streams is None:
-        args.streams = 1 if args.config in ("c4", "c5") else 3
+        args.streams = 2 if args.config in ("c4", "c5") else 3
     if args.impl == "reference":
         run_reference(args)
     else:
