@@ -202,6 +202,15 @@ griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *
 griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace *ws,
                                            uint32_t *out_docids, float *out_scores,
                                            uint32_t *out_counts);
+/* Zero-copy read of the last collected batch: collect with all three outputs
+ * NULL waits and checks status without copying; then this returns read-only
+ * host pointers to the [nq*k] docIDs, [nq*k] scores and [nq] counts in the
+ * workspace's pinned staging, valid until the next submit on that workspace
+ * (for ws = NULL also until the next griffin_query / griffin_query_batch).
+ * GRIFFIN_ERR_INVALID_ARG while a batch is still uncollected. */
+griffin_status griffin_query_batch_results(griffin_index *ix, griffin_workspace *ws,
+                                           const uint32_t **docids, const float **scores,
+                                           const uint32_t **counts);
 
 /* Shard merge: given G per-shard sorted key runs
  * d_keys[g][nq*k] and counts d_counts[g][nq] (laid out contiguously, g-major, as

@@ -93,6 +93,8 @@ _SIGS = {
     "griffin_workspace_sync_status": [_vp, _vp],
     "griffin_query_batch_submit": [_vp, _vp, _u32, _vp, _vp, _u32, _vp],
     "griffin_query_batch_collect": [_vp, _vp, _vp, _vp, _vp],
+    "griffin_query_batch_results": [_vp, _vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp),
+                                    ctypes.POINTER(_vp)],
     "griffin_merge_topk_device": [_vp, _u32, _u32, _u32, _vp, _vp, _vp, _vp, _vp],
     "griffin_keys_to_results_device": [_vp, _u32, _u32, _vp, _vp, _vp, _vp, _vp],
     "griffin_set_mode": [_vp, ctypes.c_int],
@@ -175,8 +177,26 @@ def _submit(ih, wh, offsets, terms, k, stream):
 def _collect(ih, wh, pend, out=None):
     """out: optional (docids u32 >= nq*k, scores f32 >= nq*k, counts u32 >= nq)
     arrays to fill (a serving loop reuses them instead of faulting in fresh
-    pages every batch)."""
+    pages every batch), or "view": no copy — read-only numpy views of the
+    workspace's pinned staging (griffin_query_batch_results), valid until the
+    next submit on that workspace."""
     nq, k = pend
+    if isinstance(out, str) and out == "view":
+        lib = load_library()
+        _check(lib.griffin_query_batch_collect(ih, wh, None, None, None))
+        pd, ps, pc = _vp(), _vp(), _vp()
+        _check(lib.griffin_query_batch_results(ih, wh, ctypes.byref(pd), ctypes.byref(ps),
+                                               ctypes.byref(pc)))
+
+        def view(p, n, ct, dt):
+            if n == 0:
+                return np.zeros(0, dt)
+            a = np.ctypeslib.as_array(ctypes.cast(p, ctypes.POINTER(ct)), shape=(n,)).view(dt)
+            a.flags.writeable = False
+            return a
+        return (view(pd, nq * k, ctypes.c_uint32, np.uint32).reshape(nq, k),
+                view(ps, nq * k, ctypes.c_float, np.float32).reshape(nq, k),
+                view(pc, nq, ctypes.c_uint32, np.uint32))
     if out is None:
         d = np.zeros(max(nq * k, 1), np.uint32)
         s = np.zeros(max(nq * k, 1), np.float32)

@@ -634,6 +634,20 @@ griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *
   return GRIFFIN_OK;
 }
 
+griffin_status griffin_query_batch_results(griffin_index *ix, griffin_workspace *ws,
+                                           const uint32_t **docids, const float **scores,
+                                           const uint32_t **counts) {
+  if (!ix || !docids || !scores || !counts) return invalid("null argument");
+  Workspace &w = ws ? *reinterpret_cast<Workspace *>(ws) : ix->ws;
+  if (w.pending || !w.h_pinned) return invalid("no collected batch on this workspace");
+  const size_t nk = (size_t)w.pend_nq * w.pend_k;
+  const uint8_t *ho = static_cast<const uint8_t *>(w.h_pinned) + w.pend_out;
+  *docids = reinterpret_cast<const uint32_t *>(ho);
+  *scores = reinterpret_cast<const float *>(ho + nk * 4);
+  *counts = reinterpret_cast<const uint32_t *>(ho + nk * 8);
+  return GRIFFIN_OK;
+}
+
 griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace *ws,
                                            uint32_t *out_docids, float *out_scores,
                                            uint32_t *out_counts) {
@@ -641,7 +655,9 @@ griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace 
   Workspace &w = ws ? *reinterpret_cast<Workspace *>(ws) : ix->ws;
   if (!w.pending) return invalid("no submitted batch on this workspace");
   const size_t nk = (size_t)w.pend_nq * w.pend_k;
-  if (w.pend_nq && (!out_docids || !out_scores || !out_counts)) return invalid("null argument");
+  const bool copy = out_docids || out_scores || out_counts;
+  if (w.pend_nq && copy && (!out_docids || !out_scores || !out_counts))
+    return invalid("null argument");
   {
     DeviceGuard guard(ix->device);
     w.pending = false;
@@ -654,7 +670,7 @@ griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace 
     griffin_status s = read_status(ix, w, w.pend_stream);   // clears the device flag
     if (s) return s;
   }
-  if (w.pend_nq) {
+  if (w.pend_nq && copy) {
     std::memcpy(out_docids, ho, nk * 4);
     std::memcpy(out_scores, ho + nk * 4, nk * 4);
     std::memcpy(out_counts, ho + nk * 8, (size_t)w.pend_nq * 4);

@@ -610,6 +610,12 @@ def test_submit_collect_pipelined_workspaces(tiny):
     assert gd.base is out[0] or gd is out[0] or np.shares_memory(gd, out[0])
     assert_topk_equal(gd, gs, gc, od, os_, oc)
     assert_topk_equal(*gx.griffin_query_batch(sub.offsets, sub.terms, k), od, os_, oc)
+    # zero-copy views of a workspace's pinned staging
+    w = wss[1]
+    w.griffin_query_batch_submit(sub.offsets, sub.terms, k)
+    vd, vs, vc = w.griffin_query_batch_collect("view")
+    assert not vd.flags.writeable
+    assert_topk_equal(vd, vs, vc, od, os_, oc)
     for w in wss:
         w.close()
 
