@@ -2,17 +2,30 @@
 """Benchmark of the B200 Griffin-GPU conjunctive query path.
 
 One "step" = one pass of the whole hot path (plus a8 for
-N > 1) over one batch: the BASELINE.json configs[1] workload — a 10M-doc
-synthetic Zipfian index (EF blocks of 128) and its 1000-query 2-5 term log,
-BM25 top-10 — with the query log already resident in HBM.  Prints ONE JSON line.
+N > 1) over one batch of queries with the query log resident in HBM.  Default
+workload: BASELINE.json configs[4] (C5) — the 50M-doc ClueWeb-shaped synthetic
+index (EF blocks of 128, ~1.9 B postings) and a batch of 10K concurrent 2-5
+term queries, BM25 top-1000 — the largest single-GPU configuration.  The timed
+loop rotates through the config's distinct query batches (3 by default).
+Prints ONE JSON line.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c5] [--impl reference]
 
+Measurements on the same line:
+  value       queries/s, batches pipelined over --streams workspaces (device API)
+  roofline    the dominant kernel's §8(d) algorithmic bytes per launch / its
+              ISOLATED launch duration (one batch in flight, profiling pass,
+              CUDA events on the launching stream), vs the measured HBM peak;
+              traffic = ncu DRAM bytes per launch from profiles/
+  sync_qps    §8(d)'s definition: batch / median wall time of one synchronous
+              griffin_query_batch call (host buffers, H2D + D2H inside)
+  e2e         the same metric through the host-buffer C ABI, pipelined
+  parity      the last timed batch vs the CPU oracle on the cpu_baseline sample
 N > 1 is launched by torchrun (one process per GPU): each rank holds one
-docID-range shard of the same corpus, runs the batch, and the per-shard top-k
-keys are all-gathered over NCCL and merged by the library's k-way merge kernel.
-The reference arm (--impl reference) times the CPU oracle (the test oracle,
-as it stands) on the same workload; there is no installable reference code.
+docID-range shard; per-shard top-k keys are all-gathered over NCCL and merged by
+the library's k-way merge kernel.  The reference arm (--impl reference) times
+the CPU oracle (the test oracle, as it stands) on a bounded sample of the same
+workload; there is no installable reference code (PAPER.md only).
 """
 from __future__ import annotations
 
@@ -31,10 +44,10 @@ import numpy as np  # noqa: E402
 
 WORKLOAD_DESC = {
     "c1": "C1: single 2-term AND query, 100K-doc synthetic Zipf index (lists ~10K and ~1K), EF block 128, BM25 top-10",
-    "c2": "C2: 10M-doc synthetic Zipf index (alpha 0.8, df 1K..5M, 42K terms, 0.19B postings), replayed 1000-query 2-5 term log, EF block 128, BM25 top-10",
+    "c2": "C2: 10M-doc synthetic Zipf index (alpha 0.8, df 1K..5M, 42K terms, 0.19B postings), 1000-query 2-5 term batches, EF block 128, BM25 top-10",
     "c3": "C3: GOV2-shaped 25M-doc synthetic Zipf index (df up to 10M), 1000-query log, BM25 top-10",
-    "c4": "C4: ClueWeb-shaped 50M-doc synthetic Zipf index (df up to 30M), 10K-query log, BM25 top-10",
-    "c5": "C5: 50M-doc index, 10K concurrent queries, BM25 top-1000",
+    "c4": "C4: ClueWeb-shaped 50M-doc synthetic Zipf index (alpha 0.8, df 1K..30M, 395K terms, 1.9B postings), 10K-query batches, EF block 128, BM25 top-10",
+    "c5": "C5: ClueWeb-shaped 50M-doc synthetic Zipf index (alpha 0.8, df 1K..30M, 395K terms, 1.9B postings), 10K concurrent 2-5 term queries per batch, EF block 128, BM25 top-1000",
 }
 
 
@@ -43,14 +56,13 @@ def _peaks():
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
-        return float(d["hbm_gbs"]), "measured"
-    return 6650.0, "fallback"
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, STREAM copy)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
 
 
 class ClockSampler:
     """SM clock + throttle reasons sampled during the timed region: NVML in a
-    background thread every 2 ms (the timed region can be tens of ms), with
-    nvidia-smi as a fallback."""
+    background thread every 2 ms, with nvidia-smi as a fallback."""
 
     def __init__(self, gpu_index: int):
         self.gpu = gpu_index
@@ -131,58 +143,103 @@ def _cpu_info():
     return os.cpu_count() or 1, model
 
 
-def oracle_baseline(corpus, ql, k, block, budget_s=12.0, threads=None):
-    """Time the oracle (as it stands) on a bounded prefix of the query log."""
-    import oracle
-    cores, model = _cpu_info()
-    threads = threads or cores
-    t0 = time.time()
-    ox = oracle.OracleIndex(corpus, block_size=block)
-    build_s = time.time() - t0
-    m = min(ql.num_queries, max(threads, 16))
-    while True:
-        sub = ql.slice(0, m)
+def load_workload(name):
+    """(corpus, [batch query logs], cfg); large corpora come from the
+    on-disk synth cache (generated once, memory-mapped by every rank)."""
+    from synth import batch_of, make_workload
+    corpus, ql, cfg = make_workload(name)
+    batches = [batch_of(ql, cfg, i) for i in range(cfg.get("batches", 1))]
+    return corpus, batches, cfg
+
+
+def config_dict(args, corpus, cfg, nq, extra=None):
+    """The `config` object, identical on both arms (ours and --impl reference)."""
+    d = {"workload": WORKLOAD_DESC[args.config], "num_docs": corpus.num_docs,
+         "num_terms": corpus.num_terms, "num_postings": corpus.num_postings,
+         "queries_per_step": nq, "k": cfg["k"], "block_size": cfg["block"],
+         "batches_rotated": cfg.get("batches", 1),
+         "l2": "inputs larger than L2 (index > 126 MB L2, rotating query batches)",
+         "parallelism": (f"docid-range shards x{args.gpus}" if args.gpus > 1 else "1 shard")}
+    if extra:
+        d.update(extra)
+    return d
+
+
+class OracleSample:
+    """The CPU oracle (tests' checker, as it stands) over the lists of a bounded
+    sample of one batch: timed as the cpu_baseline / reference arm, and its
+    answers are the parity reference for the same queries on the GPU."""
+
+    def __init__(self, corpus, batch, k, block, budget_s, threads=None):
+        import oracle
+        from synth import sub_corpus
+        self.cores, self.model = _cpu_info()
+        self.threads = threads or self.cores
+        self.k = k
+        # grow the sample until one pass costs ~budget/3 (bounded CPU work)
+        m = min(batch.num_queries, max(self.threads, 16))
+        while True:
+            sub = batch.slice(0, m)
+            t0 = time.time()
+            ox = oracle.OracleIndex(sub_corpus(corpus, sub.terms), block_size=block)
+            self.build_s = time.time() - t0
+            t0 = time.perf_counter()
+            res = ox.query_batch(sub, k, nthreads=self.threads)
+            dt = time.perf_counter() - t0
+            if dt >= budget_s / 3 or m >= batch.num_queries:
+                break
+            m = min(batch.num_queries, int(m * max(2.0, budget_s / 3 / max(dt, 1e-3))))
+        self.ox, self.sub, self.m, self.res, self.dt = ox, sub, m, res, dt
+
+    def run(self):
         t0 = time.perf_counter()
-        ox.query_batch(sub, k, nthreads=threads)
-        dt = time.perf_counter() - t0
-        if dt >= budget_s / 3 or m >= ql.num_queries:
-            break
-        m = min(ql.num_queries, int(m * max(2.0, budget_s / 3 / max(dt, 1e-3))))
-    return {"value": m / dt, "unit": "queries/s", "cores": threads, "kind": "oracle",
-            "sample": f"first {m} of the {ql.num_queries}-query log, {threads} std::threads, "
-                      f"round-robin; oracle index build {build_s:.1f}s not timed",
-            "cpu_model": model, "seconds": dt}, ox, m
+        self.res = self.ox.query_batch(self.sub, self.k, nthreads=self.threads)
+        return time.perf_counter() - t0
+
+    def baseline(self, value, nq_batch):
+        return {"value": value, "unit": "queries/s", "cores": self.threads, "kind": "oracle",
+                "sample": f"first {self.m} of a {nq_batch}-query batch, {self.threads} std::threads "
+                          f"round-robin; oracle indexes only the sample's lists (same N, dl, df) "
+                          f"in {self.build_s:.1f}s, not timed",
+                "cpu_model": self.model}
 
 
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    from synth import make_workload
-    corpus, ql, cfg = make_workload(args.config)
+    corpus, batches, cfg = load_workload(args.config)
     k = cfg["k"]
-    base, ox, m = oracle_baseline(corpus, ql, k, cfg["block"], budget_s=6.0)
-    sub = ql.slice(0, m)
-    threads = base["cores"]
+    last = batches[(args.steps - 1) % len(batches)]
+    osm = OracleSample(corpus, last, k, cfg["block"], budget_s=args.cpu_budget)
     for _ in range(args.warmup):
-        ox.query_batch(sub, k, nthreads=threads)
-    times = []
-    for _ in range(args.steps):
-        t0 = time.perf_counter()
-        ox.query_batch(sub, k, nthreads=threads)
-        times.append(time.perf_counter() - t0)
+        osm.run()
+    times = [osm.run() for _ in range(args.steps)]
     ms = 1e3 * statistics.mean(times)
-    qps = m / (ms / 1e3)
-    base["value"] = qps
+    qps = osm.m / (ms / 1e3)
     line = {"impl": "reference", "metric": "queries/sec", "value": qps, "unit": "queries/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/f32",
-            "data": "synthetic",
-            "config": {"workload": WORKLOAD_DESC[args.config], "num_docs": corpus.num_docs,
-                       "queries_per_step": m, "k": k, "block_size": cfg["block"]},
-            "cpu_baseline": base,
-            "e2e": {"value": qps, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "u32/f32", "data": "synthetic",
+            "config": config_dict(args, corpus, cfg, last.num_queries),
+            "cpu_baseline": osm.baseline(qps, last.num_queries),
+            "e2e": {"value": qps, "unit": "queries/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    line["cpu_baseline"]["queries_per_step_timed"] = osm.m
     print(json.dumps(line), flush=True)
+
+
+def _keys_to_rows(keys, counts, nq, k):
+    """(score desc, docID asc) rows from the library's u64 keys (host, for the
+    parity check): key = f32 score bits << 32 | (0xFFFFFFFF - docID)."""
+    kk = keys.view(np.uint64).reshape(nq, k)
+    d = (np.uint64(0xFFFFFFFF) - (kk & np.uint64(0xFFFFFFFF))).astype(np.uint32)
+    s = (kk >> np.uint64(32)).astype(np.uint32).view(np.float32)
+    c = counts.view(np.uint32)[:nq]
+    valid = np.arange(k)[None, :] < c[:, None]
+    d = np.where(valid, d, np.uint32(0xFFFFFFFF))
+    s = np.where(valid, s, np.float32(-np.inf))
+    return d, s, c
 
 
 def run_gpu(args):
@@ -190,9 +247,7 @@ def run_gpu(args):
     import torch.distributed as dist
 
     import paper_conf_ppopp_0044ws18_b200 as g
-    from paper_conf_ppopp_0044ws18_b200.sharded import (ShardedSearcher, exchange_sliced,
-                                                        gather_runs)
-    from synth import make_workload
+    from paper_conf_ppopp_0044ws18_b200.sharded import gather_runs
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -203,36 +258,33 @@ def run_gpu(args):
     else:
         torch.cuda.set_device(0)
     dev = torch.cuda.current_device()
-    corpus, ql, cfg = make_workload(args.config)
-    k, B = cfg["k"], cfg["block"]
-    nq = ql.num_queries
-    # docid: rank r holds docID-range shard r and the per-shard top-k are exchanged
-    # (all-gather, or the query-sliced all-to-all); replicate: every rank holds the
-    # whole index and runs its own batch, no exchange
-    replicate = world > 1 and args.shard_mode == "replicate"
-    sharded = world > 1 and not replicate
     t0 = time.time()
-    if replicate:
-        ix = g.GriffinIndex(corpus, block_size=B, device=dev)
-    else:
-        ix = g.GriffinIndex(corpus, block_size=B, device=dev, shard_index=rank, num_shards=world)
+    corpus, batches, cfg = load_workload(args.config)
+    gen_s = time.time() - t0
+    k, B = cfg["k"], cfg["block"]
+    NB = len(batches)
+    nq = batches[0].num_queries
+    sharded = world > 1
+    t0 = time.time()
+    ix = g.GriffinIndex(corpus, block_size=B, device=dev, shard_index=rank if sharded else 0,
+                        num_shards=world)
     build_s = time.time() - t0
     st = ix.griffin_index_stats()
-    ix.griffin_reserve(ql.offsets, ql.terms, k)
-    max_terms = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
+    ix.griffin_set_reuse({"auto": 2, "on": 1, "off": 0}[args.reuse])
     stream = torch.cuda.current_stream()
-    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
-    d_terms = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
-    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
-    cnts = torch.zeros(nq, dtype=torch.int32, device="cuda")
-    # batches in flight: slot 0 = the index's own workspace on the current
-    # stream, slots 1.. = extra workspaces on their own streams (serving engine
-    # overlapping consecutive batches); each slot has its own outputs
+    dq = []   # per batch: (d_off, d_terms, max_terms)
+    for b in batches:
+        ix.griffin_reserve(b.offsets, b.terms, k)
+        mt = int(max(len(set(b.query(q).tolist())) for q in range(b.num_queries)))
+        dq.append((torch.from_numpy(b.offsets.astype(np.int32)).cuda(),
+                   torch.from_numpy(b.terms.astype(np.int32)).cuda(), mt))
     nstreams = max(1, args.streams) if not sharded else 1
-    slots = [(None, stream, keys, cnts)]
+    slots = [(None, stream, torch.zeros(nq * k, dtype=torch.int64, device="cuda"),
+              torch.zeros(nq, dtype=torch.int32, device="cuda"))]
     for _ in range(nstreams - 1):
         w = ix.griffin_workspace_create()
-        w.griffin_workspace_reserve(ql.offsets, ql.terms, k)
+        for b in batches:
+            w.griffin_workspace_reserve(b.offsets, b.terms, k)
         slots.append((w, torch.cuda.Stream(), torch.zeros(nq * k, dtype=torch.int64, device="cuda"),
                       torch.zeros(nq, dtype=torch.int32, device="cuda")))
     if sharded:
@@ -242,225 +294,244 @@ def run_gpu(args):
 
     def step_on(i):
         w, st_, kk_, cc_ = slots[i % len(slots)]
+        d_off, d_t, mt = dq[i % NB]
         if w is None:
-            ix.griffin_query_batch_device(d_off, d_terms, max_terms, k, kk_, cc_, st_)
+            ix.griffin_query_batch_device(d_off, d_t, mt, k, kk_, cc_, st_)
         else:
-            w.griffin_query_batch_device_ws(d_off, d_terms, max_terms, k, kk_, cc_, st_)
-
-    def step():
-        ix.griffin_query_batch_device(d_off, d_terms, max_terms, k, keys, cnts, stream)
-        if sharded and args.exchange == "allgather":
-            ak, ac = gather_runs(keys, cnts)
-            ix.griffin_merge_topk_device(world, nq, k, ak, ac, out_keys, out_cnts, stream)
-        elif sharded:
-            ak, ac, (lo, hi) = exchange_sliced(keys, cnts, k)
-            if hi > lo:
-                ix.griffin_merge_topk_device(world, hi - lo, k, ak, ac, out_keys, out_cnts, stream)
+            w.griffin_query_batch_device_ws(d_off, d_t, mt, k, kk_, cc_, st_)
+        if sharded:   # a8: all-gather of per-shard top-k + k-way merge (NCCL)
+            ak, ac = gather_runs(kk_, cc_)
+            ix.griffin_merge_topk_device(world, nq, k, ak, ac, out_keys, out_cnts, st_)
 
     for i in range(args.warmup):
         step_on(i)
     torch.cuda.synchronize()
     ix.griffin_sync_status()
+    for w, _, _, _ in slots[1:]:
+        w.griffin_workspace_sync_status()
     ix.griffin_reset_profile()
-    ix.griffin_set_profiling(True)
+
+    # ---- timed region: batches pipelined over the slots (rotating batches) ----
     clocks = ClockSampler(dev)
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-          for _ in range(args.steps)]
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     clocks.start()
-    if len(slots) == 1:
-        for i in range(args.steps):
-            flush.fill_(i)                   # L2 flush between timed steps (outside events)
-            ev[i][0].record(stream)
-            step()
-            ev[i][1].record(stream)
-    else:
-        # overlapped batches: one event pair around the whole region (start on the
-        # first stream, end after every stream's last batch); no per-step flush —
-        # the inputs (index >> L2) are larger than L2
-        for _, st_, _, _ in slots[1:]:
-            st_.wait_stream(stream)
-        ev[0][0].record(stream)
-        for i in range(args.steps):
-            step_on(i)
-        for _, st_, _, _ in slots[1:]:
-            stream.wait_stream(st_)
-        ev[0][1].record(stream)
+    for _, st_, _, _ in slots[1:]:
+        st_.wait_stream(stream)
+    ev0.record(stream)
+    for i in range(args.steps):
+        step_on(i)
+    for _, st_, _, _ in slots[1:]:
+        stream.wait_stream(st_)
+    ev1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clk = clocks.stop()
-    ix.griffin_set_profiling(False)
-    prof = ix.griffin_get_profile()
+    total_ms = ev0.elapsed_time(ev1)
+    launches = int(ix.griffin_get_profile()["launches_total"])
     ix.griffin_sync_status()
-    if len(slots) == 1:
-        step_ms = [a.elapsed_time(b) for a, b in ev]
-        total_ms = sum(step_ms)
-    else:
-        total_ms = ev[0][0].elapsed_time(ev[0][1])
+    for w, _, _, _ in slots[1:]:
+        w.griffin_workspace_sync_status()
     if world > 1:
         t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     ms_per_step = total_ms / args.steps
-    # replicate: every rank answered its own full batch (weak scaling)
-    qps = (world if replicate else 1) * nq * args.steps / (total_ms / 1e3)
-    peak, peak_kind = _peaks()
-    ms_x = prof["ms_intersect"]
-    achieved = prof["alg_bytes"] / (ms_x / 1e3) / 1e9 if ms_x > 0 else 0.0
-    ms_d = prof["ms_decode"]
-    achieved_d = prof["dec_alg_bytes"] / (ms_d / 1e3) / 1e9 if ms_d > 0 else 0.0
-    kernels = {
-        "intersect_kernel": {
-            "what": "fused EF decode + merge-path/gallop intersection + BM25 (all SvS rounds)",
-            "ms_per_step": ms_x / args.steps, "launches": prof["launches_intersect"],
-            "alg_bytes_per_launch": prof["alg_bytes"] / max(1, prof["launches_intersect"]),
-            "achieved_gbs": achieved, "share_of_step": ms_x / total_ms if total_ms else None,
-            "decoded_postings_per_step": prof["decoded_postings"] / args.steps},
-        "decode_once_kernel": {
-            "what": "batch decode-once: Para-EF decode of hot lists into the HBM arena",
-            "ms_per_step": ms_d / args.steps, "launches": prof["launches_decode"],
-            "alg_bytes_per_launch": prof["dec_alg_bytes"] / max(1, prof["launches_decode"]),
-            "achieved_gbs": achieved_d, "share_of_step": ms_d / total_ms if total_ms else None,
-            "decoded_postings_per_step": prof["dec_postings"] / args.steps},
-    }
-    dom = "intersect_kernel" if ms_x >= ms_d else "decode_once_kernel"
-    kd = kernels[dom]
-    roof = {"bound": "hbm", "kernel": dom, "achieved": kd["achieved_gbs"], "peak": peak,
-            "unit": "GB/s", "frac": kd["achieved_gbs"] / peak if peak else None, "traffic": None,
-            "peak_kind": peak_kind, "alg_bytes_per_launch": kd["alg_bytes_per_launch"],
-            "ms_per_launch": kd["ms_per_step"] * args.steps / max(1, kd["launches"]),
-            "share_of_step": kd["share_of_step"]}
-    # per-GPU figures of this rank; the job aggregate for N ranks is N x (max-time) based
-    decoded_ps = ((prof["decoded_postings"] + prof["dec_postings"]) / (total_ms / 1e3)
-                  if total_ms > 0 else 0.0)
-
-    # ---- e2e: the public host-buffer C-ABI call, H2D of the step's queries and
-    # D2H of its results inside every timed step (wall clock, max over ranks)
-    e2e_times = []
+    qps = nq * args.steps / (total_ms / 1e3)
+    # results of the last timed step (its slot's outputs are untouched since)
+    last_i = args.steps - 1
+    _, _, lk, lc = slots[last_i % len(slots)]
     if sharded:
-        searcher = ShardedSearcher.from_index(ix)
-    if world > 1:
-        h_off = torch.from_numpy(ql.offsets.astype(np.int32)).pin_memory()
-        h_terms = torch.from_numpy(ql.terms.astype(np.int32)).pin_memory()
+        lk, lc = out_keys, out_cnts
+    last_keys, last_cnts = lk.cpu().numpy(), lc.cpu().numpy()
+    last_batch = batches[last_i % NB]
+
+    # ---- isolated pass: one batch at a time, L2 flushed between, per-stage
+    # CUDA events on the launching stream -> per-kernel durations ----
+    n_iso = max(NB, min(args.steps, 2 * NB))
+    ix.griffin_reset_profile()
+    ix.griffin_set_profiling(True)
+    iso = []
+    for i in range(n_iso):
+        flush.fill_(i)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        d_off, d_t, mt = dq[i % NB]
+        ix.griffin_query_batch_device(d_off, d_t, mt, k, slots[0][2], slots[0][3], stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        iso.append(e0.elapsed_time(e1))
+    ix.griffin_set_profiling(False)
+    prof = ix.griffin_get_profile()
+    ix.griffin_sync_status()
+    iso_ms = sum(iso)
+    peak, peak_kind = _peaks()
+
+    def kern(ms, alg, c8d, launches_, post, what):
+        per = max(1, launches_)
+        return {"what": what, "ms_per_step": ms / n_iso, "launches_per_step": launches_ / n_iso,
+                "ms_per_launch": ms / per, "share_of_step": ms / iso_ms if iso_ms else None,
+                "alg_bytes_per_launch": c8d / per, "all_bytes_per_launch": alg / per,
+                "achieved_gbs": (c8d / per) / (ms / per / 1e3) / 1e9 if ms > 0 else 0.0,
+                "achieved_all_bytes_gbs": (alg / per) / (ms / per / 1e3) / 1e9 if ms > 0 else 0.0,
+                "decoded_postings_per_step": post / n_iso}
+
+    kernels = {
+        "intersect_kernel": kern(prof["ms_intersect"], prof["alg_bytes"], prof["c8d_bytes"],
+                                 prof["launches_intersect"], prof["decoded_postings"],
+                                 "fused EF decode + merge-path/gallop intersection + BM25 (all SvS rounds)"),
+        "decode_once_kernel": kern(prof["ms_decode"], prof["dec_alg_bytes"],
+                                   prof["dec_c8d_bytes"], prof["launches_decode"],
+                                   prof["dec_postings"],
+                                   "batch decode-once: Para-EF decode of hot lists into the HBM arena"),
+    }
+    stage_ms = {kk: prof[kk] / n_iso for kk in
+                ("ms_plan", "ms_decode", "ms_intersect", "ms_compact", "ms_topk", "ms_merge")}
+    dom = max(kernels, key=lambda n: kernels[n]["ms_per_step"])
+    kd = kernels[dom]
+    traffic = _ncu_traffic(args.config, dom)
+    roof = {"bound": "hbm", "kernel": dom, "achieved": kd["achieved_gbs"], "peak": peak,
+            "unit": "GB/s", "frac": kd["achieved_gbs"] / peak, "traffic": traffic,
+            "peak_kind": peak_kind,
+            "numerator": ("SURVEY §8(d) algorithmic bytes per launch (compressed payload + 8 B skip/meta "
+                          "of every block the method reads, decoded-arena postings charged at their "
+                          "compressed size, 8 B per intermediate entry, tf sector + norm per survivor)"),
+            "alg_bytes_per_launch": kd["alg_bytes_per_launch"],
+            "achieved_all_bytes": kd["achieved_all_bytes_gbs"],
+            "frac_all_bytes": kd["achieved_all_bytes_gbs"] / peak,
+            "all_bytes_per_launch": kd["all_bytes_per_launch"],
+            "ms_per_launch": kd["ms_per_launch"], "share_of_step": kd["share_of_step"],
+            "timing": (f"isolated: {n_iso} batches one at a time, 256 MB L2 flush between, "
+                       "per-stage CUDA events on the launching stream")}
+    decoded_ps = (prof["decoded_postings"] + prof["dec_postings"]) / (iso_ms / 1e3) if iso_ms else 0.0
+
+    # ---- §8(d) QPS: median wall time of one synchronous griffin_query_batch ----
+    sync_ms = []
     if not sharded:
-        # griffin_query_batch split into submit/collect over the slots'
-        # workspaces: the same host-buffer call with len(slots) batches in
-        # flight (H2D of the queries, the path, D2H of the results per batch)
-        # (slot 0 = the index's own workspace; no extra device memory)
+        for i in range(2 + max(5, NB)):
+            b = batches[i % NB]
+            t0 = time.perf_counter()
+            ix.griffin_query_batch(b.offsets, b.terms, k)
+            if i >= 2:
+                sync_ms.append((time.perf_counter() - t0) * 1e3)
+
+    # ---- e2e: host-buffer C ABI, pipelined submit/collect over the slots ----
+    e2e_s = None
+    h2d = (nq + 1) * 4 + int(np.mean([len(b.terms) for b in batches])) * 4
+    d2h = nq * k * 8 + nq * 4
+    if not sharded:
         e2e_ws = [ix] + [sl[0] for sl in slots[1:]]
         e2e_st = [sl[1] for sl in slots]
-
-        # results read in place from each slot's pinned staging (zero-copy views,
-        # griffin_query_batch_results), valid until that slot's next submit
-        e2e_out = ["view"] * len(e2e_ws)
 
         def e2e_run(n):
             nw = len(e2e_ws)
             for i in range(n):
                 w = e2e_ws[i % nw]
                 if i >= nw:
-                    w.griffin_query_batch_collect(e2e_out[i % nw])
-                w.griffin_query_batch_submit(ql.offsets, ql.terms, k, e2e_st[i % nw])
+                    w.griffin_query_batch_collect("view")
+                b = batches[i % NB]
+                w.griffin_query_batch_submit(b.offsets, b.terms, k, e2e_st[i % nw])
             for i in range(max(0, n - nw), n):
-                e2e_ws[i % nw].griffin_query_batch_collect(e2e_out[i % nw])
+                e2e_ws[i % nw].griffin_query_batch_collect("view")
 
         e2e_run(args.warmup)
-        if world > 1:
-            dist.barrier()
         t0 = time.perf_counter()
         e2e_run(args.steps)
-        e2e_times.append(time.perf_counter() - t0)
-    for i in range(args.warmup + args.steps if sharded else 0):
-        if world > 1:
+        e2e_s = time.perf_counter() - t0
+    else:
+        from paper_conf_ppopp_0044ws18_b200.sharded import ShardedSearcher
+        searcher = ShardedSearcher.from_index(ix)
+        times = []
+        for i in range(args.warmup + args.steps):
+            b = batches[i % NB]
+            h_off = torch.from_numpy(b.offsets.astype(np.int32)).pin_memory()
+            h_t = torch.from_numpy(b.terms.astype(np.int32)).pin_memory()
             dist.barrier()
-        t0 = time.perf_counter()
-        e_off = h_off.to("cuda", non_blocking=True)
-        e_terms = h_terms.to("cuda", non_blocking=True)
-        if args.exchange == "allgather":
-            dd, ss, cc = searcher.search(e_off, e_terms, max_terms, k, stream)
-        else:
-            _, _, dd, ss, cc = searcher.search_sliced(e_off, e_terms, max_terms, k, stream)
-        dd, ss, cc = dd.cpu(), ss.cpu(), cc.cpu()
-        dt = time.perf_counter() - t0
-        if i >= args.warmup:
-            e2e_times.append(dt)
-    e2e_s = sum(e2e_times)
+            t0 = time.perf_counter()
+            dd, ss, cc = searcher.search(h_off.to("cuda", non_blocking=True),
+                                         h_t.to("cuda", non_blocking=True), dq[i % NB][2], k, stream)
+            dd, ss, cc = dd.cpu(), ss.cpu(), cc.cpu()
+            if i >= args.warmup:
+                times.append(time.perf_counter() - t0)
+        e2e_s = sum(times)
     if world > 1:
         t = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_s = float(t.item())
-    h2d = (nq + 1) * 4 + len(ql.terms) * 4
-    d2h = nq * k * 8 + nq * 4
-    if sharded and args.exchange == "sliced":   # each rank reads back its own slice
-        d2h = -(-nq // world) * (k * 8 + 4)
 
-    # ---- closed-loop single-query latency (griffin_query, one in flight)
+    # ---- closed-loop single-query latency (griffin_query, one in flight) ----
     lat = []
-    nlat = min(nq, args.latency_queries)
-    for q in range(min(nlat, 64)):          # warm-up: capture the per-term-count graphs
-        ix.griffin_query(ql.query(q), k)
-    for q in range(nlat):
-        t0 = time.perf_counter()
-        ix.griffin_query(ql.query(q), k)
-        lat.append((time.perf_counter() - t0) * 1e3)
-    lat.sort()
+    if not sharded:
+        b0 = batches[0]
+        nlat = min(b0.num_queries, args.latency_queries)
+        for q in range(min(nlat, 64)):          # warm-up: capture the per-term-count graphs
+            ix.griffin_query(b0.query(q), k)
+        for q in range(nlat):
+            t0 = time.perf_counter()
+            ix.griffin_query(b0.query(q), k)
+            lat.append((time.perf_counter() - t0) * 1e3)
+        lat.sort()
 
     def pct(p):
         return lat[min(len(lat) - 1, int(np.ceil(p / 100 * len(lat))) - 1)] if lat else None
 
+    sw = ix.griffin_debug_decode_all(iters=3)
     line = {
         "metric": "queries/sec", "value": qps, "unit": "queries/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
-        "higher_is_better": True, "scaling": "weak" if replicate else "strong",
-        "vs_baseline": None, "dtype": "u32/f32", "data": "synthetic",
-        "config": {"workload": WORKLOAD_DESC[args.config], "num_docs": corpus.num_docs,
-                   "num_terms": corpus.num_terms, "num_postings": corpus.num_postings,
-                   "queries_per_step": nq, "k": k, "block_size": B,
-                   "l2": ("flushed between timed steps (256 MB write)" if len(slots) == 1 else
-                          "inputs larger than L2 (index %.0f MB, L2 126 MB); not flushed" %
-                          ((st["payload_bytes"] + st["skip_bytes"] + st["tf_bytes"]) / 1e6)),
-                   "batches_in_flight": len(slots),
-                   "parallelism": (f"docid-range shards x{world}, {args.exchange} exchange"
-                                   if sharded else f"replicated index x{world}, no exchange"
-                                   if replicate else "1 shard"),
-                   "index_bytes_per_shard": st["payload_bytes"] + st["skip_bytes"] + st["tf_bytes"],
-                   "index_build_s": build_s},
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "u32/f32", "data": "synthetic",
+        "config": config_dict(args, corpus, cfg, nq),
+        "batches_in_flight": len(slots),
+        "index": {"bytes_per_shard": st["payload_bytes"] + st["skip_bytes"] + st["tf_bytes"],
+                  "payload_bytes": st["payload_bytes"], "build_s": build_s,
+                  "corpus_load_s": gen_s, "reuse": args.reuse},
         "decoded_postings_per_s": decoded_ps * world,
-        "reuse": "auto (decode-once of hot lists per batch)",
-        "hbm_gbs": achieved,
-        "latency_ms": {"p50": pct(50), "p99": pct(99), "queries": nlat,
+        "sync_qps": {"value": nq / (statistics.median(sync_ms) / 1e3) if sync_ms else None,
+                     "unit": "queries/s", "median_ms": statistics.median(sync_ms) if sync_ms else None,
+                     "calls": len(sync_ms),
+                     "how": "SURVEY §8(d): batch size / median wall time of one synchronous "
+                            "griffin_query_batch (host buffers, H2D + D2H inside), rotating batches"},
+        "latency_ms": {"p50": pct(50), "p99": pct(99), "queries": len(lat),
                        "mode": "closed-loop griffin_query (host buffers), one in flight"},
         "roofline": roof,
         "kernels": kernels,
-        "stage_ms_note": ("CUDA-event durations per stage summed over all launches; with "
-                          "batches_in_flight > 1 the stages of different batches overlap"),
-        "stage_ms_per_step": {kk: prof[kk] / args.steps for kk in
-                              ("ms_plan", "ms_decode", "ms_intersect", "ms_compact", "ms_topk",
-                               "ms_merge")},
-        "gpu_launches": int(prof["launches_total"]),
-        "e2e": {"value": (world if replicate else 1) * nq * args.steps / e2e_s,
-                "unit": "queries/s", "h2d_bytes_per_step": h2d,
-                "d2h_bytes_per_step": d2h,
+        "stage_ms_per_step_isolated": stage_ms,
+        "isolated_ms_per_step": iso_ms / n_iso,
+        "gpu_launches": launches,
+        "e2e": {"value": nq * args.steps / e2e_s if e2e_s else None, "unit": "queries/s",
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "how": ("griffin_query_batch_submit/collect (host buffers; pinned staging, H2D queries, "
-                        "D2H results), batches_in_flight workspaces" if not sharded else
-                        "ShardedSearcher.search (pinned H2D queries, D2H results)")},
+                        "D2H results read in place), batches_in_flight workspaces, rotating batches"
+                        if not sharded else "ShardedSearcher.search (pinned H2D queries, D2H results)")},
         "clocks": clk,
+        "decode_sweep": {"ms": sw["ms"], "postings": sw["postings"], "bytes": sw["bytes"],
+                         "gbs": sw["bytes"] / (sw["ms"] / 1e3) / 1e9,
+                         "postings_per_s": sw["postings"] / (sw["ms"] / 1e3),
+                         "frac_of_hbm_peak": sw["bytes"] / (sw["ms"] / 1e3) / 1e9 / peak,
+                         "note": "every block of the shard decoded once per launch; the index "
+                                 "(> L2) is streamed from HBM"},
     }
-    # decode-only sweep over every block of the shard (SURVEY §8(d) C5 sweep row)
-    sw = ix.griffin_debug_decode_all(iters=3)
-    line["decode_sweep"] = {"ms": sw["ms"], "postings": sw["postings"], "bytes": sw["bytes"],
-                            "gbs": sw["bytes"] / (sw["ms"] / 1e3) / 1e9,
-                            "postings_per_s": sw["postings"] / (sw["ms"] / 1e3),
-                            "frac_of_hbm_peak": sw["bytes"] / (sw["ms"] / 1e3) / 1e9 / peak}
-    traffic = _ncu_traffic(args.config, dom)
-    if traffic is not None:
-        line["roofline"]["traffic"] = traffic
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        base, _, _ = oracle_baseline(corpus, ql, k, B, budget_s=args.cpu_budget)
-        line["cpu_baseline"] = base
+    if rank == 0 and not args.no_cpu_baseline:
+        # oracle on a bounded sample of the LAST timed batch: the cpu_baseline,
+        # and the parity reference for the same queries of the GPU's results
+        osm = OracleSample(corpus, last_batch, k, B, budget_s=args.cpu_budget)
+        dt = osm.run()
+        line["cpu_baseline"] = osm.baseline(osm.m / dt, nq)
+        gd, gs, gc = _keys_to_rows(last_keys, last_cnts, nq, k)
+        od, os_, oc = osm.res
+        m = osm.m
+        ok_c = np.array_equal(gc[:m], oc)
+        ok_d = np.array_equal(gd[:m], od)
+        ok_s = np.array_equal(gs[:m].view(np.uint32), os_.view(np.uint32))
+        line["parity"] = {"queries_checked": m, "of": nq, "batch": last_i % NB,
+                          "bit_exact": bool(ok_c and ok_d and ok_s),
+                          "what": "last timed step's top-k (docIDs, order, score bits, counts) "
+                                  "vs the CPU oracle on the same queries"}
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -468,14 +539,15 @@ def run_gpu(args):
 
 
 def _ncu_traffic(config, kernel):
-    """dram read+write bytes per launch of `kernel` from the committed ncu summary."""
+    """ncu dram read+write bytes per launch of `kernel` from the committed summary."""
     p = os.path.join(ROOT, "profiles", f"ncu_summary_{config}.json")
     if not os.path.exists(p):
         return None
     try:
         with open(p) as f:
             d = json.load(f)
-        return d.get("dram_bytes_per_launch", {}).get(kernel)
+        v = d.get("dram_bytes_per_launch", {}).get(kernel)
+        return v if v else None
     except (OSError, ValueError):
         return None
 
@@ -485,22 +557,20 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="c2", choices=sorted(WORKLOAD_DESC))
+    ap.add_argument("--config", default="c5", choices=sorted(WORKLOAD_DESC))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--latency-queries", type=int, default=1000)
     ap.add_argument("--streams", type=int, default=None,
                     help="batches in flight on separate streams/workspaces (N=1 only); default "
-                         "3 for the 1K-query configs, 2 for the 10K-query top-1000 batches "
-                         "(three workspaces of those exceed HBM)")
-    ap.add_argument("--shard-mode", default="docid", choices=["docid", "replicate"],
-                    help="N>1: docID-range shards + exchange, or a replicated index per rank")
-    ap.add_argument("--exchange", default="allgather", choices=["allgather", "sliced"],
-                    help="docid shards: all-gather of per-shard top-k, or query-sliced all-to-all")
+                         "3 for the 1K-query configs, 2 for the 10K-query batches")
+    ap.add_argument("--reuse", default="auto", choices=["auto", "on", "off"],
+                    help="batch decode-once of hot lists into an HBM arena")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.streams is None:
         args.streams = 2 if args.config in ("c4", "c5") else 3
+    args.gpus = int(os.environ.get("WORLD_SIZE", args.gpus))
     if args.impl == "reference":
         run_reference(args)
     else:

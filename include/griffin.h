@@ -61,8 +61,8 @@ typedef enum {
 /* Corpus in CSR form (host pointers).  Term t's postings are
  * docids[list_offsets[t] .. list_offsets[t+1]) with matching tfs; docIDs strictly
  * increasing and < num_docs; tfs >= 1 (the per-posting "document frequency" of
- * P:357-361 / P:1009-1010 read as term frequency); tfs > 65535 are
- * clamped to 65535.  doc_lengths[num_docs] are the BM25 document lengths
+ * P:357-361 / P:1009-1010 read as term frequency), any value up to
+ * 2^32-1, stored losslessly.  doc_lengths[num_docs] are the BM25 document lengths
  * (SURVEY A13); their sum must be > 0. */
 typedef struct {
   uint32_t num_docs;
@@ -77,7 +77,8 @@ typedef struct {
   uint32_t block_size;   /* EF block length B: 64..512, multiple of 32; 0 -> 128 */
   double bm25_k1;        /* BM25 k1 (paper silent); <= 0 -> 1.2 */
   double bm25_b;         /* BM25 b; < 0 -> 0.75 */
-  uint32_t gallop_ratio; /* T: a round gallops iff |S| > T*|R|; 0 -> block_size */
+  uint32_t gallop_ratio; /* T: a round gallops iff |S| > T*|R|; 0 -> max(4, block_size/8),
+                            the B200 crossover measured in DESIGN.md (the paper's T = B) */
   int32_t device;        /* CUDA device ordinal to build on; < 0 -> current device */
   uint32_t shard_index;  /* docID-range shard g of num_shards */
   uint32_t num_shards;   /* 0 or 1 -> unsharded */
@@ -118,6 +119,13 @@ typedef struct {
   uint64_t dec_alg_bytes;    /* compressed bytes + skip entries read, decoded u32 written */
   uint64_t dec_payload_bytes;
   uint64_t dec_postings;
+  /* SURVEY §8(d) algorithmic bytes: as alg_bytes, but postings read from the
+   * decode-once arena are charged at their blocks' compressed size (payload +
+   * 8-B skip/meta) instead of 4 B each; dec_c8d_bytes = the compressed bytes
+   * the decode-once kernel reads (its arena writes are not algorithmic). */
+  uint64_t c8d_bytes;
+  uint64_t dec_c8d_bytes;
+  uint64_t arena_postings;   /* decoded-arena postings read by the intersect kernels */
 } griffin_profile;
 
 /* ---- index ------------------------------------------------------------------

@@ -69,7 +69,9 @@ class Profile(ctypes.Structure):
                 ("payload_bytes", ctypes.c_uint64), ("decoded_postings", ctypes.c_uint64),
                 ("survivors", ctypes.c_uint64), ("ms_decode", ctypes.c_double),
                 ("launches_decode", ctypes.c_uint64), ("dec_alg_bytes", ctypes.c_uint64),
-                ("dec_payload_bytes", ctypes.c_uint64), ("dec_postings", ctypes.c_uint64)]
+                ("dec_payload_bytes", ctypes.c_uint64), ("dec_postings", ctypes.c_uint64),
+                ("c8d_bytes", ctypes.c_uint64), ("dec_c8d_bytes", ctypes.c_uint64),
+                ("arena_postings", ctypes.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -174,12 +176,34 @@ def _submit(ih, wh, offsets, terms, k, stream):
     return (len(off) - 1, k)
 
 
-def _collect(ih, wh, pend, out=None):
+class _ViewKeeper:
+    """Base object of zero-copy result views: keeps the owning workspace (or
+    index) alive and defers its close() until the last view is gone, so a view
+    never points into freed pinned memory.  Its contents are only meaningful
+    until the next submit on that workspace (the library keeps superseded
+    staging buffers allocated until the workspace is freed)."""
+
+    def __init__(self, owner):
+        # a workspace's views also pin its index (destroying the index frees
+        # every workspace of it)
+        self.owners = [owner] + ([owner.index] if hasattr(owner, "index") else [])
+        for o in self.owners:
+            o._live_views += 1
+
+    def __del__(self):
+        for o in self.owners:
+            o._live_views -= 1
+            if o._live_views == 0 and o._close_deferred:
+                o._close_deferred = False
+                o.close()
+
+
+def _collect(ih, wh, pend, out=None, owner=None):
     """out: optional (docids u32 >= nq*k, scores f32 >= nq*k, counts u32 >= nq)
     arrays to fill (a serving loop reuses them instead of faulting in fresh
     pages every batch), or "view": no copy — read-only numpy views of the
     workspace's pinned staging (griffin_query_batch_results), valid until the
-    next submit on that workspace."""
+    next submit on that workspace; the views keep `owner` alive."""
     nq, k = pend
     if isinstance(out, str) and out == "view":
         lib = load_library()
@@ -187,11 +211,14 @@ def _collect(ih, wh, pend, out=None):
         pd, ps, pc = _vp(), _vp(), _vp()
         _check(lib.griffin_query_batch_results(ih, wh, ctypes.byref(pd), ctypes.byref(ps),
                                                ctypes.byref(pc)))
+        keeper = _ViewKeeper(owner) if owner is not None else None
 
         def view(p, n, ct, dt):
             if n == 0:
                 return np.zeros(0, dt)
-            a = np.ctypeslib.as_array(ctypes.cast(p, ctypes.POINTER(ct)), shape=(n,)).view(dt)
+            buf = (ct * n).from_address(p.value)
+            buf._keeper = keeper   # numpy holds buf as the array's base
+            a = np.frombuffer(buf, dtype=dt)
             a.flags.writeable = False
             return a
         return (view(pd, nq * k, ctypes.c_uint32, np.uint32).reshape(nq, k),
@@ -258,7 +285,13 @@ class GriffinIndex:
         self.num_terms = len(off) - 1
         self.block_size = block_size
 
+    _live_views = 0
+    _close_deferred = False
+
     def close(self):
+        if self._live_views:   # zero-copy result views still point into its staging
+            self._close_deferred = True
+            return
         if getattr(self, "h", None) and _lib is not None:
             _lib.griffin_index_destroy(self.h)
             self.h = None
@@ -316,7 +349,7 @@ class GriffinIndex:
         self._pend = _submit(self.h, None, offsets, terms, k, stream)
 
     def griffin_query_batch_collect(self, out=None):
-        out = _collect(self.h, None, getattr(self, "_pend", (0, 1)), out)
+        out = _collect(self.h, None, getattr(self, "_pend", (0, 1)), out, owner=self)
         self._pend = (0, 1)
         return out
 
@@ -411,7 +444,13 @@ class GriffinWorkspace:
         _check(load_library().griffin_workspace_create(index.h, ctypes.byref(h)))
         self.h = h
 
+    _live_views = 0
+    _close_deferred = False
+
     def close(self):
+        if self._live_views:   # zero-copy result views still point into its staging
+            self._close_deferred = True
+            return
         if getattr(self, "h", None) and _lib is not None and getattr(self.index, "h", None):
             _lib.griffin_workspace_destroy(self.index.h, self.h)
         self.h = None
@@ -441,7 +480,7 @@ class GriffinWorkspace:
         self._pend = _submit(self.index.h, self.h, offsets, terms, k, stream)
 
     def griffin_query_batch_collect(self, out=None):
-        out = _collect(self.index.h, self.h, getattr(self, "_pend", (0, 1)), out)
+        out = _collect(self.index.h, self.h, getattr(self, "_pend", (0, 1)), out, owner=self)
         self._pend = (0, 1)
         return out
 

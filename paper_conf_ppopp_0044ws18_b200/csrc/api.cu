@@ -36,7 +36,7 @@ static griffin_status invalid(const std::string &m) {
 
 static griffin_status ensure_pinned_ws(Workspace &w, size_t bytes) {
   if (w.h_pinned_bytes >= bytes) return GRIFFIN_OK;
-  if (w.h_pinned) cudaFreeHost(w.h_pinned);
+  if (w.h_pinned) w.old_pinned.push_back(w.h_pinned);   // freed with the workspace
   w.h_pinned = nullptr;
   w.h_pinned_bytes = 0;
   size_t nb = bytes + bytes / 4 + 4096;
@@ -134,7 +134,12 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   if (!c || !out) return invalid("null corpus/out");
   *out = nullptr;
   griffin_build_opts opts{};
-  if (o) opts = *o;
+  if (o) {
+    opts = *o;
+  } else {   // NULL: every documented default (b = 0.75, the current device)
+    opts.bm25_b = -1.0;
+    opts.device = -1;
+  }
   const uint32_t B = opts.block_size ? opts.block_size : 128;
   if (B < 64 || B > 512 || (B % 32)) return invalid("block_size must be 64..512 and a multiple of 32");
   const double k1 = opts.bm25_k1 > 0 ? opts.bm25_k1 : 1.2;
@@ -237,7 +242,7 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
     uint64_t o = post_off[t];
     for (uint64_t p = lo[t]; p < hi[t]; ++p, ++o) {
       ldoc[o] = c->docids[p] - ix->doc_base;
-      ltf[o] = std::min<uint32_t>(c->tfs[p], 65535u);
+      ltf[o] = c->tfs[p];   // lossless: packed at bits(max tf - 1) <= 32
     }
   }
   griffin_status s = encode_index(ix, ldoc.data(), ltf.data(), post_off);
@@ -311,8 +316,9 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
   if (!ix) return invalid("null index");
   if (nq == 0) return GRIFFIN_OK;
   if (!qoffs || !terms || !out_docids || !out_scores || !out_counts) return invalid("null argument");
-  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
   std::lock_guard<std::mutex> lk(ix->mu);
+  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
+  ix->ws.results_valid = false;
   DeviceGuard guard(ix->device);
   uint32_t max_terms = 1;
   griffin_status s = reserve_for(ix, ix->ws, nq, qoffs, terms, k, &max_terms);
@@ -458,9 +464,10 @@ griffin_status griffin_query(griffin_index *ix, const uint32_t *terms, uint32_t 
                              uint32_t *out_docids, float *out_scores, uint32_t *out_count) {
   if (nterms == 0) return invalid("nterms must be > 0");
   if (!ix || !terms || !out_docids || !out_scores || !out_count) return invalid("null argument");
-  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
   if (ix->use_graphs && !ix->profiling) {
     std::lock_guard<std::mutex> lk(ix->mu);
+    if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
+    ix->ws.results_valid = false;
     DeviceGuard guard(ix->device);
     griffin_status s = query_graph(ix, terms, nterms, k, out_docids, out_scores, out_count);
     if (s != GRIFFIN_ERR_UNSUPPORTED) return s;
@@ -485,8 +492,9 @@ griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq, const 
   if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
   if (max_terms == 0 || max_terms > GRIFFIN_MAX_TERMS) return invalid("max_terms out of range");
   if (nq == 0) return GRIFFIN_OK;
-  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
   std::lock_guard<std::mutex> lk(ix->mu);
+  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
+  ix->ws.results_valid = false;
   DeviceGuard guard(ix->device);
   return run_batch(ix, ix->ws, nq, d_qoffs, d_terms, max_terms, k, d_out_keys, d_out_counts,
                    static_cast<cudaStream_t>(stream), true, ix->mode);
@@ -519,6 +527,8 @@ static void free_workspace(Workspace &w) {
                     &w.sbkt_tmp, &w.flt, &w.fstate})
     b->release();
   if (w.h_pinned) cudaFreeHost(w.h_pinned);
+  for (void *p : w.old_pinned) cudaFreeHost(p);
+  w.old_pinned.clear();
   w.h_pinned = nullptr;
   w.h_pinned_bytes = 0;
   if (w.done) cudaEventDestroy(w.done);
@@ -581,8 +591,9 @@ griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *
   if (!ix) return invalid("null index");
   if (nq && (!qoffs || !terms)) return invalid("null argument");
   Workspace &w = ws ? *reinterpret_cast<Workspace *>(ws) : ix->ws;
-  if (w.pending) return invalid("workspace has a submitted batch not yet collected");
   std::lock_guard<std::mutex> lk(ix->mu);
+  if (w.pending) return invalid("workspace has a submitted batch not yet collected");
+  w.results_valid = false;
   DeviceGuard guard(ix->device);
   cudaStream_t st = stream ? static_cast<cudaStream_t>(stream) : ix->stream;
   uint32_t max_terms = 1;
@@ -639,7 +650,8 @@ griffin_status griffin_query_batch_results(griffin_index *ix, griffin_workspace 
                                            const uint32_t **counts) {
   if (!ix || !docids || !scores || !counts) return invalid("null argument");
   Workspace &w = ws ? *reinterpret_cast<Workspace *>(ws) : ix->ws;
-  if (w.pending || !w.h_pinned) return invalid("no collected batch on this workspace");
+  if (w.pending || !w.results_valid || !w.h_pinned)
+    return invalid("no successfully collected batch on this workspace");
   const size_t nk = (size_t)w.pend_nq * w.pend_k;
   const uint8_t *ho = static_cast<const uint8_t *>(w.h_pinned) + w.pend_out;
   *docids = reinterpret_cast<const uint32_t *>(ho);
@@ -660,21 +672,33 @@ griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace 
     return invalid("null argument");
   {
     DeviceGuard guard(ix->device);
-    w.pending = false;
-    GRIFFIN_CUDA_TRY(cudaEventSynchronize(w.done));   // without the index lock: others submit
+    cudaError_t e = cudaEventSynchronize(w.done);   // without the index lock: others submit
+    if (e != cudaSuccess) {
+      w.results_valid = false;
+      w.pending = false;
+      set_error(std::string("cudaEventSynchronize: ") + cudaGetErrorString(e));
+      return GRIFFIN_ERR_CUDA;
+    }
   }
   const uint8_t *ho = static_cast<const uint8_t *>(w.h_pinned) + w.pend_out;
   if (*reinterpret_cast<const int *>(ho + nk * 8 + (size_t)w.pend_nq * 4)) {
     std::lock_guard<std::mutex> lk(ix->mu);
     DeviceGuard guard(ix->device);
     griffin_status s = read_status(ix, w, w.pend_stream);   // clears the device flag
-    if (s) return s;
+    if (s) {
+      w.results_valid = false;
+      w.pending = false;
+      return s;
+    }
   }
   if (w.pend_nq && copy) {
     std::memcpy(out_docids, ho, nk * 4);
     std::memcpy(out_scores, ho + nk * 4, nk * 4);
     std::memcpy(out_counts, ho + nk * 8, (size_t)w.pend_nq * 4);
   }
+  // only now may a synchronous call on this workspace reuse the staging
+  w.results_valid = true;
+  w.pending = false;
   return GRIFFIN_OK;
 }
 
@@ -761,6 +785,7 @@ griffin_status griffin_reset_profile(griffin_index *ix) {
     if (w->scal.p) {
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.p, 0, 4 * 8));
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDec, 0, 3 * 8));
+      GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalArena, 0, 3 * 8));
     }
   return GRIFFIN_OK;
 }
@@ -787,6 +812,7 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
   all.push_back(&ix->ws);
   out->alg_bytes = out->payload_bytes = out->decoded_postings = out->survivors = 0;
   out->dec_alg_bytes = out->dec_payload_bytes = out->dec_postings = 0;
+  out->c8d_bytes = out->dec_c8d_bytes = out->arena_postings = 0;
   for (Workspace *w : all) {
     if (!w->scal.p) continue;
     unsigned long long c[kScalCount];
@@ -798,6 +824,9 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
     out->dec_alg_bytes += c[kScalDec + 0];
     out->dec_payload_bytes += c[kScalDec + 1];
     out->dec_postings += c[kScalDec + 2];
+    out->arena_postings += c[kScalArena];
+    out->c8d_bytes += c[0] - 4ull * c[kScalArena] + c[kScalArena + 1];
+    out->dec_c8d_bytes += c[kScalDecC8d];
   }
   return GRIFFIN_OK;
 }
@@ -921,6 +950,8 @@ griffin_status griffin_debug_intersect(griffin_index *ix, const uint32_t *terms,
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
   const uint32_t offs[2] = {0, nterms};
+  if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
+  ix->ws.results_valid = false;
   uint32_t max_terms = 1;
   griffin_status s = reserve_for(ix, ix->ws, 1, offs, terms, 1, &max_terms);
   if (s) return s;

@@ -468,6 +468,212 @@ __device__ __forceinline__ void warp_decode_staged(const uint32_t *__restrict__ 
   warp_decode_staged(stg, first, y, dst, cnt, lut, s);
 }
 
+// ---- run decoder: several blocks per warp, 32 consecutive elements per lane -----
+// (B = 64/128/256/512.)  Alg. 1 re-cut for instruction count rather than for
+// the paper's thread-per-element mapping: a group of Lb = B/32 lanes decodes one
+// block, so one warp pass decodes 32/Lb blocks (16 at B = 64, 8 at B = 128)
+// and every per-block and per-lane step is paid once per 32 postings:
+//  * Alg. 1 l.2-3 (prefix sum): lane l of the group popcounts high words l,
+//    l+Lb and l+2Lb (a block's unary stream has L < 3n <= 3*32*Lb bits); one
+//    packed shuffle scan of width Lb gives all three inclusive prefixes.
+//  * l.4-8 (scheduling): element k0 = 32t, where lane t starts, lies in the
+//    word whose [exclusive, inclusive) prefix interval contains 32t; an
+//    interval of <= 32 ones holds at most one multiple of 32, so every word
+//    lane writes (word, exclusive prefix) straight into its target's record (no
+//    search), and the target selects the bit with the byte LUT.
+//  * l.9-10: the next ones come from a 96-bit stream of the high bits after the
+//    current one, bit-reversed into three registers: FLO finds the next one
+//    (i = its reversed index; 31 - i zeros precede it, so h += 31 - i), and a
+//    funnel shift by 32 - i drops it and refills from the lower registers.  The
+//    stream is re-seeded from shared memory after 16 elements (the position of
+//    element 15's one is k0 + 15 + h), so no select is needed for the second
+//    half.  x = first + (h << b) + low, low fields funnel-shifted out of the
+//    staged low stream (a lane's 32 fields start word-aligned at word l*b).
+//  * A lane that meets 32 zeros in a row inside its stream (~1e-4 of lanes at
+//    the 1/3 .. 1/2 densities EF gives) takes the serial window walk.
+// Inputs in lanes [l0, l0+nb): the block's meta word y, first docID f and its
+// staged offset so (16-B units from stg).  Block i goes to dst + i*B.  `rec` is
+// 32 words of per-warp scratch; stg needs kRunSlack words of read slack.
+constexpr uint32_t kRunSlack = 40;   // a partial block's last lane reads <= 32 + 4 words past it
+__host__ __device__ inline bool run_decoder_ok(uint32_t B) {
+  return B == 64 || B == 128 || B == 256 || B == 512;
+}
+
+// Serial fallback (rare): elements [kfrom, kto) of the block, element kfrom's
+// one being the first one at or after high-stream bit c; refilled 32-bit window.
+template <class Sink>
+__device__ __forceinline__ void lane_walk(const uint32_t *__restrict__ blk, const uint32_t *__restrict__ hs,
+                                       uint32_t first, uint32_t b, uint32_t mask, uint32_t kfrom,
+                                       uint32_t kto, uint32_t c, uint32_t *dst, Sink &sink) {
+  uint32_t wb = c;
+  uint32_t win = __funnelshift_r(hs[wb >> 5], hs[(wb >> 5) + 1], wb);
+  for (uint32_t k = kfrom; k < kto; ++k) {
+    while (win == 0u) {
+      wb += 32u;
+      win = __funnelshift_r(hs[wb >> 5], hs[(wb >> 5) + 1], wb);
+    }
+    const uint32_t p = wb + (__ffs(win) - 1u);
+    win &= win - 1u;
+    const uint32_t bp = k * b;
+    const uint32_t lo = __funnelshift_r(blk[bp >> 5], blk[(bp >> 5) + 1], bp) & mask;
+    sink.put(dst + k, first + (((p - k) << b) | lo));
+  }
+}
+
+// FLO: bit index of the highest set bit (0xFFFFFFFF for 0)
+__device__ __forceinline__ uint32_t flo_u32(uint32_t x) {
+  uint32_t r;
+  asm("bfind.u32 %0, %1;" : "=r"(r) : "r"(x));
+  return r;
+}
+// x << s for s in [0, 32] (32 -> 0)
+__device__ __forceinline__ uint32_t shl_c(uint32_t x, uint32_t s) {
+  uint32_t r;
+  asm("shl.b32 %0, %1, %2;" : "=r"(r) : "r"(x), "r"(s));
+  return r;
+}
+
+// 96 high-stream bits starting at bit c, bit-reversed (bit c -> bit 31 of s0)
+__device__ __forceinline__ void seed_stream(const uint32_t *__restrict__ hs, uint32_t c,
+                                            uint32_t &s0, uint32_t &s1, uint32_t &s2) {
+  const uint32_t cw = c >> 5;
+  const uint32_t a0 = hs[cw], a1 = hs[cw + 1], a2 = hs[cw + 2], a3 = hs[cw + 3];
+  s0 = __brev(__funnelshift_r(a0, a1, c));
+  s1 = __brev(__funnelshift_r(a1, a2, c));
+  s2 = __brev(__funnelshift_r(a2, a3, c));
+}
+
+// next one of the stream: returns its reversed index i (h grows by 31 - i);
+// bad collects i (its top bit is set iff the stream's first word was empty)
+__device__ __forceinline__ uint32_t stream_next(uint32_t &s0, uint32_t &s1, uint32_t &s2,
+                                                uint32_t &bad) {
+  const uint32_t i = flo_u32(s0);
+  bad |= i;
+  const uint32_t sh = 32u - i;   // drop the one and the zeros before it
+  s0 = __funnelshift_lc(s1, s0, sh);
+  s1 = __funnelshift_lc(s2, s1, sh);
+  s2 = shl_c(s2, sh);
+  return i;
+}
+
+template <uint32_t LG, class Sink>
+__device__ __forceinline__ void warp_decode_runs_t(const uint32_t *__restrict__ stg, uint32_t l0,
+                                                   uint32_t nb, uint32_t y_l, uint32_t f_l,
+                                                   uint32_t so_l, uint32_t *dst,
+                                                   uint32_t *__restrict__ rec,
+                                                   const uint8_t *__restrict__ lut, Sink &sink) {
+  constexpr uint32_t Lb = 1u << LG, bpw = 32u >> LG, B = Lb * 32u;
+  const uint32_t lane = lane_id();
+  const uint32_t g = lane >> LG, l = lane & (Lb - 1u);
+  uint32_t *r = rec + (g << LG);
+  for (uint32_t i = 0; i < nb; i += bpw) {
+    const uint32_t bi = i + g;
+    const bool act = bi < nb;
+    const uint32_t src = (l0 + (act ? bi : nb - 1u)) & 31u;
+    const uint32_t y = __shfl_sync(0xffffffffu, y_l, src);
+    const uint32_t first = __shfl_sync(0xffffffffu, f_l, src);
+    const uint32_t so = __shfl_sync(0xffffffffu, so_l, src);
+    const uint32_t b = meta_b(y), n = act ? meta_n(y) : 0u, hw = act ? meta_hw(y) : 0u;
+    const uint32_t *blk = stg + so * 4u;
+    const uint32_t *hs = blk + low_words(n, b);
+    const uint32_t wa = l < hw ? hs[l] : 0u;
+    const uint32_t wb = l + Lb < hw ? hs[l + Lb] : 0u;
+    const uint32_t wc = l + 2u * Lb < hw ? hs[l + 2u * Lb] : 0u;
+    const uint32_t ca = __popc(wa), cb = __popc(wb), cc = __popc(wc);
+    uint32_t c = ca | (cb << 10) | (cc << 20);   // three 10-bit counters (<= 512 each)
+#pragma unroll
+    for (uint32_t d = 1; d < Lb; d <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, c, d, Lb);
+      if (l >= d) c += t;
+    }
+    const uint32_t tot = __shfl_sync(0xffffffffu, c, Lb - 1u, Lb);
+    const uint32_t ta = tot & 0x3FFu, tb = (tot >> 10) & 0x3FFu;
+    {  // exclusive prefixes of words l, l+Lb, l+2Lb; record the target (if any) of each
+      const uint32_t ea = (c & 0x3FFu) - ca;
+      const uint32_t eb = ta + ((c >> 10) & 0x3FFu) - cb;
+      const uint32_t ec = ta + tb + (c >> 20) - cc;
+      const uint32_t xa = (ea + 31u) >> 5, xb = (eb + 31u) >> 5, xc = (ec + 31u) >> 5;
+      if ((xa << 5) < ea + ca) r[xa] = l | (ea << 8);
+      if ((xb << 5) < eb + cb) r[xb] = (l + Lb) | (eb << 8);
+      if ((xc << 5) < ec + cc) r[xc] = (l + 2u * Lb) | (ec << 8);
+    }
+    __syncwarp();
+    const uint32_t k0 = l << 5;
+    if (k0 < n) {
+      const uint32_t rv = r[l];
+      const uint32_t w = rv & 0xFFu, ex = rv >> 8;
+      const uint32_t p0 = (w << 5) + select_in_word(hs[w], k0 - ex, lut);
+      const uint32_t ne = min(32u, n - k0);
+      const uint32_t mask = b ? (0xFFFFFFFFu >> (32u - b)) : 0u;
+      // low fields: element k0 + j at bit j*b of the lane's run (word l*b)
+      const uint32_t *lw = blk + l * b;
+      uint32_t s0, s1, s2, bad = 0u;
+      uint32_t h = p0 - k0;   // high part of the current element
+      uint32_t *out = dst + bi * B;
+      // (a lane of a list's partial last block decodes all 32 slots from the
+      // staged bytes after its block — the staging area's read slack covers
+      // them — and stores only its ne elements)
+      seed_stream(hs, p0 + 1u, s0, s1, s2);
+#pragma unroll
+      for (uint32_t half = 0; half < 2; ++half) {
+        // half 1 re-seeds after element 15's one, at bit k0 + 15 + h + 1
+        if (half) seed_stream(hs, k0 + 16u + h, s0, s1, s2);
+        const uint32_t c_half = k0 + half * 16u + h;   // search start for the walk
+        uint32_t lo[16], v[16];
+        if (b <= 16u) {   // two fields per 32-bit window
+#pragma unroll
+          for (uint32_t j = 0; j < 16; j += 2) {
+            const uint32_t o = (half * 16u + j) * b;
+            const uint32_t wv = __funnelshift_r(lw[o >> 5], lw[(o >> 5) + 1], o);
+            lo[j] = wv & mask;
+            lo[j + 1] = (wv >> b) & mask;
+          }
+        } else {
+#pragma unroll
+          for (uint32_t j = 0; j < 16; ++j) {
+            const uint32_t o = (half * 16u + j) * b;
+            lo[j] = __funnelshift_r(lw[o >> 5], lw[(o >> 5) + 1], o) & mask;
+          }
+        }
+#pragma unroll
+        for (uint32_t j = 0; j < 16; ++j) {
+          if (half || j) h += 31u - stream_next(s0, s1, s2, bad);
+          v[j] = first + (h << b) + lo[j];
+        }
+        if (ne == 32u && !(bad >> 31)) {
+#pragma unroll
+          for (uint32_t j = 0; j < 16; j += 4)
+            sink.put4(out + k0 + half * 16u + j, make_uint4(v[j], v[j + 1], v[j + 2], v[j + 3]));
+        } else if (!(bad >> 31)) {   // partial block: this lane's first ne elements
+#pragma unroll
+          for (uint32_t j = 0; j < 16; ++j)
+            if (half * 16u + j < ne) sink.put(out + k0 + half * 16u + j, v[j]);
+        } else {   // a run of >= 32 zeros inside the stream: walk this half (and the next)
+          lane_walk(blk, hs, first, b, mask, k0 + half * 16u, k0 + ne,
+                    half ? c_half : p0, out, sink);
+          break;
+        }
+        if (half * 16u + 16u >= ne) break;
+      }
+    }
+    __syncwarp();
+  }
+}
+
+template <class Sink>
+__device__ __forceinline__ void warp_decode_runs(const uint32_t *__restrict__ stg, uint32_t l0,
+                                                 uint32_t nb, uint32_t y_l, uint32_t f_l,
+                                                 uint32_t so_l, uint32_t *dst, uint32_t B,
+                                                 uint32_t *__restrict__ rec,
+                                                 const uint8_t *__restrict__ lut, Sink &sink) {
+  switch (B) {   // uniform per index: only one instantiation ever runs
+    case 64: warp_decode_runs_t<1>(stg, l0, nb, y_l, f_l, so_l, dst, rec, lut, sink); break;
+    case 128: warp_decode_runs_t<2>(stg, l0, nb, y_l, f_l, so_l, dst, rec, lut, sink); break;
+    case 256: warp_decode_runs_t<3>(stg, l0, nb, y_l, f_l, so_l, dst, rec, lut, sink); break;
+    default: warp_decode_runs_t<4>(stg, l0, nb, y_l, f_l, so_l, dst, rec, lut, sink); break;
+  }
+}
+
 // ---- EF NextGEQ inside one staged block -------------------
 // Index of the first element >= x of the block staged at stg (n if none) and
 // its value in `val`, without decoding the block: the elements whose high part

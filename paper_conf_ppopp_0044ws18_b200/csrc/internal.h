@@ -2,6 +2,7 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdint>
 #include <mutex>
 #include <string>
@@ -63,15 +64,20 @@ struct Workspace {
   DevBuf arena;                                        // decoded lists, nblocks * B u32
   DevBuf sbkt_cnt, sbkt_pos, sbkt_tmp;                 // S-locality unit order buckets
   size_t nq_cap = 0, unit_cap = 0, entry_cap = 0;
-  // pinned host staging
+  // pinned host staging; a grown buffer's predecessors stay allocated until the
+  // workspace is freed (zero-copy result views may still point into them)
   void *h_pinned = nullptr;
   size_t h_pinned_bytes = 0;
+  std::vector<void *> old_pinned;
   // griffin_query_batch_submit/collect: the batch in flight on this workspace
   cudaEvent_t done = nullptr;
   cudaStream_t pend_stream = nullptr;
   uint32_t pend_nq = 0, pend_k = 0;
   size_t pend_out = 0;   // byte offset of the results in h_pinned
-  bool pending = false;
+  // a submitted batch not yet collected; read by synchronous calls under the
+  // index mutex, cleared by collect only after the results were read out
+  std::atomic<bool> pending{false};
+  bool results_valid = false;   // the last collect succeeded (griffin_query_batch_results)
 };
 
 // Offsets of the scalar block (u64 slots).
@@ -83,7 +89,9 @@ enum : int {
   kScalTotals = 7,    // u64 x2: sum cap, sum units (written by plan kernels)
   kScalDec = 10,      // 3 x u64: decode-once alg bytes, payload bytes, postings
   kScalPerm = 13,     // 2 x u64: unit order list head (merge units) / tail (the rest)
-  kScalCount = 15
+  kScalArena = 15,    // 2 x u64: decoded-arena postings read by intersect, their compressed bytes
+  kScalDecC8d = 17,   // u64: decode-once compressed bytes read (payload + skip/meta)
+  kScalCount = 18
 };
 
 constexpr uint32_t kBumpChunk = 256;   // bump-area entries grabbed per warp atomic

@@ -198,8 +198,13 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
 
 // ------------------------------------------------------------------- intersect
 
+// Per-warp counters live in the warp's shared memory (lane 0 updates them),
+// not in registers: the kernel runs at the 80-register cap.
+enum : int { kCAlg = 0, kCPay, kCPost, kCSurv, kCApost, kCAcomp, kCNum };
 struct Acc {
-  unsigned long long alg = 0, pay = 0, post = 0, surv = 0;
+  // alg bytes, payload bytes, decoded postings, survivors, decoded-arena postings
+  // read, their compressed bytes
+  unsigned long long *ctr = nullptr;
   // this warp's bump chunk in warp smem: {next free entry (u64), entries left (u32)}
   unsigned long long *boff = nullptr;
   uint32_t *bleft = nullptr;
@@ -238,13 +243,23 @@ __host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D) {
 constexpr uint32_t kTileSlack = 64;
 // read slack after the staging area: decoders read a word or two past a block's
 // high stream (look-ahead windows), also when it ends the staging area
-constexpr uint32_t kStgSlack = 4;
+constexpr uint32_t kStgSlack = kRunSlack;   // >= the run decoder's over-read
+// per-warp header words: mbarrier (0-1), bump left (2), bump offset (4-5),
+// counters (8-19)
+constexpr uint32_t kWarpHdr = 24;
 // with_tile = false: no decode tile (kernels that decode straight to HBM)
 __host__ __device__ inline uint32_t warp_smem_words(uint32_t B, uint32_t D, bool with_tile = true) {
-  return 8 + 64 + (B + 32) + stage_words(B, D) + kStgSlack +
+  return kWarpHdr + 64 + (B + 32) + stage_words(B, D) + kStgSlack +
          (with_tile ? (D + 2) * B + kTileSlack : 0u);
 }
 constexpr uint32_t kLutBytes = 2048;
+// Run length (D + 2 blocks) of the decode-only kernels (sweep, decode-once):
+// 2048 postings, i.e. two full passes of the run decoder (32/Lb = 1024/B
+// blocks per pass), so its lane groups are never idle inside a run.
+__host__ __device__ inline uint32_t sweep_D(uint32_t B) {
+  const uint32_t r = 2048u / B;
+  return r > 4u ? r - 2u : 2u;
+}
 
 struct WarpSmem {
   uint64_t *mbar;
@@ -261,7 +276,7 @@ __device__ __forceinline__ WarpSmem carve_warp_smem(uint4 *smem4, uint32_t B, ui
   uint32_t *wb = reinterpret_cast<uint32_t *>(base + kLutBytes) +
                  (threadIdx.x >> 5) * warp_smem_words(B, D, with_tile);
   w.mbar = reinterpret_cast<uint64_t *>(wb);   // words 0-1; 2: bump left; 4-5: bump offset
-  w.cnt = wb + 8;
+  w.cnt = wb + kWarpHdr;
   w.aux = w.cnt + 64;
   w.stg = w.aux + B + 32;
   w.tile = with_tile ? w.stg + stage_words(B, D) + kStgSlack : nullptr;
@@ -310,6 +325,10 @@ template <class Sink, bool PAIR = true>
 __device__ __forceinline__ void decode_staged_lanes(const WarpSmem &w, uint32_t B, uint32_t l0,
                                                     uint32_t nb, uint32_t y, uint32_t f,
                                                     uint32_t so, uint32_t *dst, Sink &sink) {
+  if (run_decoder_ok(B)) {   // power-of-two B: several blocks per warp pass
+    warp_decode_runs(w.stg, l0, nb, y, f, so, dst, B, w.cnt, w.lut, sink);
+    return;
+  }
   uint32_t i0 = 0;
   if (PAIR && B == 128u) {   // pairs; an odd last block takes the single-block decoder
     const uint32_t npair = nb & ~1u;
@@ -443,8 +462,8 @@ __device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, co
   if (lane == 0) {
     a.unit_off[u] = off;
     a.unit_cnt[u] = cnt;
-    acc.surv += cnt;
-    acc.alg += (unsigned long long)cnt * (KIND == 0 ? 20u : 16u);
+    acc.ctr[kCSurv] += cnt;
+    acc.ctr[kCAlg] += (unsigned long long)cnt * (KIND == 0 ? 20u : 16u);
   }
 }
 
@@ -518,8 +537,8 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
   if (lane == 0) {
     a.unit_off[u] = off;
     a.unit_cnt[u] = cnt;
-    acc.surv += cnt;
-    acc.alg += (unsigned long long)cnt * (RC ? 20u : 16u);
+    acc.ctr[kCSurv] += cnt;
+    acc.ctr[kCAlg] += (unsigned long long)cnt * (RC ? 20u : 16u);
   }
 }
 
@@ -910,7 +929,7 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
     nrm[e] = __float_as_uint(__ldg(ix.norm + v.x));
   }
   __syncwarp();
-  if (lane == 0) acc.alg += n * 12u;
+  if (lane == 0) acc.ctr[kCAlg] += n * 12u;
   for (uint32_t r = 2; r < m && n > 0; ++r) {
     const uint32_t sid = pt[r];
     const TermInfo tS = ix.terms[sid];
@@ -931,7 +950,7 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
         probes += arena_probe_slice(decS, fS, tS.nblocks, tS.df_local, B, tileR, kidx, match,
                                     base, n);
       const uint32_t sp = __reduce_add_sync(0xffffffffu, probes);
-      if (lane == 0) acc.alg += sp * 32ull;
+      if (lane == 0) acc.ctr[kCAlg] += sp * 32ull;
     } else {
       // ---- compressed: distinct touched blocks, staged + decoded in groups ----
       uint32_t nd = 0, prev = kNone, e_first = n;
@@ -972,9 +991,9 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
         const uint32_t pay = __reduce_add_sync(0xffffffffu, lane < ng ? sz * 16u : 0u);
         const uint32_t pst = __reduce_add_sync(0xffffffffu, lane < ng && !a.nextgeq ? nn : 0u);
         if (lane == 0) {
-          acc.pay += pay;
-          acc.post += pst;
-          acc.alg += pay + 8u * ng;
+          acc.ctr[kCPay] += pay;
+          acc.ctr[kCPost] += pst;
+          acc.ctr[kCAlg] += pay + 8u * ng;
         }
         const uint32_t soff = warp_incl_scan(sz) - sz;
         stage_blocks(ix, sm, ng, mm, soff, sz, false);
@@ -1039,7 +1058,7 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
       __syncwarp();
     }
     n = nn2;
-    if (lane == 0) acc.alg += n * 4u;
+    if (lane == 0) acc.ctr[kCAlg] += n * 4u;
   }
   // ---- emit the survivors ----
   unsigned long long off = 0;
@@ -1054,8 +1073,8 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
   if (lane == 0) {
     a.unit_off[u] = off;
     a.unit_cnt[u] = cnt;
-    acc.surv += cnt;
-    acc.alg += cnt * 8ull;
+    acc.ctr[kCSurv] += cnt;
+    acc.ctr[kCAlg] += cnt * 8ull;
   }
   __syncwarp();
 }
@@ -1077,9 +1096,12 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
   Acc acc;
   acc.bleft = reinterpret_cast<uint32_t *>(sm.mbar) + 2;
   acc.boff = reinterpret_cast<unsigned long long *>(sm.mbar) + 2;
+  acc.ctr = reinterpret_cast<unsigned long long *>(sm.mbar) + 4;
   if (lane == 0) {
     *acc.bleft = 0;
     *acc.boff = 0;
+#pragma unroll
+    for (int c = 0; c < kCNum; ++c) acc.ctr[c] = 0;
   }
   // dynamic unit tickets (balances long gallop/probe units); the next ticket is
   // requested at the start of a unit so its latency overlaps the unit's work
@@ -1116,7 +1138,11 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         }
         mbar_wait(sm.mbar, sm.phase);
         sm.phase ^= 1u;
-        if (lane == 0) acc.alg += n * 4u;
+        if (lane == 0) {
+          acc.ctr[kCAlg] += n * 4u;
+          acc.ctr[kCApost] += n;
+          acc.ctr[kCAcomp] += block_size16(ix.meta[(uint64_t)tR.block0 + lu].y) * 16u + 8u;
+        }
       } else {
         const uint64_t gb = (uint64_t)tR.block0 + lu;
         const uint2 m = ix.meta[gb];
@@ -1125,9 +1151,9 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         stage_blocks(ix, sm, 1, m, 0, sz, true);
         warp_decode_staged(sm.stg, f, m.y, sm.tile, sm.cnt, sm.lut);
         if (lane == 0) {
-          acc.pay += sz * 16u;
-          acc.post += n;
-          acc.alg += sz * 16u + 8u;
+          acc.ctr[kCPay] += sz * 16u;
+          acc.ctr[kCPost] += n;
+          acc.ctr[kCAlg] += sz * 16u + 8u;
         }
       }
       emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, 0, n, lu * B, acc);
@@ -1187,7 +1213,7 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         const bool own = (isR && rb0 + lane >= i0) || (isS && sb0 + (lane - nRb) >= j0);
         const uint32_t nn = isR ? min(B, nR - (rb0 + lane) * B)
                                 : (isS ? min(B, tS.df_local - (sb0 + lane - nRb) * B) : 0u);
-        uint32_t pay = 0, post = 0, alg = 0;
+        uint32_t pay = 0, post = 0, alg = 0, ap = 0, ac = 0;
         if (own) {
           if (lm) {
             pay = sz * 16u;
@@ -1195,15 +1221,25 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
             alg = pay + 8u;
           } else {
             alg = nn * (isR && !RC ? 8u : 4u);  // intermediate (docID+score) or decoded arena
+            if (!(isR && !RC)) {   // arena block: its compressed size for the §8(d) count
+              ap = nn;
+              const uint64_t gb = isR ? (uint64_t)tR.block0 + rb0 + lane
+                                      : (uint64_t)tS.block0 + sb0 + (lane - nRb);
+              ac = block_size16(ix.meta[gb].y) * 16u + 8u;
+            }
           }
         }
         const uint32_t sp = __reduce_add_sync(0xffffffffu, pay);
         const uint32_t sn = __reduce_add_sync(0xffffffffu, post);
         const uint32_t sa = __reduce_add_sync(0xffffffffu, alg);
+        const uint32_t sap = __reduce_add_sync(0xffffffffu, ap);
+        const uint32_t sac = __reduce_add_sync(0xffffffffu, ac);
         if (lane == 0) {
-          acc.pay += sp;
-          acc.post += sn;
-          acc.alg += sa;
+          acc.ctr[kCPay] += sp;
+          acc.ctr[kCPost] += sn;
+          acc.ctr[kCAlg] += sa;
+          acc.ctr[kCApost] += sap;
+          acc.ctr[kCAcomp] += sac;
         }
       }
       // ---- TMA: decoded-arena ranges -> tiles; compressed payloads -> stg (one
@@ -1353,7 +1389,11 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         }
         mbar_wait(sm.mbar, sm.phase);
         sm.phase ^= 1u;
-        if (lane == 0) acc.alg += n * 4u;
+        if (lane == 0) {
+          acc.ctr[kCAlg] += n * 4u;
+          acc.ctr[kCApost] += n;
+          acc.ctr[kCAcomp] += block_size16(ix.meta[(uint64_t)tR.block0 + lu].y) * 16u + 8u;
+        }
       } else if (RC) {
         const uint64_t gb = (uint64_t)tR.block0 + lu;
         const uint2 m = ix.meta[gb];
@@ -1362,13 +1402,13 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
         stage_blocks(ix, sm, 1, m, 0, sz, true);
         warp_decode_staged(sm.stg, f, m.y, tileR, sm.cnt, sm.lut);
         if (lane == 0) {
-          acc.pay += sz * 16u;
-          acc.post += n;
-          acc.alg += sz * 16u + 8u;
+          acc.ctr[kCPay] += sz * 16u;
+          acc.ctr[kCPost] += n;
+          acc.ctr[kCAlg] += sz * 16u + 8u;
         }
       } else {
         load_r_chunk(Rq, nR, B, lu, tileR);
-        if (lane == 0) acc.alg += n * 8u;
+        if (lane == 0) acc.ctr[kCAlg] += n * 8u;
       }
       __syncwarp();
       const uint32_t k_lo = rec.z, k_hi = rec.w;   // from the partition stage
@@ -1404,7 +1444,7 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
           probes += arena_probe_slice(decS, fS, tS.nblocks, tS.df_local, B, tileR, kidx, match,
                                       base, n);
         const uint32_t sp = __reduce_add_sync(0xffffffffu, probes);
-        if (lane == 0) acc.alg += sp * 32ull;
+        if (lane == 0) acc.ctr[kCAlg] += sp * 32ull;
         __syncwarp();
         if (RC)
           emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
@@ -1465,9 +1505,9 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
           const uint32_t sa = __reduce_add_sync(
               0xffffffffu, own ? (sdec ? nn * 4u : sz * 16u + 8u) : 0u);
           if (lane == 0) {
-            acc.pay += sp;
-            acc.post += spn;
-            acc.alg += sa;
+            acc.ctr[kCPay] += sp;
+            acc.ctr[kCPost] += spn;
+            acc.ctr[kCAlg] += sa;
           }
         }
         uint32_t soff = 0;
@@ -1535,10 +1575,11 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
     }
   }
   if (lane == 0) {
-    if (acc.alg) atomicAdd(a.scal + kScalCounters + 0, acc.alg);
-    if (acc.pay) atomicAdd(a.scal + kScalCounters + 1, acc.pay);
-    if (acc.post) atomicAdd(a.scal + kScalCounters + 2, acc.post);
-    if (acc.surv) atomicAdd(a.scal + kScalCounters + 3, acc.surv);
+    const int slot[kCNum] = {kScalCounters, kScalCounters + 1, kScalCounters + 2,
+                             kScalCounters + 3, kScalArena, kScalArena + 1};
+#pragma unroll
+    for (int c = 0; c < kCNum; ++c)
+      if (acc.ctr[c]) atomicAdd(a.scal + slot[c], acc.ctr[c]);
   }
 }
 
@@ -2067,6 +2108,7 @@ __global__ void __launch_bounds__(256) decode_list_kernel(DevIndex ix, uint32_t 
 // Decode sweep: every block of the shard once (runs of D+2 blocks per warp).
 __global__ void __launch_bounds__(256) decode_all_kernel(DevIndex ix, uint32_t D, uint64_t nblocks,
                                                          unsigned long long *acc) {
+  // D = sweep_D(B): the launcher sizes shared memory for it
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
   WarpSmem w = carve_warp_smem(smem4, ix.B, D, false);   // no tile: XorSink
@@ -2156,7 +2198,7 @@ __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t 
   const uint32_t V = ix.num_terms, run = D + 2, B = ix.B;
   const uint64_t total = run_base[V];
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
-  unsigned long long alg = 0, pay = 0, post = 0;
+  unsigned long long alg = 0, pay = 0, post = 0, c8d = 0;
   for (uint64_t r = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); r < total;
        r += nwarps) {
     const uint32_t lo = run_term[r];
@@ -2171,12 +2213,14 @@ __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t 
       pay += p;
       post += n;
       alg += p + 8ull * nb + 4ull * n;
+      c8d += p + 8ull * nb;
     }
   }
   if (lane == 0) {
     if (alg) atomicAdd(scal + kScalDec + 0, alg);
     if (pay) atomicAdd(scal + kScalDec + 1, pay);
     if (post) atomicAdd(scal + kScalDec + 2, post);
+    if (c8d) atomicAdd(scal + kScalDecC8d, c8d);
   }
 }
 
@@ -2364,20 +2408,21 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     GRIFFIN_CUDA_TRY(w.runs.reserve((size_t)V * 4));
     GRIFFIN_CUDA_TRY(w.run_base.reserve(((size_t)V + 2) * 8));
     GRIFFIN_CUDA_TRY(w.vtmp.reserve(((size_t)V / kScanTile + 4) * 8));
-    GRIFFIN_CUDA_TRY(w.run_term.reserve((ix->nblocks / (ix->D + 2) + (size_t)V + 2) * 4));
+    const uint32_t Dsw = sweep_D(ix->B);
+    GRIFFIN_CUDA_TRY(w.run_term.reserve((ix->nblocks / (Dsw + 2) + (size_t)V + 2) * 4));
     GRIFFIN_CUDA_TRY(w.arena.reserve((ix->nblocks * ix->B + 64) * 4));
     GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.demand.p, 0, (size_t)V * 4, st));
     ra.T = ix->T;
     demand_kernel<<<qblocks, 256, 0, st>>>(di, ra, w.demand.as<uint32_t>());
     select_kernel<<<(V + 255) / 256, 256, 0, st>>>(di, w.demand.as<uint32_t>(),
                                                    w.tdec.as<uint8_t>(), w.runs.as<uint32_t>(),
-                                                   ix->D + 2);
+                                                   Dsw + 2);
     GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(w.runs.as<uint32_t>(), w.run_base.as<uint64_t>(), V,
                                               w.vtmp.as<uint64_t>(), st, &ix->launch_count));
     run_map_kernel<<<(uint32_t)(((uint64_t)V * 32 + 255) / 256), 256, 0, st>>>(V, w.runs.as<uint32_t>(),
                                                     w.run_base.as<uint64_t>(),
                                                     w.run_term.as<uint32_t>());
-    const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D, false) * 4 * 8;
+    const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, Dsw, false) * 4 * 8;
     static thread_local int cfg_dev = -1;
     static thread_local size_t cfg_smem = 0;
     if (cfg_dev != ix->device || cfg_smem < smem) {
@@ -2389,7 +2434,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, decode_once_kernel, 256, smem);
     decode_once_kernel<<<num_sms(ix->device) * std::max(1, per_sm), 256, smem, st>>>(
-        di, ix->D, w.run_base.as<uint64_t>(), w.run_term.as<uint32_t>(), w.arena.as<uint32_t>(),
+        di, Dsw, w.run_base.as<uint64_t>(), w.run_term.as<uint32_t>(), w.arena.as<uint32_t>(),
         scal);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
     ix->launch_count += 4;
@@ -2556,14 +2601,15 @@ griffin_status launch_decode_list(griffin_index *ix, uint32_t term, uint32_t *d_
 
 griffin_status launch_decode_all(griffin_index *ix, unsigned long long *d_acc, cudaStream_t st) {
   if (!ix->nblocks) return GRIFFIN_OK;
-  const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D, false) * 4 * 8;
+  const uint32_t Dsw = sweep_D(ix->B);
+  const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, Dsw, false) * 4 * 8;
   GRIFFIN_CUDA_TRY(cudaFuncSetAttribute(decode_all_kernel,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, decode_all_kernel, 256, smem);
   ix->launch_count += 1;
   decode_all_kernel<<<num_sms(ix->device) * std::max(1, per_sm), 256, smem, st>>>(
-      ix->dev(), ix->D, ix->nblocks, d_acc);
+      ix->dev(), Dsw, ix->nblocks, d_acc);
   GRIFFIN_CUDA_TRY(cudaGetLastError());
   return GRIFFIN_OK;
 }

@@ -6,7 +6,9 @@ method's arithmetic (no Elias-Fano coding, no intersection, no BM25, no top-k)
 and imports neither ``oracle`` nor the product package.
 """
 from .corpus import (Corpus, QueryLog, CONFIGS, make_corpus, make_queries,
-                     make_workload, make_pair_workload, make_ratio_groups, zipf_dfs)
+                     make_workload, make_pair_workload, make_ratio_groups, zipf_dfs,
+                     batch_of, cache_dir, sub_corpus)
 
 __all__ = ["Corpus", "QueryLog", "CONFIGS", "make_corpus", "make_queries",
-           "make_workload", "make_pair_workload", "make_ratio_groups", "zipf_dfs"]
+           "make_workload", "make_pair_workload", "make_ratio_groups", "zipf_dfs",
+           "batch_of", "cache_dir", "sub_corpus"]

@@ -10,10 +10,11 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import paper_conf_ppopp_0044ws18_b200 as g  # noqa: E402
-from synth import make_workload  # noqa: E402
+from synth import batch_of, make_workload  # noqa: E402
 
 cfg_name = sys.argv[1] if len(sys.argv) > 1 else "c2"
 c, ql, cfg = make_workload(cfg_name)
+ql = batch_of(ql, cfg, 0)
 k = cfg["k"]
 nq = ql.num_queries
 ix = g.GriffinIndex(c, block_size=int(os.environ.get("PROBE_B", cfg["block"])))
