@@ -25,6 +25,8 @@
 #include <algorithm>
 #include <cstdio>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "internal.h"
 #include "scan.cuh"
 
@@ -2275,12 +2277,18 @@ griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t
   return GRIFFIN_OK;
 }
 
+// Per-stage instrumentation: an NVTX range around the stage's host-side
+// launches (always; a no-op without an attached tool such as nsys/ncu
+// --nvtx), and, while profiling is on, CUDA events on the launching stream.
+static const char *const kStageNames[6] = {"griffin/plan", "griffin/intersect", "griffin/compact",
+                                           "griffin/topk", "griffin/merge", "griffin/decode_once"};
 struct StageTimer {
   griffin_index *ix;
   cudaStream_t st;
   int stage;
   cudaEvent_t a = nullptr, b = nullptr;
   StageTimer(griffin_index *ix_, cudaStream_t st_, int stage_) : ix(ix_), st(st_), stage(stage_) {
+    nvtxRangePushA(kStageNames[stage]);
     if (!ix->profiling) return;
     if (ix->ev_next + 2 > ix->ev_pool.size()) {
       for (int i = 0; i < 64; ++i) {
@@ -2294,6 +2302,7 @@ struct StageTimer {
     cudaEventRecord(a, st);
   }
   ~StageTimer() {
+    nvtxRangePop();
     if (!a) return;
     cudaEventRecord(b, st);
     ix->pending.push_back({stage, {a, b}});

@@ -186,9 +186,13 @@ def _term_list(t: int, num_docs: int, dfs: np.ndarray, seed: int,
     return lst
 
 
-# ---- parallel generation (fork workers; each term's streams depend only on
-# (seed, term), so the result is identical to the sequential loop) ----------
+# ---- parallel generation (spawned workers; each term's streams depend only
+# on (seed, term), so the result is identical to the sequential loop) --------
 _PAR = {}
+
+
+def _par_init(params):
+    _PAR.update(params)
 
 
 def _par_phase1(args):
@@ -240,13 +244,18 @@ def _make_corpus_parallel(num_docs, dfs, seed, planted, extra_lists, num_terms, 
         load[w] += size[t] + 64
     for a in assign:
         a.sort()
-    _PAR.update(num_docs=num_docs, dfs=dfs, seed=seed, planted=planted, extra=extra_lists)
+    params = dict(num_docs=num_docs, dfs=dfs, seed=seed, planted=planted, extra=extra_lists)
     tmpdir = os.path.join(outdir, "tmp")
     os.makedirs(tmpdir, exist_ok=True)
+    # fork: make_workload runs this in a fresh single-threaded interpreter
+    # (see _generate_into), so forking is safe; a dead worker raises
+    # BrokenProcessPool instead of hanging
+    from concurrent.futures import ProcessPoolExecutor
     ctx = mp.get_context("fork")
     lens = np.zeros(num_terms, np.uint64)
-    with ctx.Pool(workers) as pool:
-        for wid, ls in pool.imap_unordered(_par_phase1, [(w, assign[w], tmpdir) for w in range(workers)]):
+    with ProcessPoolExecutor(workers, mp_context=ctx, initializer=_par_init,
+                             initargs=(params,)) as pool:
+        for wid, ls in pool.map(_par_phase1, [(w, assign[w], tmpdir) for w in range(workers)]):
             lens[assign[wid]] = np.array(ls, np.uint64)
         offsets = np.zeros(num_terms + 1, dtype=np.uint64)
         np.cumsum(lens, out=offsets[1:])
@@ -254,9 +263,8 @@ def _make_corpus_parallel(num_docs, dfs, seed, planted, extra_lists, num_terms, 
         dpath, tpath = os.path.join(outdir, "docids.npy"), os.path.join(outdir, "tfs.npy")
         np.lib.format.open_memmap(dpath, mode="w+", dtype=np.uint32, shape=(P,)).flush()
         np.lib.format.open_memmap(tpath, mode="w+", dtype=np.uint32, shape=(P,)).flush()
-        list(pool.imap_unordered(_par_phase2, [(w, assign[w], tmpdir, offsets, dpath, tpath)
-                                               for w in range(workers)]))
-    _PAR.clear()
+        list(pool.map(_par_phase2, [(w, assign[w], tmpdir, offsets, dpath, tpath)
+                                    for w in range(workers)]))
     os.rmdir(tmpdir)
     return offsets
 
@@ -378,8 +386,7 @@ def make_workload(name: str, seed: Optional[int] = None, num_queries: Optional[i
                 if not os.path.exists(done):
                     os.makedirs(d, exist_ok=True)
                     nw = workers or min(32, os.cpu_count() or 1)
-                    make_corpus(cfg["num_docs"], dfs, seed, queries=ql,
-                                plant_fixed=cfg.get("plant_fixed"), outdir=d, workers=max(2, nw))
+                    _generate_into(d, name, seed, num_queries, overrides, max(2, nw))
                     open(done, "w").close()
             corpus = _load_corpus(d, cfg["num_docs"])
         except OSError:
@@ -404,6 +411,33 @@ def sub_corpus(c: Corpus, terms) -> Corpus:
     tfs = np.concatenate([np.asarray(c.tf_list(t)) for t in keep] or [np.zeros(0, np.uint32)])
     return Corpus(num_docs=c.num_docs, offsets=off, docids=docs.astype(np.uint32),
                   tfs=tfs.astype(np.uint32), doc_lengths=c.doc_lengths)
+
+
+def _generate_into(d, name, seed, num_queries, overrides, workers):
+    """Generate a workload's corpus into cache dir d in a fresh interpreter (the
+    caller may hold CUDA contexts and threads, which forked workers must not
+    inherit)."""
+    import subprocess
+    import sys
+    arg = json.dumps({"d": d, "name": name, "seed": seed, "num_queries": num_queries,
+                      "overrides": overrides, "workers": workers})
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    subprocess.run([sys.executable, "-c", "import sys, json; sys.path.insert(0, sys.argv[2]); "
+                    "from synth.corpus import _generate_main; _generate_main(json.loads(sys.argv[1]))",
+                    arg, root], check=True)
+
+
+def _generate_main(a):
+    cfg = dict(CONFIGS[a["name"]])
+    cfg.update(a["overrides"])
+    if a["num_queries"] is not None:
+        cfg["num_queries"] = a["num_queries"]
+    cfg.setdefault("batches", 1)
+    dfs = zipf_dfs(cfg["alpha"], cfg["df_max"], cfg["df_min"], cfg.get("num_terms"))
+    ql = make_queries(cfg["num_queries"] * cfg["batches"], len(dfs), a["seed"],
+                      beta=cfg.get("beta", 0.9))
+    make_corpus(cfg["num_docs"], dfs, a["seed"], queries=ql, plant_fixed=cfg.get("plant_fixed"),
+                outdir=a["d"], workers=a["workers"])
 
 
 def batch_of(ql: QueryLog, cfg, i: int) -> QueryLog:

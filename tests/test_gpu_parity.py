@@ -3,13 +3,15 @@
 Bar (BASELINE.json north_star): docID sets and top-k ordering bit-exact with ties
 by docID; BM25 scores within 1e-5 relative — in practice bit-identical, which is
 what these tests require (same f32 op order on both sides)."""
+import os
+
 import numpy as np
 import pytest
 
 import oracle
 import paper_conf_ppopp_0044ws18_b200 as g
 from helpers import corpus_from_lists, random_corpus, random_queries
-from synth import QueryLog, make_pair_workload, make_workload
+from synth import QueryLog, batch_of, make_pair_workload, make_workload, sub_corpus
 
 pytestmark = pytest.mark.gpu
 
@@ -277,46 +279,68 @@ def test_docid_sharding_merge_equals_unsharded(tiny, G):
 
 # ---------------------------------------------------------------- full size (bench config)
 
-@pytest.mark.slow
-def test_c2_full_size_sampled():
-    """BASELINE configs[1] at full size, in the launch configuration bench.py
-    times (one batch of all 1000 queries, device API): a sample of queries is
-    checked one by one against the oracle; the rest via invariants."""
+def _timed_config_run(c, batches, k, slots, steps):
+    """Run `steps` batches exactly as bench.py times them: device API, `slots`
+    workspaces (the index's own + extra ones) each on its own stream, batch i
+    on slot i % slots, rotating through `batches`; returns the host results of
+    every step's batch (keys -> rows) plus the index (for further checks)."""
     import torch
-    c, ql, cfg = make_workload("c2")
     gx = g.GriffinIndex(c, block_size=128)
-    k = cfg["k"]
-    nq = ql.num_queries
-    gx.griffin_reserve(ql.offsets, ql.terms, k)
-    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
-    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
-    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
-    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
-    cnt = torch.zeros(nq, dtype=torch.int32, device="cuda")
-    gx.griffin_query_batch_device(d_off, d_t, mt, k, keys, cnt, torch.cuda.current_stream())
-    dd = torch.zeros(nq * k, dtype=torch.int32, device="cuda")
-    ds = torch.zeros(nq * k, dtype=torch.float32, device="cuda")
-    gx.griffin_keys_to_results_device(nq, k, keys, cnt, dd, ds)
+    dq = []
+    for b in batches:
+        gx.griffin_reserve(b.offsets, b.terms, k)
+        mt = int(max(len(set(b.query(q).tolist())) for q in range(b.num_queries)))
+        dq.append((torch.from_numpy(b.offsets.astype(np.int32)).cuda(),
+                   torch.from_numpy(b.terms.astype(np.int32)).cuda(), mt))
+    nq = batches[0].num_queries
+    sl = [(None, torch.cuda.current_stream())]
+    for _ in range(slots - 1):
+        w = gx.griffin_workspace_create()
+        for b in batches:
+            w.griffin_workspace_reserve(b.offsets, b.terms, k)
+        sl.append((w, torch.cuda.Stream()))
+    outs = [(torch.zeros(nq * k, dtype=torch.int64, device="cuda"),
+             torch.zeros(nq, dtype=torch.int32, device="cuda")) for _ in range(steps)]
+    for i in range(steps):
+        w, st = sl[i % slots]
+        d_off, d_t, mt = dq[i % len(batches)]
+        kk, cc = outs[i]
+        if w is None:
+            gx.griffin_query_batch_device(d_off, d_t, mt, k, kk, cc, st)
+        else:
+            w.griffin_query_batch_device_ws(d_off, d_t, mt, k, kk, cc, st)
     torch.cuda.synchronize()
     gx.griffin_sync_status()
-    gd = dd.cpu().numpy().view(np.uint32).reshape(nq, k)
-    gs = ds.cpu().numpy().reshape(nq, k)
-    gc = cnt.cpu().numpy().view(np.uint32)
-    # invariants for every query: sorted by (score desc, docID asc); every docID
-    # is in all of the query's lists
-    for q in range(nq):
-        n = gc[q]
-        for i in range(1, n):
-            assert gs[q, i] < gs[q, i - 1] or (gs[q, i] == gs[q, i - 1] and gd[q, i] > gd[q, i - 1])
-        for t in set(ql.query(q).tolist()):
-            lst = c.list(t)
-            pos = np.searchsorted(lst, gd[q, :n])
-            assert np.all(lst[np.minimum(pos, len(lst) - 1)] == gd[q, :n])
+    for w, _ in sl[1:]:
+        w.griffin_workspace_sync_status()
+    res = []
+    for kk, cc in outs:
+        keys = kk.cpu().numpy().view(np.uint64).reshape(nq, k)
+        cnt = cc.cpu().numpy().view(np.uint32)
+        d = (np.uint64(0xFFFFFFFF) - (keys & np.uint64(0xFFFFFFFF))).astype(np.uint32)
+        sc = (keys >> np.uint64(32)).astype(np.uint32).view(np.float32)
+        valid = np.arange(k)[None, :] < cnt[:, None]
+        res.append((np.where(valid, d, np.uint32(0xFFFFFFFF)),
+                    np.where(valid, sc, np.float32(-np.inf)), cnt))
+    return gx, res
+
+
+@pytest.mark.slow
+def test_c2_full_size_all_queries_timed_config():
+    """BASELINE configs[1] at full size in the launch configuration bench.py
+    times for it (3 workspaces on 3 streams, rotating the config's 3 batches of
+    1000 queries): EVERY query of every batch bit-exact against the oracle."""
+    c, ql, cfg = make_workload("c2")
+    batches = [batch_of(ql, cfg, i) for i in range(cfg["batches"])]
+    k = cfg["k"]
+    gx, res = _timed_config_run(c, batches, k, slots=3, steps=6)
+    del gx
     ox = oracle.OracleIndex(c, block_size=128)
-    sample = np.random.default_rng(0).choice(nq, size=25, replace=False)
-    for q in sample:
-        od, os_, oc = ox.query(ql.query(q), k)
-        assert_topk_equal(gd[q], gs[q], gc[q], od, os_, oc)
+    for i, b in enumerate(batches):
+        od, os_, oc = ox.query_batch(b, k, nthreads=os.cpu_count() or 4)
+        for step in (i, i + 3):   # each batch ran twice, on different slots
+            gd, gs, gc = res[step]
+            assert_topk_equal(gd, gs, gc, od, os_, oc)
 
 
 def test_large_batch_s_locality_order():
@@ -345,68 +369,63 @@ def test_large_batch_s_locality_order():
                       cnt.cpu().numpy().view(np.uint32), od, os_, oc)
 
 
-def _sub_corpus(c, terms):
-    """The corpus with every list outside `terms` emptied: N, doc lengths (so
-    avgdl and every norm) and the kept lists (so their df and idf) are unchanged,
-    hence the oracle scores the sampled queries exactly as on the full corpus."""
-    from synth import Corpus
-    keep = np.zeros(c.num_terms, bool)
-    keep[list(terms)] = True
-    df = np.where(keep, c.df(), 0)
-    off = np.zeros(c.num_terms + 1, np.uint64)
-    off[1:] = np.cumsum(df)
-    docs = np.concatenate([c.list(t) for t in sorted(terms)] or [np.zeros(0, np.uint32)])
-    tfs = np.concatenate([c.tf_list(t) for t in sorted(terms)] or [np.zeros(0, np.uint32)])
-    return Corpus(num_docs=c.num_docs, offsets=off, docids=docs.astype(np.uint32),
-                  tfs=tfs.astype(np.uint32), doc_lengths=c.doc_lengths)
-
-
 @pytest.mark.slow
-def test_c5_full_size_sampled():
-    """BASELINE configs[4] at full size (50M docs, ~1.86 B postings, 10K queries,
-    top-1000) in the launch configuration of the C5 batch (one batch of all
-    queries, device API, decode-once reuse on): invariants on every query and 12
-    sampled queries bit-exact against the oracle (built over the sampled
-    queries' complete lists with the full corpus' N and doc lengths)."""
-    import torch
+def test_c5_full_size_timed_config():
+    """BASELINE configs[4] at full size (50M docs, ~1.9 B postings, 10K queries
+    per batch, top-1000) in bench.py's launch configuration (2 workspaces on 2
+    streams, rotating batches, decode-once reuse on): invariants on every query
+    of two batches and the first 1000 queries of batch 0 plus 200 of batch 1
+    bit-exact against the oracle (built over those queries' complete lists with
+    the full corpus' N and doc lengths, synth.sub_corpus)."""
     c, ql, cfg = make_workload("c5")
+    batches = [batch_of(ql, cfg, i) for i in range(2)]
     k = cfg["k"]
-    nq = ql.num_queries
-    gx = g.GriffinIndex(c, block_size=128)
-    gx.griffin_reserve(ql.offsets, ql.terms, k)
-    mt = int(max(len(set(ql.query(q).tolist())) for q in range(nq)))
-    d_off = torch.from_numpy(ql.offsets.astype(np.int32)).cuda()
-    d_t = torch.from_numpy(ql.terms.astype(np.int32)).cuda()
-    keys = torch.zeros(nq * k, dtype=torch.int64, device="cuda")
-    cnt = torch.zeros(nq, dtype=torch.int32, device="cuda")
-    gx.griffin_query_batch_device(d_off, d_t, mt, k, keys, cnt, torch.cuda.current_stream())
-    dd = torch.zeros(nq * k, dtype=torch.int32, device="cuda")
-    ds = torch.zeros(nq * k, dtype=torch.float32, device="cuda")
-    gx.griffin_keys_to_results_device(nq, k, keys, cnt, dd, ds)
-    torch.cuda.synchronize()
-    gx.griffin_sync_status()
+    gx, res = _timed_config_run(c, batches, k, slots=2, steps=2)
     del gx
-    gd = dd.cpu().numpy().view(np.uint32).reshape(nq, k)
-    gs = ds.cpu().numpy().reshape(nq, k)
-    gc = cnt.cpu().numpy().view(np.uint32)
-    assert gc.max() > 100, "the planted co-occurrences should give large results"
-    for q in range(nq):
-        n = gc[q]
-        s_, d_ = gs[q, :n], gd[q, :n]
-        assert np.all((s_[1:] < s_[:-1]) | ((s_[1:] == s_[:-1]) & (d_[1:] > d_[:-1])))
-        assert np.all(gd[q, n:] == 0xFFFFFFFF) and np.all(np.isneginf(gs[q, n:]))
-        for t in set(ql.query(q).tolist()):
-            lst = c.list(t)
-            pos = np.searchsorted(lst, d_)
-            assert np.all(lst[np.minimum(pos, len(lst) - 1)] == d_)
-    sample = np.random.default_rng(5).choice(nq, size=12, replace=False)
-    terms = set()
-    for q in sample:
-        terms |= set(ql.query(q).tolist())
-    ox = oracle.OracleIndex(_sub_corpus(c, terms), block_size=128)
-    for q in sample:
-        od, os_, oc = ox.query(ql.query(q), k)
-        assert_topk_equal(gd[q], gs[q], gc[q], od, os_, oc)
+    for (gd, gs, gc), b in zip(res, batches):
+        nq = b.num_queries
+        assert gc.max() > 100, "the planted co-occurrences should give large results"
+        for q in range(nq):
+            n = gc[q]
+            s_, d_ = gs[q, :n], gd[q, :n]
+            assert np.all((s_[1:] < s_[:-1]) | ((s_[1:] == s_[:-1]) & (d_[1:] > d_[:-1])))
+            assert np.all(gd[q, n:] == 0xFFFFFFFF) and np.all(np.isneginf(gs[q, n:]))
+    for (gd, gs, gc), b, m in zip(res, batches, (1000, 200)):
+        sub = b.slice(0, m)
+        ox = oracle.OracleIndex(sub_corpus(c, sub.terms), block_size=128)
+        od, os_, oc = ox.query_batch(sub, k, nthreads=os.cpu_count() or 4)
+        assert_topk_equal(gd[:m], gs[:m], gc[:m], od, os_, oc)
+        del ox
+
+
+@pytest.mark.parametrize("B", [64, 128])
+def test_large_tf_values_lossless(B):
+    """tf is stored losslessly (SURVEY A19): tf in {65535, 65536, 2^20, 2^32-1}
+    scores exactly as the oracle (no 16-bit clamp)."""
+    rng = np.random.default_rng(7)
+    N = 300_000
+    big = np.array([65535, 65536, 1 << 20, 0xFFFFFFFF, 1, 2], np.uint32)
+    lists, tfs = [], []
+    for t in range(6):
+        df = [500, 3000, 20000, 150, 80000, 7][t]
+        lst = np.sort(rng.choice(N, size=df, replace=False)).astype(np.uint32)
+        tf = rng.choice(big, size=df).astype(np.uint32)
+        lists.append(lst)
+        tfs.append(tf)
+    # shared docs so every query has results
+    common = np.sort(rng.choice(N, size=300, replace=False)).astype(np.uint32)
+    lists = [np.union1d(l, common).astype(np.uint32) for l in lists]
+    tfs = [rng.choice(big, size=len(l)).astype(np.uint32) for l in lists]
+    c = corpus_from_lists(N, lists, tfs, rng.integers(1, 5000, size=N).astype(np.uint32))
+    qs = [[0, 1], [1, 2], [0, 4], [2, 3, 4], [0, 1, 2, 3, 4], [5, 4], [4]]
+    ql = QueryLog(offsets=np.cumsum([0] + [len(q) for q in qs]).astype(np.uint32),
+                  terms=np.concatenate([np.array(q, np.uint32) for q in qs]))
+    gx = g.GriffinIndex(c, block_size=B)
+    ox = oracle.OracleIndex(c, block_size=B)
+    for k in (10, 400):
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+        od, os_, oc = ox.query_batch(ql, k)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
 
 
 @pytest.mark.slow
