@@ -235,6 +235,8 @@ griffin_status griffin_keys_to_results_device(griffin_index *ix, uint32_t nq, ui
 
 /* ---- configuration / instrumentation ---------------------------------------- */
 griffin_status griffin_set_mode(griffin_index *ix, int mode); /* griffin_mode; default AUTO */
+/* 0 off; 1 per-stage CUDA events + algorithmic-byte counters; 2 events only
+ * (kernel durations without the counting work); 3 counters only. */
 griffin_status griffin_set_profiling(griffin_index *ix, int on);
 /* Batch list reuse: 0 = off (every round decodes its blocks, fused), 1 = on,
  * 2 = auto (default; on for batches of >= 8 queries).  When on, lists whose

@@ -383,7 +383,8 @@ class GriffinIndex:
         """Probe-pass survivors per unit (multiple of 32 in [32, B]; 0 = B)."""
         _check(load_library().griffin_set_probe_chunk(self.h, chunk))
 
-    def griffin_set_profiling(self, on: bool):
+    def griffin_set_profiling(self, on):
+        """False/0 off, True/1 events + counters, 2 events only, 3 counters only."""
         _check(load_library().griffin_set_profiling(self.h, int(on)))
 
     def griffin_get_profile(self) -> dict:

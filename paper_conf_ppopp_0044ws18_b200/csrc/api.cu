@@ -197,6 +197,8 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   ix->D = std::max<uint32_t>(2, 1024 / B);
   if (const char *e = std::getenv("GRIFFIN_TUNE_D")) ix->D = std::max<uint32_t>(2, (uint32_t)std::atoi(e));  // A/B probes
   if (const char *e = std::getenv("GRIFFIN_TOPK_FILTER")) ix->topk_filter = std::atoi(e);  // A/B
+  if (const char *e = std::getenv("GRIFFIN_TDEC")) ix->Tdec = std::max(1, std::atoi(e));  // A/B
+  if (const char *e = std::getenv("GRIFFIN_T")) ix->T = std::max(1, std::atoi(e));        // A/B
   if (const char *e = std::getenv("GRIFFIN_SORDER")) {   // A/B probes: 0 = off, else 1 + shift
     const int v = std::atoi(e);
     ix->sorder = v > 0;
@@ -766,7 +768,8 @@ griffin_status griffin_set_probe_chunk(griffin_index *ix, uint32_t chunk) {
 griffin_status griffin_set_profiling(griffin_index *ix, int on) {
   if (!ix) return invalid("null index");
   std::lock_guard<std::mutex> lk(ix->mu);
-  ix->profiling = on != 0;
+  if (on < 0 || on > 3) return invalid("profiling must be 0 (off), 1 (events + counters), 2 (events) or 3 (counters)");
+  ix->profiling = on == 1 ? 3 : on == 2 ? 1 : on == 3 ? 2 : 0;
   return GRIFFIN_OK;
 }
 

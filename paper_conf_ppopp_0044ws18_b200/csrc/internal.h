@@ -101,6 +101,7 @@ struct RoundArgs {
   int forced_mode;
   int probe;
   int nextgeq;   // gallop into compressed S by EF NextGEQ (no block decode)
+  int count;     // maintain the algorithmic-byte / postings counters (profiling)
   uint32_t pchunk;   // probe pass: survivors per unit (multiple of 32, <= B)
   const uint32_t *plan_terms;
   const uint32_t *plan_m;
@@ -169,7 +170,7 @@ struct griffin_index {
   int sorder = 1;   // merge units ordered by the S blocks they read (L2 reuse across queries)
   uint32_t sorder_shift = 6;
   uint32_t P = 0;   // probe chunk (0 = B)
-  bool profiling = false;
+  int profiling = 0;   // bit 0: per-stage CUDA events, bit 1: algorithmic-byte counters
   griffin_profile prof{};
   std::vector<cudaEvent_t> ev_pool;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending;  // stage, events

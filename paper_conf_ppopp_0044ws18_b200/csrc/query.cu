@@ -1210,8 +1210,8 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
       const uint32_t totR16 = __reduce_add_sync(0xffffffffu, (lm && isR) ? sz : 0u);
       const uint32_t totS16 = __reduce_add_sync(0xffffffffu, (lm && isS) ? sz : 0u);
       const uint32_t soff = isR ? m.x - mR0 : (isS ? totR16 + (m.x - mS0) : 0u);
-      // ---- accounting: blocks whose head lies in this unit ----
-      {
+      // ---- accounting: blocks whose head lies in this unit (profiling) ----
+      if (a.count) {
         const bool own = (isR && rb0 + lane >= i0) || (isS && sb0 + (lane - nRb) >= j0);
         const uint32_t nn = isR ? min(B, nR - (rb0 + lane) * B)
                                 : (isS ? min(B, tS.df_local - (sb0 + lane - nRb) * B) : 0u);
@@ -2289,7 +2289,7 @@ struct StageTimer {
   cudaEvent_t a = nullptr, b = nullptr;
   StageTimer(griffin_index *ix_, cudaStream_t st_, int stage_) : ix(ix_), st(st_), stage(stage_) {
     nvtxRangePushA(kStageNames[stage]);
-    if (!ix->profiling) return;
+    if (!(ix->profiling & 1)) return;
     if (ix->ev_next + 2 > ix->ev_pool.size()) {
       for (int i = 0; i < 64; ++i) {
         cudaEvent_t e;
@@ -2453,6 +2453,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
   // multi-list probe replaces SvS rounds 2..m-1 (auto mode, B small enough for its smem)
   ra.probe = forced_mode == 0 && ix->probe && ix->D >= 5;
   ra.nextgeq = ix->nextgeq;
+  ra.count = (ix->profiling & 2) ? 1 : 0;
   ra.pchunk = probe_chunk(ix);
   uint32_t rounds = std::max<uint32_t>(1, max_terms > 0 ? max_terms - 1 : 1);
   if (ra.probe) rounds = std::min<uint32_t>(rounds, 2);
