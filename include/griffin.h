@@ -54,7 +54,7 @@ typedef enum {
   GRIFFIN_ERR_UNSORTED = 2,    /* a list not strictly increasing or a docID >= N */
   GRIFFIN_ERR_OOM = 3,         /* device allocation failed / workspace too small */
   GRIFFIN_ERR_CUDA = 4,        /* CUDA runtime error (message in griffin_last_error) */
-  GRIFFIN_ERR_NCCL = 5,        /* reserved: collective failure reported by a caller */
+  GRIFFIN_ERR_NCCL = 5,        /* NCCL missing or a collective failed (multi-GPU handles) */
   GRIFFIN_ERR_UNSUPPORTED = 6  /* no CUDA device / not sm_100 */
 } griffin_status;
 
@@ -86,7 +86,40 @@ typedef struct {
                                     arena (griffin_set_reuse): galloping there costs ~log2(B)
                                     probes per R element instead of a block decode, so the
                                     crossover is lower; 0 -> max(4, block_size/8) */
+  /* ---- one handle over several GPUs ----
+   * num_gpus G > 1: the handle builds G docID-range shards itself (shard g owns
+   * [g*ceil(N/G), min(N,(g+1)*ceil(N/G))), global N/df/avgdl/idf everywhere, so
+   * each doc's score is bit-identical to the unsharded one) on devices[g]
+   * (NULL -> 0..G-1), owns their streams and NCCL communicators, and
+   * griffin_query / griffin_query_batch return the GLOBAL top-k: per-shard top-k
+   * keys are exchanged and k-way merged on the devices (exact: keys are unique,
+   * so a global top-k key is in its shard's top-k).  num_shards must then be 0/1.
+   * INVALID_ARG if G > 8 or a device ordinal is >= the visible device count;
+   * GRIFFIN_ERR_NCCL if an NCCL exchange is requested and NCCL (libnccl.so.2,
+   * loaded at run time) is missing or fails.  Devices may repeat (several
+   * shards on one GPU), which only the peer exchange supports. */
+  uint32_t num_gpus;       /* 0/1 -> a single shard (unless exchange != 0) */
+  const int32_t *devices;  /* [num_gpus] device ordinals, borrowed for the call; NULL -> 0..G-1 */
+  int32_t exchange;        /* griffin_exchange: how per-shard top-k lists meet */
 } griffin_build_opts;
+
+/* Exchange of per-shard top-k lists for a multi-GPU handle.
+ *  AUTO: PEER.  NCCL_ALLGATHER: ncclAllGather of every shard's keys/counts (one
+ *  NCCL group, one communicator per device), then the k-way merge on device 0.
+ *  PEER: one kernel on device 0 reads every shard's top-k runs in place over
+ *  NVLink (cudaDeviceEnablePeerAccess; copied with cudaMemcpyPeerAsync when
+ *  peer access is unavailable) and merges them — exchange and merge fused.
+ *  NCCL_SLICED: query-sliced all-to-all (grouped ncclSend/ncclRecv): device r
+ *  receives only the runs of query slice r and merges it (received bytes per
+ *  device ~ Q*k*8 instead of (G-1)*Q*k*8).
+ *  With num_gpus = 1, exchange != AUTO still builds a one-shard handle that runs
+ *  the chosen exchange (a one-rank NCCL communicator for the NCCL modes). */
+typedef enum {
+  GRIFFIN_EXCHANGE_AUTO = 0,
+  GRIFFIN_EXCHANGE_NCCL_ALLGATHER = 1,
+  GRIFFIN_EXCHANGE_PEER = 2,
+  GRIFFIN_EXCHANGE_NCCL_SLICED = 3
+} griffin_exchange;
 
 typedef struct {
   uint32_t shard_index, num_shards;

@@ -27,6 +27,7 @@ STATUS = {0: "GRIFFIN_OK", 1: "GRIFFIN_ERR_INVALID_ARG", 2: "GRIFFIN_ERR_UNSORTE
           3: "GRIFFIN_ERR_OOM", 4: "GRIFFIN_ERR_CUDA", 5: "GRIFFIN_ERR_NCCL",
           6: "GRIFFIN_ERR_UNSUPPORTED"}
 MODE_AUTO, MODE_MERGE, MODE_GALLOP = 0, 1, 2
+EXCHANGE_AUTO, EXCHANGE_NCCL_ALLGATHER, EXCHANGE_PEER, EXCHANGE_NCCL_SLICED = 0, 1, 2, 3
 MAX_TERMS, MAX_K = 16, 4096
 
 
@@ -46,7 +47,9 @@ class _Opts(ctypes.Structure):
     _fields_ = [("block_size", ctypes.c_uint32), ("bm25_k1", ctypes.c_double),
                 ("bm25_b", ctypes.c_double), ("gallop_ratio", ctypes.c_uint32),
                 ("device", ctypes.c_int32), ("shard_index", ctypes.c_uint32),
-                ("num_shards", ctypes.c_uint32), ("gallop_ratio_decoded", ctypes.c_uint32)]
+                ("num_shards", ctypes.c_uint32), ("gallop_ratio_decoded", ctypes.c_uint32),
+                ("num_gpus", ctypes.c_uint32), ("devices", ctypes.c_void_p),
+                ("exchange", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -261,11 +264,14 @@ def griffin_merge_path_split(a, b, diag: int, fixup: bool = True) -> Tuple[int, 
 
 
 class GriffinIndex:
-    """Owns one `griffin_index` (one docID-range shard on one device)."""
+    """Owns one `griffin_index`: one docID-range shard on one device, or with
+    num_gpus > 1 (or an explicit exchange) a handle over num_gpus shards on
+    `devices` whose queries return the global top-k (include/griffin.h)."""
 
     def __init__(self, corpus, block_size: int = 128, k1: float = 1.2, b: float = 0.75,
                  gallop_ratio: int = 0, device: int = -1, shard_index: int = 0,
-                 num_shards: int = 1, gallop_ratio_decoded: int = 0):
+                 num_shards: int = 1, gallop_ratio_decoded: int = 0, num_gpus: int = 1,
+                 devices=None, exchange: int = EXCHANGE_AUTO):
         lib = load_library()
         self._arrays = [np.ascontiguousarray(corpus.offsets, np.uint64),
                         np.ascontiguousarray(corpus.docids, np.uint32),
@@ -274,8 +280,10 @@ class GriffinIndex:
         off, doc, tf, dl = self._arrays
         c = _Corpus(corpus.num_docs, len(off) - 1, off.ctypes.data, doc.ctypes.data,
                     tf.ctypes.data, dl.ctypes.data)
+        devs = None if devices is None else np.ascontiguousarray(devices, np.int32)
         o = _Opts(block_size, k1, b, gallop_ratio, device, shard_index, num_shards,
-                  gallop_ratio_decoded)
+                  gallop_ratio_decoded, num_gpus, devs.ctypes.data if devs is not None else None,
+                  exchange)
         h = ctypes.c_void_p()
         status = lib.griffin_index_build(ctypes.byref(c), ctypes.byref(o), ctypes.byref(h))
         self._arrays = None
@@ -554,4 +562,5 @@ class GriffinPfd:
 
 __all__ = ["GriffinIndex", "GriffinWorkspace", "GriffinPfd", "GriffinError", "load_library", "griffin_last_error",
            "griffin_shard_range", "griffin_merge_path_split", "MODE_AUTO", "MODE_MERGE",
-           "MODE_GALLOP", "LIB_PATH"]
+           "MODE_GALLOP", "EXCHANGE_AUTO", "EXCHANGE_NCCL_ALLGATHER", "EXCHANGE_PEER",
+           "EXCHANGE_NCCL_SLICED", "LIB_PATH"]

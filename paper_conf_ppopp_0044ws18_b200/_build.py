@@ -8,7 +8,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libgriffin.so")
-SOURCES = ["api.cu", "encode.cu", "query.cu", "pfd.cu"]
+SOURCES = ["api.cu", "encode.cu", "query.cu", "pfd.cu", "multi.cu"]
 HEADERS = ["griffin_dev.cuh", "internal.h", "scan.cuh"]
 ROOT = os.path.dirname(HERE)
 PUBLIC_HEADER = os.path.join(ROOT, "include", "griffin.h")

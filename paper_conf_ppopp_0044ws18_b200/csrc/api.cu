@@ -16,25 +16,18 @@ namespace griffin {
 static thread_local std::string g_err;
 void set_error(const std::string &msg) { g_err = msg; }
 
-struct DeviceGuard {
-  int prev = -1;
-  explicit DeviceGuard(int dev) {
-    cudaGetDevice(&prev);
-    if (prev != dev) cudaSetDevice(dev);
-  }
-  ~DeviceGuard() {
-    int cur = -1;
-    cudaGetDevice(&cur);
-    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
-  }
-};
 
 static griffin_status invalid(const std::string &m) {
   set_error(m);
   return GRIFFIN_ERR_INVALID_ARG;
 }
 
-static griffin_status ensure_pinned_ws(Workspace &w, size_t bytes) {
+static griffin_status multi_unsupported() {
+  set_error("not available on a multi-GPU handle (num_gpus > 1): use griffin_query / griffin_query_batch");
+  return GRIFFIN_ERR_UNSUPPORTED;
+}
+
+griffin_status ensure_pinned_ws(Workspace &w, size_t bytes) {
   if (w.h_pinned_bytes >= bytes) return GRIFFIN_OK;
   if (w.h_pinned) w.old_pinned.push_back(w.h_pinned);   // freed with the workspace
   w.h_pinned = nullptr;
@@ -49,9 +42,9 @@ static griffin_status ensure_pinned(griffin_index *ix, size_t bytes) {
 }
 
 // Host validation of one batch's query terms + workspace reservation.
-static griffin_status reserve_for(griffin_index *ix, Workspace &w, uint32_t nq,
-                                  const uint32_t *qoffs, const uint32_t *terms, uint32_t k,
-                                  uint32_t *max_terms) {
+griffin_status reserve_for(griffin_index *ix, Workspace &w, uint32_t nq,
+                           const uint32_t *qoffs, const uint32_t *terms, uint32_t k,
+                           uint32_t *max_terms) {
   if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
   uint64_t caps = 0, units = 0;
   uint32_t mt = 1;
@@ -129,23 +122,8 @@ griffin_status griffin_merge_path_split(const uint32_t *a, uint32_t na, const ui
   return GRIFFIN_OK;
 }
 
-griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_opts *o,
-                                   griffin_index **out) {
-  if (!c || !out) return invalid("null corpus/out");
-  *out = nullptr;
-  griffin_build_opts opts{};
-  if (o) {
-    opts = *o;
-  } else {   // NULL: every documented default (b = 0.75, the current device)
-    opts.bm25_b = -1.0;
-    opts.device = -1;
-  }
-  const uint32_t B = opts.block_size ? opts.block_size : 128;
-  if (B < 64 || B > 512 || (B % 32)) return invalid("block_size must be 64..512 and a multiple of 32");
-  const double k1 = opts.bm25_k1 > 0 ? opts.bm25_k1 : 1.2;
-  const double bb = opts.bm25_b >= 0 ? opts.bm25_b : 0.75;
-  const uint32_t G = opts.num_shards ? opts.num_shards : 1;
-  if (G > GRIFFIN_MAX_SHARDS || opts.shard_index >= G) return invalid("bad shard index / count");
+// Host validation of a corpus (once per build, also for G shards).
+static griffin_status validate_corpus(const griffin_corpus *c, uint64_t *sum_dl_out) {
   const uint32_t N = c->num_docs, V = c->num_terms;
   if (N == 0 || N >= 0xFFFFFFFFu) return invalid("num_docs must be in [1, 2^32-2]");
   if (!c->list_offsets || !c->doc_lengths) return invalid("null corpus arrays");
@@ -168,15 +146,17 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   uint64_t sum_dl = 0;
   for (uint32_t d = 0; d < N; ++d) sum_dl += c->doc_lengths[d];
   if (sum_dl == 0) return invalid("sum of doc_lengths must be > 0");
+  *sum_dl_out = sum_dl;
+  return GRIFFIN_OK;
+}
 
+static griffin_status check_device(int dev) {
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
     set_error("no CUDA device");
     return GRIFFIN_ERR_UNSUPPORTED;
   }
-  int dev = opts.device;
-  if (dev < 0) cudaGetDevice(&dev);
-  if (dev >= ndev) return invalid("device ordinal out of range");
+  if (dev < 0 || dev >= ndev) return invalid("device ordinal out of range");
   cudaDeviceProp prop;
   GRIFFIN_CUDA_TRY(cudaGetDeviceProperties(&prop, dev));
   if (prop.major != 10 || prop.minor != 0) {
@@ -184,8 +164,18 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
               std::to_string(prop.minor));
     return GRIFFIN_ERR_UNSUPPORTED;
   }
-  DeviceGuard guard(dev);
+  return GRIFFIN_OK;
+}
 
+// One docID-range shard (g of G) of a validated corpus on device `dev`.
+static griffin_status build_shard(const griffin_corpus *c, const griffin_build_opts &opts,
+                                  uint64_t sum_dl, uint32_t G, uint32_t g, int dev,
+                                  griffin_index **out) {
+  const uint32_t B = opts.block_size ? opts.block_size : 128;
+  const double k1 = opts.bm25_k1 > 0 ? opts.bm25_k1 : 1.2;
+  const double bb = opts.bm25_b >= 0 ? opts.bm25_b : 0.75;
+  const uint32_t N = c->num_docs, V = c->num_terms;
+  DeviceGuard guard(dev);
   griffin_index *ix = new griffin_index();
   ix->device = dev;
   ix->B = B;
@@ -208,9 +198,9 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   ix->bm25_b = bb;
   ix->N = N;
   ix->V = V;
-  ix->shard = opts.shard_index;
+  ix->shard = g;
   ix->nshards = G;
-  griffin_shard_range(N, G, opts.shard_index, &ix->doc_base, &ix->doc_end);
+  griffin_shard_range(N, G, g, &ix->doc_base, &ix->doc_end);
   ix->k1p1 = (float)(k1 + 1.0);
   if (cudaStreamCreateWithFlags(&ix->stream, cudaStreamNonBlocking) != cudaSuccess) {
     delete ix;
@@ -267,10 +257,80 @@ griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_
   return GRIFFIN_OK;
 }
 
+griffin_status griffin_index_build(const griffin_corpus *c, const griffin_build_opts *o,
+                                   griffin_index **out) {
+  if (!c || !out) return invalid("null corpus/out");
+  *out = nullptr;
+  griffin_build_opts opts{};
+  if (o) {
+    opts = *o;
+  } else {   // NULL: every documented default (b = 0.75, the current device)
+    opts.bm25_b = -1.0;
+    opts.device = -1;
+  }
+  const uint32_t B = opts.block_size ? opts.block_size : 128;
+  if (B < 64 || B > 512 || (B % 32)) return invalid("block_size must be 64..512 and a multiple of 32");
+  const uint32_t NG = opts.num_gpus ? opts.num_gpus : 1;
+  if (NG > GRIFFIN_MAX_SHARDS) return invalid("num_gpus must be in [1, 8]");
+  if (opts.exchange < 0 || opts.exchange > 3) return invalid("exchange must be 0..3");
+  const uint32_t G = opts.num_shards ? opts.num_shards : 1;
+  if (G > GRIFFIN_MAX_SHARDS || opts.shard_index >= G) return invalid("bad shard index / count");
+  const bool multi = NG > 1 || opts.exchange != 0;
+  if (multi && G > 1) return invalid("num_gpus > 1 builds every shard itself (num_shards must be 0/1)");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    set_error("no CUDA device");
+    return GRIFFIN_ERR_UNSUPPORTED;
+  }
+  std::vector<int> devs(NG);
+  for (uint32_t g = 0; g < NG; ++g) {
+    int d = opts.devices ? opts.devices[g] : (NG > 1 ? (int)g : opts.device);
+    if (d < 0) cudaGetDevice(&d);
+    if (d >= ndev) return invalid(NG > 1 ? "num_gpus > visible devices (or a device ordinal out of range)"
+                                         : "device ordinal out of range");
+    griffin_status s = check_device(d);
+    if (s) return s;
+    devs[g] = d;
+  }
+  uint64_t sum_dl = 0;
+  griffin_status s = validate_corpus(c, &sum_dl);
+  if (s) return s;
+  if (!multi) return build_shard(c, opts, sum_dl, G, opts.shard_index, devs[0], out);
+  // num_gpus > 1: one handle over NG docID-range shards
+  griffin_index *cx = new griffin_index();
+  cx->device = devs[0];
+  cx->B = B;
+  cx->N = c->num_docs;
+  cx->V = c->num_terms;
+  cx->nshards = NG;
+  cx->doc_base = 0;
+  cx->doc_end = c->num_docs;
+  for (uint32_t g = 0; g < NG; ++g) {
+    griffin_index *sh = nullptr;
+    if ((s = build_shard(c, opts, sum_dl, NG, g, devs[g], &sh))) {
+      griffin_index_destroy(cx);
+      return s;
+    }
+    cx->shards.push_back(sh);
+  }
+  if ((s = cluster_init(cx, opts.exchange))) {
+    griffin_index_destroy(cx);
+    return s;
+  }
+  *out = cx;
+  return GRIFFIN_OK;
+}
+
 static void free_workspace(Workspace &w);
 
 void griffin_index_destroy(griffin_index *ix) {
   if (!ix) return;
+  if (ix->cl || !ix->shards.empty()) {   // multi-GPU handle
+    cluster_destroy(ix);
+    for (griffin_index *sh : ix->shards) griffin_index_destroy(sh);
+    delete ix;
+    return;
+  }
   {
     DeviceGuard guard(ix->device);
     if (ix->stream) cudaStreamSynchronize(ix->stream);
@@ -296,6 +356,25 @@ void griffin_index_destroy(griffin_index *ix) {
 griffin_status griffin_index_stats(const griffin_index *ix, griffin_stats *out) {
   if (!ix || !out) return invalid("null argument");
   std::memset(out, 0, sizeof(*out));
+  if (ix->cl) {   // multi-GPU handle: totals over its shards
+    for (const griffin_index *sh : ix->shards) {
+      griffin_stats t;
+      griffin_index_stats(sh, &t);
+      out->num_postings += t.num_postings;
+      out->num_blocks += t.num_blocks;
+      out->payload_bytes += t.payload_bytes;
+      out->skip_bytes += t.skip_bytes;
+      out->tf_bytes += t.tf_bytes;
+      out->device_bytes += t.device_bytes;
+    }
+    out->shard_index = 0;
+    out->num_shards = (uint32_t)ix->shards.size();
+    out->doc_base = 0;
+    out->doc_end = ix->N;
+    out->block_size = ix->B;
+    out->num_terms = ix->V;
+    return GRIFFIN_OK;
+  }
   out->shard_index = ix->shard;
   out->num_shards = ix->nshards;
   out->doc_base = ix->doc_base;
@@ -318,6 +397,7 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
   if (!ix) return invalid("null index");
   if (nq == 0) return GRIFFIN_OK;
   if (!qoffs || !terms || !out_docids || !out_scores || !out_counts) return invalid("null argument");
+  if (ix->cl) return cluster_query_batch(ix, nq, qoffs, terms, k, out_docids, out_scores, out_counts);
   std::lock_guard<std::mutex> lk(ix->mu);
   if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
   ix->ws.results_valid = false;
@@ -466,7 +546,7 @@ griffin_status griffin_query(griffin_index *ix, const uint32_t *terms, uint32_t 
                              uint32_t *out_docids, float *out_scores, uint32_t *out_count) {
   if (nterms == 0) return invalid("nterms must be > 0");
   if (!ix || !terms || !out_docids || !out_scores || !out_count) return invalid("null argument");
-  if (ix->use_graphs && !ix->profiling) {
+  if (ix->use_graphs && !ix->profiling && !ix->cl) {
     std::lock_guard<std::mutex> lk(ix->mu);
     if (ix->ws.pending) return invalid("the index's workspace holds a submitted batch not yet collected");
     ix->ws.results_valid = false;
@@ -480,6 +560,7 @@ griffin_status griffin_query(griffin_index *ix, const uint32_t *terms, uint32_t 
 
 griffin_status griffin_reserve(griffin_index *ix, uint32_t nq, const uint32_t *qoffs,
                                const uint32_t *terms, uint32_t k) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix || (nq && (!qoffs || !terms))) return invalid("null argument");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -490,6 +571,7 @@ griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq, const 
                                           const uint32_t *d_terms, uint32_t max_terms, uint32_t k,
                                           uint64_t *d_out_keys, uint32_t *d_out_counts,
                                           void *stream) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix) return invalid("null index");
   if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
   if (max_terms == 0 || max_terms > GRIFFIN_MAX_TERMS) return invalid("max_terms out of range");
@@ -503,6 +585,7 @@ griffin_status griffin_query_batch_device(griffin_index *ix, uint32_t nq, const 
 }
 
 griffin_status griffin_sync_status(griffin_index *ix) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix) return invalid("null index");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -512,6 +595,7 @@ griffin_status griffin_sync_status(griffin_index *ix) {
 }
 
 griffin_status griffin_workspace_create(griffin_index *ix, griffin_workspace **out) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix || !out) return invalid("null argument");
   std::lock_guard<std::mutex> lk(ix->mu);
   Workspace *w = new Workspace();
@@ -590,6 +674,7 @@ griffin_status griffin_workspace_sync_status(griffin_index *ix, griffin_workspac
 griffin_status griffin_query_batch_submit(griffin_index *ix, griffin_workspace *ws, uint32_t nq,
                                           const uint32_t *qoffs, const uint32_t *terms,
                                           uint32_t k, void *stream) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix) return invalid("null index");
   if (nq && (!qoffs || !terms)) return invalid("null argument");
   Workspace &w = ws ? *reinterpret_cast<Workspace *>(ws) : ix->ws;
@@ -708,6 +793,7 @@ griffin_status griffin_merge_topk_device(griffin_index *ix, uint32_t num_runs, u
                                          uint32_t k, const uint64_t *d_keys,
                                          const uint32_t *d_counts, uint64_t *d_out_keys,
                                          uint32_t *d_out_counts, void *stream) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix) return invalid("null index");
   if (num_runs == 0 || num_runs > 32) return invalid("num_runs must be in [1, 32]");
   if (k == 0 || k > GRIFFIN_MAX_K) return invalid("k must be in [1, 4096]");
@@ -720,6 +806,7 @@ griffin_status griffin_merge_topk_device(griffin_index *ix, uint32_t num_runs, u
 griffin_status griffin_keys_to_results_device(griffin_index *ix, uint32_t nq, uint32_t k,
                                               const uint64_t *d_keys, const uint32_t *d_counts,
                                               uint32_t *d_docids, float *d_scores, void *stream) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix) return invalid("null index");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -728,6 +815,13 @@ griffin_status griffin_keys_to_results_device(griffin_index *ix, uint32_t nq, ui
 }
 
 griffin_status griffin_set_mode(griffin_index *ix, int mode) {
+  if (ix && ix->cl) {   // multi-GPU handle: every shard
+    for (griffin_index *sh : ix->shards) {
+      griffin_status s = griffin_set_mode(sh, mode);
+      if (s) return s;
+    }
+    return GRIFFIN_OK;
+  }
   if (!ix || mode < 0 || mode > 2) return invalid("mode must be 0 (auto), 1 (merge) or 2 (gallop)");
   std::lock_guard<std::mutex> lk(ix->mu);
   ix->mode = mode;
@@ -735,6 +829,13 @@ griffin_status griffin_set_mode(griffin_index *ix, int mode) {
 }
 
 griffin_status griffin_set_reuse(griffin_index *ix, int mode) {
+  if (ix && ix->cl) {   // multi-GPU handle: every shard
+    for (griffin_index *sh : ix->shards) {
+      griffin_status s = griffin_set_reuse(sh, mode);
+      if (s) return s;
+    }
+    return GRIFFIN_OK;
+  }
   if (!ix || mode < 0 || mode > 2) return invalid("reuse must be 0 (off), 1 (on) or 2 (auto)");
   std::lock_guard<std::mutex> lk(ix->mu);
   ix->reuse = mode;
@@ -742,6 +843,13 @@ griffin_status griffin_set_reuse(griffin_index *ix, int mode) {
 }
 
 griffin_status griffin_set_nextgeq(griffin_index *ix, int on) {
+  if (ix && ix->cl) {   // multi-GPU handle: every shard
+    for (griffin_index *sh : ix->shards) {
+      griffin_status s = griffin_set_nextgeq(sh, on);
+      if (s) return s;
+    }
+    return GRIFFIN_OK;
+  }
   if (!ix || on < 0 || on > 1) return invalid("nextgeq must be 0 or 1");
   std::lock_guard<std::mutex> lk(ix->mu);
   if (ix->nextgeq != on) {   // captured single-query graphs bake the option in
@@ -753,6 +861,13 @@ griffin_status griffin_set_nextgeq(griffin_index *ix, int on) {
 }
 
 griffin_status griffin_set_probe_chunk(griffin_index *ix, uint32_t chunk) {
+  if (ix && ix->cl) {   // multi-GPU handle: every shard
+    for (griffin_index *sh : ix->shards) {
+      griffin_status s = griffin_set_probe_chunk(sh, chunk);
+      if (s) return s;
+    }
+    return GRIFFIN_OK;
+  }
   if (!ix) return invalid("null index");
   if (chunk != 0 && (chunk < 32 || chunk > ix->B || chunk % 32 != 0))
     return invalid("probe chunk must be 0 or a multiple of 32 in [32, block_size]");
@@ -766,6 +881,13 @@ griffin_status griffin_set_probe_chunk(griffin_index *ix, uint32_t chunk) {
 }
 
 griffin_status griffin_set_profiling(griffin_index *ix, int on) {
+  if (ix && ix->cl) {   // multi-GPU handle: every shard
+    for (griffin_index *sh : ix->shards) {
+      griffin_status s = griffin_set_profiling(sh, on);
+      if (s) return s;
+    }
+    return GRIFFIN_OK;
+  }
   if (!ix) return invalid("null index");
   std::lock_guard<std::mutex> lk(ix->mu);
   if (on < 0 || on > 3) return invalid("profiling must be 0 (off), 1 (events + counters), 2 (events) or 3 (counters)");
@@ -774,6 +896,7 @@ griffin_status griffin_set_profiling(griffin_index *ix, int on) {
 }
 
 griffin_status griffin_reset_profile(griffin_index *ix) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix) return invalid("null index");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -794,6 +917,7 @@ griffin_status griffin_reset_profile(griffin_index *ix) {
 }
 
 griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix || !out) return invalid("null argument");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -840,6 +964,7 @@ griffin_status griffin_debug_block_streams(griffin_index *ix, uint32_t term, uin
                                            uint32_t *first, uint32_t *n, uint32_t *b,
                                            uint32_t *low, uint64_t low_cap, uint64_t *low_bits,
                                            uint32_t *high, uint64_t high_cap, uint64_t *high_bits) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix || term >= ix->V) return invalid("bad term");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -884,6 +1009,7 @@ griffin_status griffin_debug_block_streams(griffin_index *ix, uint32_t term, uin
 
 griffin_status griffin_debug_decode_list(griffin_index *ix, uint32_t term, uint32_t *out,
                                          uint64_t cap, uint64_t *n) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix || term >= ix->V || !n) return invalid("bad arguments");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -908,6 +1034,7 @@ griffin_status griffin_debug_decode_list(griffin_index *ix, uint32_t term, uint3
 
 griffin_status griffin_debug_decode_all(griffin_index *ix, int iters, double *ms,
                                         uint64_t *checksum, uint64_t *postings, uint64_t *bytes) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix || iters <= 0) return invalid("bad arguments");
   std::lock_guard<std::mutex> lk(ix->mu);
   DeviceGuard guard(ix->device);
@@ -948,6 +1075,7 @@ griffin_status griffin_debug_decode_all(griffin_index *ix, int iters, double *ms
 griffin_status griffin_debug_intersect(griffin_index *ix, const uint32_t *terms, uint32_t nterms,
                                        int mode, uint32_t *out_docids, uint64_t cap,
                                        uint64_t *count) {
+  if (ix && ix->cl) return multi_unsupported();
   if (!ix || !terms || nterms == 0 || !count) return invalid("bad arguments");
   if (mode < 0 || mode > 2) return invalid("bad mode");
   std::lock_guard<std::mutex> lk(ix->mu);

@@ -131,8 +131,16 @@ struct RoundArgs {
 
 }  // namespace griffin
 
+namespace griffin {
+struct Cluster;
+}
+
 struct griffin_index {
   std::mutex mu;
+  // multi-GPU handle (griffin_build_opts.num_gpus > 1): the shards and their
+  // exchange state; every query call goes through multi.cu
+  std::vector<griffin_index *> shards;
+  griffin::Cluster *cl = nullptr;
   int device = 0;
   cudaStream_t stream = nullptr;
   // options
@@ -227,5 +235,30 @@ inline uint32_t probe_chunk(const griffin_index *ix) {
 }
 void host_query_bounds(const griffin_index *ix, uint32_t *ts, uint32_t n, uint64_t *cap,
                        uint64_t *units);
+griffin_status launch_merge_topk_peer(griffin_index *ix, uint32_t G, uint32_t nq, uint32_t k,
+                                      const uint64_t *const *keys, const uint32_t *const *counts,
+                                      uint64_t *d_out_keys, uint32_t *d_out_counts, cudaStream_t st);
+// api.cu helpers used by multi.cu
+griffin_status reserve_for(griffin_index *ix, Workspace &w, uint32_t nq, const uint32_t *qoffs,
+                           const uint32_t *terms, uint32_t k, uint32_t *max_terms);
+griffin_status ensure_pinned_ws(Workspace &w, size_t bytes);
+// multi.cu
+griffin_status cluster_init(griffin_index *cx, int exchange);
+void cluster_destroy(griffin_index *cx);
+griffin_status cluster_query_batch(griffin_index *cx, uint32_t nq, const uint32_t *qoffs,
+                                   const uint32_t *terms, uint32_t k, uint32_t *out_docids,
+                                   float *out_scores, uint32_t *out_counts);
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
 
 }  // namespace griffin

@@ -2047,6 +2047,38 @@ __global__ void merge_topk_kernel(uint32_t G, uint32_t nq, uint32_t k, const uin
   }
 }
 
+// The same G-way merge reading each shard's runs where they live (NEXT-2, fused
+// exchange + merge): run g is keys[g][q*k ..], counts[g][q] — device pointers
+// that may be on peer GPUs (loads go over NVLink once peer access is enabled).
+struct PeerRuns {
+  const uint64_t *keys[GRIFFIN_MAX_SHARDS];
+  const uint32_t *counts[GRIFFIN_MAX_SHARDS];
+};
+__global__ void merge_topk_peer_kernel(uint32_t G, uint32_t nq, uint32_t k, PeerRuns r,
+                                       uint64_t *out, uint32_t *out_counts) {
+  const uint32_t lane = lane_id();
+  const uint32_t nwarps = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t q = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); q < nq; q += nwarps) {
+    const uint32_t cnt = lane < G ? min(r.counts[lane][q], k) : 0u;
+    const uint64_t *run = lane < G ? r.keys[lane] + (size_t)q * k : nullptr;
+    uint32_t p = 0;
+    uint64_t head = p < cnt ? run[0] : 0ull;
+    uint32_t i = 0;
+    for (; i < k; ++i) {
+      uint64_t best = head;
+      for (int d = 16; d; d >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, d));
+      if (best == 0ull) break;
+      if (lane == 0) out[(size_t)q * k + i] = best;
+      if (head == best) {  // keys are unique: exactly one lane advances
+        ++p;
+        head = p < cnt ? run[p] : 0ull;
+      }
+    }
+    for (uint32_t j = i + lane; j < k; j += 32) out[(size_t)q * k + j] = 0ull;
+    if (lane == 0) out_counts[q] = i;
+  }
+}
+
 __global__ void keys_to_results_kernel(uint32_t nq, uint32_t k, const uint64_t *keys,
                                        const uint32_t *counts, uint32_t *docids, float *scores) {
   const uint64_t n = (uint64_t)nq * k;
@@ -2579,6 +2611,27 @@ griffin_status launch_merge_topk(griffin_index *ix, uint32_t G, uint32_t nq, uin
   ix->launch_count += 1;
   merge_topk_kernel<<<std::min<uint32_t>((nq + 7) / 8, 148 * 16), 256, 0, st>>>(
       G, nq, k, d_keys, d_counts, d_out_keys, d_out_counts);
+  GRIFFIN_CUDA_TRY(cudaGetLastError());
+  return GRIFFIN_OK;
+}
+
+griffin_status launch_merge_topk_peer(griffin_index *ix, uint32_t G, uint32_t nq, uint32_t k,
+                                      const uint64_t *const *keys, const uint32_t *const *counts,
+                                      uint64_t *d_out_keys, uint32_t *d_out_counts,
+                                      cudaStream_t st) {
+  if (nq == 0) return GRIFFIN_OK;
+  if (G == 0 || G > GRIFFIN_MAX_SHARDS) {
+    set_error("peer merge: 1..8 runs");
+    return GRIFFIN_ERR_INVALID_ARG;
+  }
+  PeerRuns r{};
+  for (uint32_t g = 0; g < G; ++g) {
+    r.keys[g] = keys[g];
+    r.counts[g] = counts[g];
+  }
+  ix->launch_count += 1;
+  merge_topk_peer_kernel<<<std::min<uint32_t>((nq + 7) / 8, num_sms(ix->device) * 16), 256, 0, st>>>(
+      G, nq, k, r, d_out_keys, d_out_counts);
   GRIFFIN_CUDA_TRY(cudaGetLastError());
   return GRIFFIN_OK;
 }

@@ -121,3 +121,17 @@ def test_build_without_gpu_fails_loudly():
 def test_invalid_arguments_rejected_on_host():
     with pytest.raises(g.GriffinError):
         g.griffin_merge_path_split([1, 2], [3], 9)
+
+
+def test_multi_gpu_options_rejected_on_host():
+    """num_gpus / exchange are checked before any device is touched (§8(b))."""
+    c = corpus_from_lists(10, [[1, 2, 3]])
+    with pytest.raises(g.GriffinError) as e:
+        g.GriffinIndex(c, num_gpus=9)
+    assert e.value.status == 1
+    with pytest.raises(g.GriffinError) as e:
+        g.GriffinIndex(c, num_gpus=2, exchange=7)
+    assert e.value.status == 1
+    with pytest.raises(g.GriffinError) as e:   # a multi handle builds its shards itself
+        g.GriffinIndex(c, num_gpus=2, num_shards=2)
+    assert e.value.status == 1
