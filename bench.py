@@ -271,6 +271,11 @@ def run_gpu(args):
     build_s = time.time() - t0
     st = ix.griffin_index_stats()
     ix.griffin_set_reuse({"auto": 2, "on": 1, "off": 0}[args.reuse])
+    # intermediate capacity per workspace buffer: packed by actual survivors, so a
+    # budget well under the sum of per-query bounds holds a batch (C5: ~1e9 bound)
+    budget = args.entry_budget if args.entry_budget is not None else \
+        (400_000_000 if args.config in ("c4", "c5") else 0)
+    ix.griffin_set_entry_budget(budget)
     stream = torch.cuda.current_stream()
     dq = []   # per batch: (d_off, d_terms, max_terms)
     for b in batches:
@@ -505,7 +510,7 @@ def run_gpu(args):
         "batches_in_flight": len(slots),
         "index": {"bytes_per_shard": st["payload_bytes"] + st["skip_bytes"] + st["tf_bytes"],
                   "payload_bytes": st["payload_bytes"], "build_s": build_s,
-                  "corpus_load_s": gen_s, "reuse": args.reuse},
+                  "corpus_load_s": gen_s, "reuse": args.reuse, "entry_budget": budget},
         "decoded_postings_per_s": decoded_ps * world,
         "sync_qps": {"value": nq / (statistics.median(sync_ms) / 1e3) if sync_ms else None,
                      "unit": "queries/s", "median_ms": statistics.median(sync_ms) if sync_ms else None,
@@ -577,15 +582,17 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--latency-queries", type=int, default=1000)
     ap.add_argument("--streams", type=int, default=None,
-                    help="batches in flight on separate streams/workspaces (N=1 only); default "
-                         "3 for the 1K-query configs, 2 for the 10K-query batches")
+                    help="batches in flight on separate streams/workspaces (N=1 only); default 3")
     ap.add_argument("--reuse", default="auto", choices=["auto", "on", "off"],
                     help="batch decode-once of hot lists into an HBM arena")
+    ap.add_argument("--entry-budget", type=int, default=None,
+                    help="intermediate entries per workspace buffer (0 = exact bound); "
+                         "default 4e8 for c4/c5, else 0")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.streams is None:
-        args.streams = 2 if args.config in ("c4", "c5") else 3
+        args.streams = 3
     args.gpus = int(os.environ.get("WORLD_SIZE", args.gpus))
     if args.impl == "reference":
         run_reference(args)

@@ -268,6 +268,15 @@ griffin_status griffin_keys_to_results_device(griffin_index *ix, uint32_t nq, ui
 
 /* ---- configuration / instrumentation ---------------------------------------- */
 griffin_status griffin_set_mode(griffin_index *ix, int mode); /* griffin_mode; default AUTO */
+/* Intermediate-result capacity of workspaces reserved from now on, in
+ * (docID, score) entries per buffer.  0 (default): the exact bound, the sum over
+ * the batch's queries of min(df of its two shortest lists) — never overflows,
+ * but tens of GB for a 10K-query batch of frequent terms (C5).  A budget caps
+ * it: survivors are packed into the intermediates by actual count (a device scan
+ * per round), so the budget only has to hold what a batch really produces; a
+ * batch that exceeds it reports GRIFFIN_ERR_OOM (griffin_sync_status / the host
+ * calls) and writes no partial results. */
+griffin_status griffin_set_entry_budget(griffin_index *ix, uint64_t entries);
 /* 0 off; 1 per-stage CUDA events + algorithmic-byte counters; 2 events only
  * (kernel durations without the counting work); 3 counters only. */
 griffin_status griffin_set_profiling(griffin_index *ix, int on);

@@ -107,6 +107,7 @@ _SIGS = {
     "griffin_set_reuse": [_vp, ctypes.c_int],
     "griffin_set_nextgeq": [_vp, ctypes.c_int],
     "griffin_set_probe_chunk": [_vp, _u32],
+    "griffin_set_entry_budget": [_vp, _u64],
     "griffin_pfd_build": [_vp, _u32, ctypes.c_int, _vp],
     "griffin_pfd_stats": [_vp, _vp],
     "griffin_pfd_block_stream": [_vp, _u32, _u32, _vp, _vp, _vp, _u32, _vp],
@@ -390,6 +391,10 @@ class GriffinIndex:
     def griffin_set_probe_chunk(self, chunk: int):
         """Probe-pass survivors per unit (multiple of 32 in [32, B]; 0 = B)."""
         _check(load_library().griffin_set_probe_chunk(self.h, chunk))
+
+    def griffin_set_entry_budget(self, entries: int):
+        """Intermediate entries per workspace buffer (0 = exact per-batch bound)."""
+        _check(load_library().griffin_set_entry_budget(self.h, entries))
 
     def griffin_set_profiling(self, on):
         """False/0 off, True/1 events + counters, 2 events only, 3 counters only."""

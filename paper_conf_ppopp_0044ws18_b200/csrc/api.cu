@@ -346,6 +346,7 @@ void griffin_index_destroy(griffin_index *ix) {
     }
     ix->extra_ws.clear();
     free_workspace(ix->ws);
+    free_workspace(ix->qws);
     for (cudaEvent_t e : ix->ev_pool) cudaEventDestroy(e);
     for (auto &g : ix->graphs) cudaGraphExecDestroy(g.exec);
     if (ix->stream) cudaStreamDestroy(ix->stream);
@@ -450,6 +451,10 @@ static uint64_t ws_identity(const Workspace &w) {
                           &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand,
                           &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.run_term, &w.arena})
     h = (h ^ (uint64_t)(uintptr_t)b->p) * 1099511628211ull;
+  // capacities are baked into a captured graph's kernel arguments too
+  for (const uint64_t v : {(uint64_t)w.nq_cap, (uint64_t)w.unit_cap, (uint64_t)w.entry_cap,
+                           (uint64_t)w.bump.bytes})
+    h = (h ^ v) * 1099511628211ull;
   return h ^ (uint64_t)(uintptr_t)w.h_pinned;
 }
 
@@ -460,11 +465,11 @@ static uint64_t ws_identity(const Workspace &w) {
 static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint32_t nterms,
                                   uint32_t k, uint32_t *out_docids, float *out_scores,
                                   uint32_t *out_count) {
-  Workspace &w = ix->ws;
+  Workspace &w = ix->qws;   // own workspace: batch reservations never move its graphs
   const uint32_t offs[2] = {0, nterms};
   uint32_t mt = 1;
   // validation + bounds (same rules as the batch path)
-  griffin_status s = reserve_for(ix, ix->ws, 1, offs, terms, k, &mt);
+  griffin_status s = reserve_for(ix, w, 1, offs, terms, k, &mt);
   if (s) return s;
   if (!ix->single_ws) {
     uint64_t mx = 0, mb = 0;
@@ -472,7 +477,9 @@ static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint
       mx = std::max<uint64_t>(mx, t.df_local);
       mb = std::max<uint64_t>(mb, t.nblocks);
     }
-    if ((s = reserve_ws(ix, w, 1, 2 * mb + 1, mx + 1))) return s;
+    // units of any one query: blocks of t0 + max(blocks of a later list, probe
+    // units of >= 32 survivors each)
+    if ((s = reserve_ws(ix, w, 1, 2 * mb + mx / 32 + 2, mx + 1))) return s;
     if ((s = reserve_topk(ix, w, 1, GRIFFIN_MAX_K))) return s;
     if ((s = reserve_topk(ix, w, 1, 2048))) return s;   // the k with the most selection levels
     GRIFFIN_CUDA_TRY(w.qoffs.reserve(8));
@@ -481,7 +488,7 @@ static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint
     GRIFFIN_CUDA_TRY(w.counts.reserve(8));
     GRIFFIN_CUDA_TRY(w.docids.reserve(GRIFFIN_MAX_K * 4));
     GRIFFIN_CUDA_TRY(w.scores.reserve(GRIFFIN_MAX_K * 4));
-    if ((s = ensure_pinned(ix, 64 * 4 + GRIFFIN_MAX_K * 8 + 64))) return s;
+    if ((s = ensure_pinned_ws(w, 64 * 4 + GRIFFIN_MAX_K * 8 + 64))) return s;
     ix->single_ws = true;
   }
   if (nterms > GRIFFIN_MAX_TERMS * 4) return GRIFFIN_ERR_UNSUPPORTED;  // caller falls back
@@ -503,7 +510,7 @@ static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint
     GRIFFIN_CUDA_TRY(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
     cudaMemcpyAsync(w.qoffs.p, h_off, 8, cudaMemcpyHostToDevice, st);
     cudaMemcpyAsync(w.qterms.p, h_terms, GRIFFIN_MAX_TERMS * 4 * 4, cudaMemcpyHostToDevice, st);
-    griffin_status rs = run_batch(ix, ix->ws, 1, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), mt, k,
+    griffin_status rs = run_batch(ix, w, 1, w.qoffs.as<uint32_t>(), w.qterms.as<uint32_t>(), mt, k,
                                   w.keys.as<uint64_t>(), w.counts.as<uint32_t>(), st, true,
                                   ix->mode);
     if (!rs)
@@ -534,7 +541,7 @@ static griffin_status query_graph(griffin_index *ix, const uint32_t *terms, uint
   GRIFFIN_CUDA_TRY(cudaGraphLaunch(exec, st));
   GRIFFIN_CUDA_TRY(cudaStreamSynchronize(st));
   if (*h_status) {
-    if ((s = read_status(ix, ix->ws))) return s;   // clears the device flag
+    if ((s = read_status(ix, w))) return s;   // clears the device flag
   }
   std::memcpy(out_docids, h_res, (size_t)k * 4);
   std::memcpy(out_scores, h_res + (size_t)k * 4, (size_t)k * 4);
@@ -880,6 +887,17 @@ griffin_status griffin_set_probe_chunk(griffin_index *ix, uint32_t chunk) {
   return GRIFFIN_OK;
 }
 
+griffin_status griffin_set_entry_budget(griffin_index *ix, uint64_t entries) {
+  if (!ix) return invalid("null index");
+  if (ix->cl) {
+    for (griffin_index *sh : ix->shards) sh->entry_budget = entries;
+    return GRIFFIN_OK;
+  }
+  std::lock_guard<std::mutex> lk(ix->mu);
+  ix->entry_budget = entries;
+  return GRIFFIN_OK;
+}
+
 griffin_status griffin_set_profiling(griffin_index *ix, int on) {
   if (ix && ix->cl) {   // multi-GPU handle: every shard
     for (griffin_index *sh : ix->shards) {
@@ -907,6 +925,7 @@ griffin_status griffin_reset_profile(griffin_index *ix) {
   ix->launch_count = 0;
   std::vector<Workspace *> all(ix->extra_ws);
   all.push_back(&ix->ws);
+  all.push_back(&ix->qws);
   for (Workspace *w : all)
     if (w->scal.p) {
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.p, 0, 4 * 8));
@@ -937,6 +956,7 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
   out->launches_total = ix->launch_count;
   std::vector<Workspace *> all(ix->extra_ws);
   all.push_back(&ix->ws);
+  all.push_back(&ix->qws);
   out->alg_bytes = out->payload_bytes = out->decoded_postings = out->survivors = 0;
   out->dec_alg_bytes = out->dec_payload_bytes = out->dec_postings = 0;
   out->c8d_bytes = out->dec_c8d_bytes = out->arena_postings = 0;

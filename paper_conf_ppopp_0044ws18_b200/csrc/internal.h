@@ -39,7 +39,9 @@ struct DevBuf {
     if (p) cudaFree(p);
     p = nullptr;
     bytes = 0;
-    size_t nb = want + want / 4 + 256;
+    // small buffers grow with 25% headroom (fewer re-allocations); large ones
+    // (intermediates, arena, candidates: GBs at C5) are sized exactly
+    size_t nb = want < (64ull << 20) ? want + want / 4 + 256 : want + 256;
     cudaError_t e = cudaMalloc(&p, nb);
     if (e == cudaSuccess) bytes = nb;
     return e;
@@ -91,7 +93,8 @@ enum : int {
   kScalPerm = 13,     // 2 x u64: unit order list head (merge units) / tail (the rest)
   kScalArena = 15,    // 2 x u64: decoded-arena postings read by intersect, their compressed bytes
   kScalDecC8d = 17,   // u64: decode-once compressed bytes read (payload + skip/meta)
-  kScalCount = 18
+  kScalRoundTot = 18, // u64: survivors of the current round (compaction scan total)
+  kScalCount = 19
 };
 
 constexpr uint32_t kBumpChunk = 256;   // bump-area entries grabbed per warp atomic
@@ -106,7 +109,9 @@ struct RoundArgs {
   const uint32_t *plan_terms;
   const uint32_t *plan_m;
   const uint32_t *cap;
-  const uint64_t *cap_off;
+  uint64_t *cap_off;      // per query, per buffer: region offset ([0,nq] rbuf0, [nq+1,2nq+1] rbuf1)
+  const uint64_t *roff_prev;   // this round's input offsets (buffer (round-1)&1)
+  uint64_t *roff_next;         // this round's output offsets (buffer round&1)
   uint32_t *rcount;
   uint8_t *rsel;
   uint32_t *qmode;
@@ -159,6 +164,7 @@ struct griffin_index {
   std::vector<griffin::TermInfo> h_terms;
   // query state
   griffin::Workspace ws;
+  griffin::Workspace qws;   // griffin_query's CUDA-graph path (sized for one query)
   std::vector<griffin::Workspace *> extra_ws;  // griffin_workspace_create
   int mode = 0;
   int reuse = 2;
@@ -178,6 +184,7 @@ struct griffin_index {
   int sorder = 1;   // merge units ordered by the S blocks they read (L2 reuse across queries)
   uint32_t sorder_shift = 6;
   uint32_t P = 0;   // probe chunk (0 = B)
+  uint64_t entry_budget = 0;   // griffin_set_entry_budget: intermediate entries per workspace (0 = exact bound)
   int profiling = 0;   // bit 0: per-stage CUDA events, bit 1: algorithmic-byte counters
   griffin_profile prof{};
   std::vector<cudaEvent_t> ev_pool;

@@ -147,7 +147,10 @@ __global__ void plan_totals_kernel(DevIndex ix, uint32_t nq, const uint32_t *pla
 
 __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
   const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
-  const bool overflow = a.scal[kScalTotals] > a.entry_cap || a.scal[kScalTotals + 1] > a.unit_cap;
+  // units must fit their arrays; intermediates are checked at compaction time
+  // against the entries actually produced (the workspace may hold fewer entries
+  // than the sum of the per-query bounds, griffin_set_entry_budget)
+  const bool overflow = a.scal[kScalTotals + 1] > a.unit_cap;
   if (q == 0) {
     a.scal[kScalBump] = 0;
     a.scal[kScalUnitCtr] = 0;
@@ -686,7 +689,7 @@ __device__ __forceinline__ void unit_record(const DevIndex &ix, const RoundArgs 
         x0 = __ldg(ix.first + tR.block0 + lu);
         x1 = lu + 1 < tR.nblocks ? __ldg(ix.first + tR.block0 + lu + 1) - 1u : 0xFFFFFFFFu;
       } else {
-        const uint2 *Rq = a.rprev + a.cap_off[q];
+        const uint2 *Rq = a.rprev + a.roff_prev[q];
         const uint32_t s0 = lu * ix.B, s1 = min(s0 + ix.B, a.rcount[q]);
         x0 = Rq[s0].x;
         x1 = Rq[s1 - 1].x;
@@ -698,7 +701,7 @@ __device__ __forceinline__ void unit_record(const DevIndex &ix, const RoundArgs 
       const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
       const TermInfo tR = ix.terms[pt[0]];
       const TermInfo tS = ix.terms[pt[a.round]];
-      const uint2 *Rq = RC ? nullptr : a.rprev + a.cap_off[q];
+      const uint2 *Rq = RC ? nullptr : a.rprev + a.roff_prev[q];
       const uint32_t nbR = RC ? tR.nblocks : (a.rcount[q] + ix.B - 1) / ix.B;
       const uint32_t nbS = tS.nblocks;
       auto hR = [&](uint32_t i) -> uint32_t {
@@ -917,7 +920,7 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
   const uint32_t G = min(D - 3u, 31u);
   const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
   const uint32_t m = a.plan_m[q];
-  const uint2 *Rq = a.rprev + a.cap_off[q];
+  const uint2 *Rq = a.rprev + a.roff_prev[q];
   const uint32_t nR = a.rcount[q];
   uint32_t *tileR = sm.tile, *sc = sm.tile + B, *nrm = sm.tile + 2 * B, *kidx = sm.tile + 3 * B;
   uint32_t *match = sm.tile + 4 * B, *tileS = sm.tile + 5 * B;
@@ -1123,7 +1126,7 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
     const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
     const uint32_t t0 = pt[0];
     const TermInfo tR = ix.terms[t0];
-    const uint2 *Rq = RC ? nullptr : a.rprev + a.cap_off[q];
+    const uint2 *Rq = RC ? nullptr : a.rprev + a.roff_prev[q];
     const uint32_t nR = RC ? tR.df_local : a.rcount[q];
     const uint32_t nbR = RC ? tR.nblocks : (nR + B - 1) / B;
     // R source: compressed EF, the batch's decoded arena, or the intermediate
@@ -1637,28 +1640,49 @@ __global__ void __launch_bounds__(kScanThreads) unit_scan_apply(const uint32_t *
   }
 }
 
-// Warp per unit: copy its survivors from the bump area to the query's region of
-// the next intermediate, in unit (= docID) order.  The warp holding a query's
-// last unit publishes the query's new |R|.
+// Warp per unit: copy its survivors from the bump area to the next
+// intermediate, in unit (= docID) order.  Rounds 1 and 2 write their buffers
+// (rbuf1, rbuf0) for the first time: survivors are packed by actual count, unit
+// u at the exclusive scan of unit counts, so a buffer only has to hold what the
+// round produces (a round that does not fit flags an overflow and writes
+// nothing).  Later rounds (the SvS loop without the probe pass) write each
+// query in place over its own region of round r-2 in the same buffer, which it
+// fits (SvS survivor sets only shrink) and which no finished query uses.  The
+// warp holding a query's last unit publishes its new |R| and region offset.
 __global__ void __launch_bounds__(256) compact_copy_kernel(RoundArgs a, const uint64_t *udst) {
   const uint32_t lane = lane_id();
   const uint64_t *ubase = a.unit_base;
   const uint64_t total = ubase[a.nq];
+  const bool packed = a.round <= 2;
+  if (packed && a.scal[kScalRoundTot] > a.entry_cap) {
+    if (blockIdx.x == 0 && threadIdx.x == 0)
+      atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
+    return;
+  }
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); u < total;
        u += nwarps) {
     const uint32_t q = a.urec[u].x;   // the partition stage's record
-    const uint64_t base = udst[ubase[q]];
     const uint64_t my = udst[u];
+    const uint64_t base = udst[ubase[q]];
     const uint32_t cnt = a.unit_cnt[u];
     const uint2 *src = a.bump + a.unit_off[u];
-    uint2 *dst = a.rnext + a.cap_off[q] + (my - base);
+    uint2 *dst = a.rnext + (packed ? my : a.roff_next[q] + (my - base));
     for (uint32_t i = lane; i < cnt; i += 32) dst[i] = src[i];
     if (lane == 0 && u + 1 == ubase[q + 1]) {
       a.rcount[q] = (uint32_t)(my + cnt - base);
       a.rsel[q] = (uint8_t)(a.round & 1u);
+      if (packed) a.roff_next[q] = base;
     }
   }
+}
+
+// Query q's final intermediate: buffer rsel[q] at q's offset in that buffer
+// (roff holds one per-query offset array per buffer: [0, nq] rbuf0, then rbuf1).
+__device__ __forceinline__ const uint2 *final_region(const uint8_t *rsel, const uint64_t *roff,
+                                                     uint32_t nq, const uint2 *rb0,
+                                                     const uint2 *rb1, uint32_t q) {
+  return rsel[q] ? rb1 + roff[(size_t)nq + 1 + q] : rb0 + roff[q];
 }
 
 // ------------------------------------------------------------------- top-k
@@ -1821,7 +1845,7 @@ __global__ void __launch_bounds__(kTopkThreads) topk_sample_kernel(
     const float mu = (float)k * (float)kFiltSample / (float)n;
     const uint32_t r = (uint32_t)ceilf(mu + 4.f * sqrtf(mu) + 2.f);
     if (r > kFiltSample / 8) continue;
-    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q];
+    const uint2 *R = final_region(rsel, cap_off, nq, rb0, rb1, q);
     for (uint32_t j = threadIdx.x; j < kFiltSample; j += blockDim.x)
       sk[j] = make_key(R[(uint32_t)(((uint64_t)j * n) / kFiltSample)], ix.doc_base);
     __syncthreads();
@@ -1860,7 +1884,7 @@ __global__ void __launch_bounds__(256) topk_filter_kernel(
     const uint32_t q = lo;
     const uint32_t ci = (uint32_t)(c - cbase[q]);
     const uint32_t len = min(kTopkSmem, ts.qn[q] - ci * kTopkSmem);
-    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q] + (size_t)ci * kTopkSmem;
+    const uint2 *R = final_region(rsel, cap_off, nq, rb0, rb1, q) + (size_t)ci * kTopkSmem;
     const uint64_t tau = ts.ftau[q];
     const uint32_t slot = ts.fslot[q];
     uint64_t *out = ts.flt + (size_t)slot * kFiltCap;
@@ -1935,7 +1959,7 @@ __global__ void __launch_bounds__(kTopkThreads) topk_chunk_kernel(
     const uint32_t lev = ts.qlev[q];
     const uint32_t len = min(kTopkSmem, ts.qn[q] - ci * kTopkSmem);
     if (lev == 0) {
-      const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q] + (size_t)ci * kTopkSmem;
+      const uint2 *R = final_region(rsel, cap_off, nq, rb0, rb1, q) + (size_t)ci * kTopkSmem;
       for (uint32_t i = threadIdx.x; i < len; i += blockDim.x) sk[i] = make_key(R[i], ix.doc_base);
     } else {
       const uint64_t *K = cand_keys(cb, ts, lev, q) + (size_t)ci * kTopkSmem;
@@ -1974,7 +1998,7 @@ __global__ void __launch_bounds__(kTopkThreads) topk_final_kernel(
   for (uint32_t q = blockIdx.x; q < nq; q += gridDim.x) {
     const uint32_t c = rcount[q];
     const uint32_t kk = min(k, c);
-    const uint2 *R = (rsel[q] ? rb1 : rb0) + cap_off[q];
+    const uint2 *R = final_region(rsel, cap_off, nq, rb0, rb1, q);
     const uint32_t lev = ts.qlev[q];
     const uint64_t *C = lev ? cand_keys(cb, ts, lev, q) : nullptr;
     const uint32_t n = ts.qn[q];
@@ -2273,11 +2297,15 @@ static int num_sms(int dev) {
 
 griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t units,
                           uint64_t entries) {
+  // `entries` is the exact per-batch bound (sum over queries of min(df0, df1));
+  // a budget caps it: the intermediates are packed by actual survivors, and a
+  // batch whose survivors exceed it reports GRIFFIN_ERR_OOM (overflow)
+  if (ix->entry_budget && entries > ix->entry_budget) entries = ix->entry_budget;
   const size_t q = (size_t)nq + 1;
   GRIFFIN_CUDA_TRY(w.plan_terms.reserve(q * kMaxTerms * 4));
   GRIFFIN_CUDA_TRY(w.plan_m.reserve(q * 4));
   GRIFFIN_CUDA_TRY(w.cap.reserve(q * 4));
-  GRIFFIN_CUDA_TRY(w.cap_off.reserve(q * 8 + 8));
+  GRIFFIN_CUDA_TRY(w.cap_off.reserve(2 * q * 8 + 8));   // per-query region offsets, per buffer
   GRIFFIN_CUDA_TRY(w.rcount.reserve(q * 4));
   GRIFFIN_CUDA_TRY(w.rsel.reserve(q));
   GRIFFIN_CUDA_TRY(w.qmode.reserve(q * 4 + q * 4));  // qmode | qunits
@@ -2434,8 +2462,6 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
         di, nq, w.plan_terms.as<uint32_t>(), w.plan_m.as<uint32_t>(), w.cap.as<uint32_t>(),
         probe_chunk(ix), scal);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
-    GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(w.cap.as<uint32_t>(), w.cap_off.as<uint64_t>(), nq,
-                                              scan_tmp, st, &ix->launch_count));
   }
   // batch reuse: decode hot lists once into the arena (decompress-then-intersect)
   const bool reuse = ix->reuse == 1 || (ix->reuse == 2 && nq >= 8);
@@ -2493,13 +2519,15 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     ra.round = r;
     ra.rprev = (r & 1) ? w.rbuf0.as<uint2>() : w.rbuf1.as<uint2>();
     ra.rnext = (r & 1) ? w.rbuf1.as<uint2>() : w.rbuf0.as<uint2>();
+    ra.roff_prev = ra.cap_off + ((r - 1) & 1u) * ((size_t)nq + 1);
+    ra.roff_next = ra.cap_off + (r & 1u) * ((size_t)nq + 1);
     {
       StageTimer t(ix, st, 0);
       plan_round_kernel<<<qblocks, 256, 0, st>>>(di, ra, qunits);
       GRIFFIN_CUDA_TRY(cudaGetLastError());
       GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(qunits, w.unit_base.as<uint64_t>(), nq, scan_tmp, st,
                                                 &ix->launch_count));
-      ix->launch_count += 3;  // plan_round + intersect + compact
+      ix->launch_count += 1;  // plan_round (the scan counts itself)
     }
     {
       StageTimer t(ix, st, 1);
@@ -2525,7 +2553,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
       }
       if (r == 1) GRIFFIN_CUDA_TRY(launch_intersect<true>(ix, ra, st));
       else GRIFFIN_CUDA_TRY(launch_intersect<false>(ix, ra, st));
-      ix->launch_count += 1;
+      ix->launch_count += 2;  // partition + intersect
     }
     {
       StageTimer t(ix, st, 2);
@@ -2533,12 +2561,13 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
       const unsigned tiles = (unsigned)(w.unit_cap / kScanTile + 1);
       uint64_t *tsum = w.unit_dst.as<uint64_t>() + (w.unit_cap + 2);
       unit_scan_sums<<<tiles, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum);
-      scan_single_kernel<uint64_t><<<1, kScanThreads, 0, st>>>(tsum, tsum, tiles, nullptr);
+      scan_single_kernel<uint64_t><<<1, kScanThreads, 0, st>>>(tsum, tsum, tiles,
+                                                               reinterpret_cast<uint64_t *>(scal + kScalRoundTot));
       unit_scan_apply<<<tiles, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum,
                                                       w.unit_dst.as<uint64_t>());
       compact_copy_kernel<<<num_sms(ix->device) * 8, 256, 0, st>>>(ra, w.unit_dst.as<uint64_t>());
       GRIFFIN_CUDA_TRY(cudaGetLastError());
-      ix->launch_count += 3;
+      ix->launch_count += 4;  // sums, single, apply, copy
     }
   }
   if (final_topk) {
@@ -2685,7 +2714,9 @@ griffin_status copy_final_docids(griffin_index *ix, uint32_t *h_out, uint64_t ca
   cudaStream_t st = ix->stream;
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(&c, w.rcount.p, 4, cudaMemcpyDeviceToHost, st));
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(&sel, w.rsel.p, 1, cudaMemcpyDeviceToHost, st));
-  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(&off, w.cap_off.p, 8, cudaMemcpyDeviceToHost, st));
+  GRIFFIN_CUDA_TRY(cudaStreamSynchronize(st));   // sel picks the offset array
+  GRIFFIN_CUDA_TRY(cudaMemcpyAsync(&off, w.cap_off.as<uint64_t>() + (sel ? 2 : 0), 8,
+                                   cudaMemcpyDeviceToHost, st));
   GRIFFIN_CUDA_TRY(cudaStreamSynchronize(st));
   *count = c;
   if (c > cap) {

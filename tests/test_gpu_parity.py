@@ -702,3 +702,30 @@ def test_nextgeq_gallop_matches_block_decode_and_oracle(B):
             gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 100)
             assert_topk_equal(gd, gs, gc, od, os_, oc)
         gx.griffin_set_mode(g.MODE_AUTO)
+
+
+def test_entry_budget_packed_intermediates(tiny):
+    """griffin_set_entry_budget: intermediates packed by actual survivors; a
+    budget that holds them gives identical results, one that does not reports
+    GRIFFIN_ERR_OOM, and the workspace recovers after the budget is raised."""
+    c, ql, ox = tiny
+    k = 10
+    od, os_, oc = ox.query_batch(ql, k)
+    # survivors of round 1 are at most the batch's results' superset; the exact
+    # bound (sum of min(df0, df1)) is far larger than what is produced
+    gx = g.GriffinIndex(c, block_size=128)
+    gx.griffin_set_entry_budget(200_000)
+    gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+    assert_topk_equal(gd, gs, gc, od, os_, oc)
+    for mode in (g.MODE_MERGE, g.MODE_GALLOP):   # multi-round SvS (no probe pass): packed tops
+        gx.griffin_set_mode(mode)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+    gy = g.GriffinIndex(c, block_size=128)
+    gy.griffin_set_entry_budget(64)
+    with pytest.raises(g.GriffinError) as e:
+        gy.griffin_query_batch(ql.offsets, ql.terms, k)
+    assert e.value.status == 3
+    gy.griffin_set_entry_budget(0)
+    gd, gs, gc = gy.griffin_query_batch(ql.offsets, ql.terms, k)
+    assert_topk_equal(gd, gs, gc, od, os_, oc)
