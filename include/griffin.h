@@ -159,6 +159,9 @@ typedef struct {
   uint64_t c8d_bytes;
   uint64_t dec_c8d_bytes;
   uint64_t arena_postings;   /* decoded-arena postings read by the intersect kernels */
+  /* unit shapes (counters mode): merge units and the elements they merged (R+S
+   * inside their docID ranges), gallop units and their R elements */
+  uint64_t merge_units, merge_elems, gallop_units, gallop_elems;
 } griffin_profile;
 
 /* ---- index ------------------------------------------------------------------

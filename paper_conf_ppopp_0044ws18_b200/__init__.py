@@ -74,7 +74,9 @@ class Profile(ctypes.Structure):
                 ("launches_decode", ctypes.c_uint64), ("dec_alg_bytes", ctypes.c_uint64),
                 ("dec_payload_bytes", ctypes.c_uint64), ("dec_postings", ctypes.c_uint64),
                 ("c8d_bytes", ctypes.c_uint64), ("dec_c8d_bytes", ctypes.c_uint64),
-                ("arena_postings", ctypes.c_uint64)]
+                ("arena_postings", ctypes.c_uint64), ("merge_units", ctypes.c_uint64),
+                ("merge_elems", ctypes.c_uint64), ("gallop_units", ctypes.c_uint64),
+                ("gallop_elems", ctypes.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

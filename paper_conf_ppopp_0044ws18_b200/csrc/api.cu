@@ -931,6 +931,7 @@ griffin_status griffin_reset_profile(griffin_index *ix) {
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.p, 0, 4 * 8));
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDec, 0, 3 * 8));
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalArena, 0, 3 * 8));
+      GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDiag, 0, 4 * 8));
     }
   return GRIFFIN_OK;
 }
@@ -960,6 +961,7 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
   out->alg_bytes = out->payload_bytes = out->decoded_postings = out->survivors = 0;
   out->dec_alg_bytes = out->dec_payload_bytes = out->dec_postings = 0;
   out->c8d_bytes = out->dec_c8d_bytes = out->arena_postings = 0;
+  out->merge_units = out->merge_elems = out->gallop_units = out->gallop_elems = 0;
   for (Workspace *w : all) {
     if (!w->scal.p) continue;
     unsigned long long c[kScalCount];
@@ -974,6 +976,10 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
     out->arena_postings += c[kScalArena];
     out->c8d_bytes += c[0] - 4ull * c[kScalArena] + c[kScalArena + 1];
     out->dec_c8d_bytes += c[kScalDecC8d];
+    out->merge_units += c[kScalDiag];
+    out->merge_elems += c[kScalDiag + 1];
+    out->gallop_units += c[kScalDiag + 2];
+    out->gallop_elems += c[kScalDiag + 3];
   }
   return GRIFFIN_OK;
 }

@@ -94,7 +94,8 @@ enum : int {
   kScalArena = 15,    // 2 x u64: decoded-arena postings read by intersect, their compressed bytes
   kScalDecC8d = 17,   // u64: decode-once compressed bytes read (payload + skip/meta)
   kScalRoundTot = 18, // u64: survivors of the current round (compaction scan total)
-  kScalCount = 19
+  kScalDiag = 19,     // 4 x u64 (counting mode): merge units, merged elements, gallop units, galloped elements
+  kScalCount = 23
 };
 
 constexpr uint32_t kBumpChunk = 256;   // bump-area entries grabbed per warp atomic

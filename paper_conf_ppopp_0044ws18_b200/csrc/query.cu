@@ -1324,6 +1324,10 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
       const uint32_t sa = __shfl_sync(0xffffffffu, r_lo, 16), sb = __shfl_sync(0xffffffffu, r_lo, 24);
       const uint32_t nr = rb - ra, ns = sb - sa;
       const uint32_t tot2 = nr + ns, L = (tot2 + 31) >> 5;
+      if (a.count && lane == 0) {   // unit-shape diagnostics (counting pass only)
+        atomicAdd(a.scal + kScalDiag, 1ull);
+        atomicAdd(a.scal + kScalDiag + 1, (unsigned long long)tot2);
+      }
       const uint32_t cap = (L >> 1) + 2;           // matches per lane <= ceil(L/2), +1 slack write
       uint32_t *ml = sm.stg + lane * cap;          // staging is free after decode
       uint32_t c = 0;
@@ -1417,6 +1421,10 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
       }
       __syncwarp();
       const uint32_t k_lo = rec.z, k_hi = rec.w;   // from the partition stage
+      if (a.count && lane == 0) {
+        atomicAdd(a.scal + kScalDiag + 2, 1ull);
+        atomicAdd(a.scal + kScalDiag + 3, (unsigned long long)n);
+      }
       // skip pointers the chunk can touch: [k_lo-1, k_hi); stage them in smem when
       // they fit (one round trip), else search them in global memory
       const uint32_t w0 = k_lo ? k_lo - 1u : 0u, span = k_hi - w0;
