@@ -866,9 +866,11 @@ __device__ __forceinline__ uint32_t arena_probe_slice(const uint32_t *__restrict
 #pragma unroll
   for (int j = 0; j < kArenaEpl; ++j) {
     if (act[j]) {
+      // a starting chunk only (the walk below finds x from any start): float
+      // arithmetic instead of a 64-bit integer division
       const uint32_t span = f1[j] > f0[j] ? f1[j] - f0[j] : 1u;
-      uint32_t est = (uint32_t)(((uint64_t)(xv[j] - f0[j]) * nb[j]) / span);
-      est = min(est, nb[j] - 1u);
+      const float fe = __fmul_rz((float)(xv[j] - f0[j]), __fdividef((float)nb[j], (float)span));
+      const uint32_t est = min(__float2uint_rz(fe), nb[j] - 1u);
       c[j] = est & ~7u;
     }
   }
@@ -881,14 +883,25 @@ __device__ __forceinline__ uint32_t arena_probe_slice(const uint32_t *__restrict
       ++chunks;
       const uint4 *p = reinterpret_cast<const uint4 *>(decS + (size_t)kb[j] * B + c[j]);
       const uint4 lo4 = __ldg(p), hi4 = __ldg(p + 1);
-      const uint32_t v[8] = {lo4.x, lo4.y, lo4.z, lo4.w, hi4.x, hi4.y, hi4.z, hi4.w};
+      uint32_t v[8] = {lo4.x, lo4.y, lo4.z, lo4.w, hi4.x, hi4.y, hi4.z, hi4.w};
       const uint32_t valid = min(8u, nb[j] - c[j]);
-      uint32_t less = 0, eq = 0;
+      if (valid < 8u) {   // a block's tail: slots past its end hold no docIDs
 #pragma unroll
-      for (uint32_t i = 0; i < 8; ++i) {
-        less += (i < valid && v[i] < xv[j]) ? 1u : 0u;
-        eq |= (i < valid && v[i] == xv[j]) ? 1u : 0u;
+        for (uint32_t i = 0; i < 8; ++i) v[i] = i < valid ? v[i] : kNone;
       }
+      // less = #{v[i] < x} by a branch-free 3-step search of the sorted chunk,
+      // eq = (v[less] == x)
+      const uint32_t x = xv[j];
+      const bool b4 = v[3] < x;
+      const uint32_t a0 = b4 ? v[4] : v[0], a1 = b4 ? v[5] : v[1], a2 = b4 ? v[6] : v[2],
+                     a3 = b4 ? v[7] : v[3];
+      const bool b2 = a1 < x;
+      const uint32_t e0 = b2 ? a2 : a0, e1 = b2 ? a3 : a1;
+      const bool b1 = e0 < x;
+      const uint32_t d0 = b1 ? e1 : e0;
+      const bool b0 = d0 < x;
+      const uint32_t less = (b4 ? 4u : 0u) + (b2 ? 2u : 0u) + (b1 ? 1u : 0u) + (b0 ? 1u : 0u);
+      const uint32_t eq = (!b0 && d0 == x) ? 1u : 0u;
       // step toward x, never reversing: a reversal means x falls between two
       // adjacent chunks, i.e. it is absent
       if (less == 0 && !eq && c[j] > 0 && dir[j] != 2u) {

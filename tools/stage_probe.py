@@ -40,7 +40,7 @@ for name, setup in variants:
     tot = []
     for rep in range(7):
         ix.griffin_reset_profile()
-        ix.griffin_set_profiling(True)
+        ix.griffin_set_profiling(2)   # stage events only
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(st)
         for _ in range(10):
