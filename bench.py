@@ -152,6 +152,14 @@ def load_workload(name):
     return corpus, batches, cfg
 
 
+def _parallelism(args):
+    if args.gpus <= 1:
+        return "1 shard"
+    if args.shard_mode == "replicate":
+        return f"replicated index x{args.gpus}, no exchange"
+    return f"docid-range shards x{args.gpus}, {args.exchange} exchange ({args.dist_backend})"
+
+
 def config_dict(args, corpus, cfg, nq, extra=None):
     """The `config` object, identical on both arms (ours and --impl reference)."""
     d = {"workload": WORKLOAD_DESC[args.config], "num_docs": corpus.num_docs,
@@ -159,7 +167,7 @@ def config_dict(args, corpus, cfg, nq, extra=None):
          "queries_per_step": nq, "k": cfg["k"], "block_size": cfg["block"],
          "batches_rotated": cfg.get("batches", 1),
          "l2": "inputs larger than L2 (index > 126 MB L2, rotating query batches)",
-         "parallelism": (f"docid-range shards x{args.gpus}" if args.gpus > 1 else "1 shard")}
+         "parallelism": _parallelism(args)}
     if extra:
         d.update(extra)
     return d
@@ -247,14 +255,19 @@ def run_gpu(args):
     import torch.distributed as dist
 
     import paper_conf_ppopp_0044ws18_b200 as g
-    from paper_conf_ppopp_0044ws18_b200.sharded import gather_runs
+    from paper_conf_ppopp_0044ws18_b200.sharded import exchange_sliced, gather_runs
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
+        # gloo (a dry run of the N>1 path on fewer GPUs than ranks): ranks share devices
+        local = local % torch.cuda.device_count() if args.dist_backend == "gloo" else local
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
     else:
         torch.cuda.set_device(0)
     dev = torch.cuda.current_device()
@@ -264,10 +277,14 @@ def run_gpu(args):
     k, B = cfg["k"], cfg["block"]
     NB = len(batches)
     nq = batches[0].num_queries
-    sharded = world > 1
+    # docid: rank r holds docID-range shard r, per-shard top-k exchanged (all-gather
+    # or query-sliced all-to-all) and merged; replicate: every
+    # rank holds the whole index and answers its own batches, no exchange
+    replicate = world > 1 and args.shard_mode == "replicate"
+    sharded = world > 1 and not replicate
     t0 = time.time()
     ix = g.GriffinIndex(corpus, block_size=B, device=dev, shard_index=rank if sharded else 0,
-                        num_shards=world)
+                        num_shards=world if sharded else 1)
     build_s = time.time() - t0
     st = ix.griffin_index_stats()
     ix.griffin_set_reuse({"auto": 2, "on": 1, "off": 0}[args.reuse])
@@ -304,9 +321,13 @@ def run_gpu(args):
             ix.griffin_query_batch_device(d_off, d_t, mt, k, kk_, cc_, st_)
         else:
             w.griffin_query_batch_device_ws(d_off, d_t, mt, k, kk_, cc_, st_)
-        if sharded:   # a8: all-gather of per-shard top-k + k-way merge (NCCL)
+        if sharded and args.exchange == "allgather":   # a8: all-gather + k-way merge (NCCL)
             ak, ac = gather_runs(kk_, cc_)
             ix.griffin_merge_topk_device(world, nq, k, ak, ac, out_keys, out_cnts, st_)
+        elif sharded:   # NEXT-2: query-sliced all-to-all, this rank merges its slice
+            ak, ac, (lo, hi) = exchange_sliced(kk_, cc_, k)
+            if hi > lo:
+                ix.griffin_merge_topk_device(world, hi - lo, k, ak, ac, out_keys, out_cnts, st_)
 
     for i in range(args.warmup):
         step_on(i)
@@ -345,11 +366,11 @@ def run_gpu(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     ms_per_step = total_ms / args.steps
-    qps = nq * args.steps / (total_ms / 1e3)
+    qps = (world if replicate else 1) * nq * args.steps / (total_ms / 1e3)
     # results of the last timed step (its slot's outputs are untouched since)
     last_i = args.steps - 1
     _, _, lk, lc = slots[last_i % len(slots)]
-    if sharded:
+    if sharded and args.exchange == "allgather":
         lk, lc = out_keys, out_cnts
     last_keys, last_cnts = lk.cpu().numpy(), lc.cpu().numpy()
     last_batch = batches[last_i % NB]
@@ -435,7 +456,7 @@ def run_gpu(args):
 
     # ---- §8(d) QPS: median wall time of one synchronous griffin_query_batch ----
     sync_ms = []
-    if not sharded:
+    if world == 1:
         for i in range(2 + max(5, NB)):
             b = batches[i % NB]
             t0 = time.perf_counter()
@@ -447,6 +468,8 @@ def run_gpu(args):
     e2e_s = None
     h2d = (nq + 1) * 4 + int(np.mean([len(b.terms) for b in batches])) * 4
     d2h = nq * k * 8 + nq * 4
+    if sharded and args.exchange == "sliced":   # each rank reads back its own slice
+        d2h = -(-nq // world) * (k * 8 + 4)
     if not sharded:
         e2e_ws = [ix] + [sl[0] for sl in slots[1:]]
         e2e_st = [sl[1] for sl in slots]
@@ -476,8 +499,14 @@ def run_gpu(args):
             h_t = torch.from_numpy(b.terms.astype(np.int32)).pin_memory()
             dist.barrier()
             t0 = time.perf_counter()
-            dd, ss, cc = searcher.search(h_off.to("cuda", non_blocking=True),
-                                         h_t.to("cuda", non_blocking=True), dq[i % NB][2], k, stream)
+            if args.exchange == "allgather":
+                dd, ss, cc = searcher.search(h_off.to("cuda", non_blocking=True),
+                                             h_t.to("cuda", non_blocking=True), dq[i % NB][2], k,
+                                             stream)
+            else:
+                _, _, dd, ss, cc = searcher.search_sliced(h_off.to("cuda", non_blocking=True),
+                                                          h_t.to("cuda", non_blocking=True),
+                                                          dq[i % NB][2], k, stream)
             dd, ss, cc = dd.cpu(), ss.cpu(), cc.cpu()
             if i >= args.warmup:
                 times.append(time.perf_counter() - t0)
@@ -489,7 +518,7 @@ def run_gpu(args):
 
     # ---- closed-loop single-query latency (griffin_query, one in flight) ----
     lat = []
-    if not sharded:
+    if world == 1:
         b0 = batches[0]
         nlat = min(b0.num_queries, args.latency_queries)
         for q in range(min(nlat, 64)):          # warm-up: capture the per-term-count graphs
@@ -507,7 +536,7 @@ def run_gpu(args):
     line = {
         "metric": "queries/sec", "value": qps, "unit": "queries/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "higher_is_better": True, "scaling": "weak" if replicate else "strong", "vs_baseline": None,
         "dtype": "u32/f32", "data": "synthetic",
         "config": config_dict(args, corpus, cfg, nq),
         "batches_in_flight": len(slots),
@@ -540,7 +569,7 @@ def run_gpu(args):
                          "note": "every block of the shard decoded once per launch; the index "
                                  "(> L2) is streamed from HBM"},
     }
-    if rank == 0 and not args.no_cpu_baseline:
+    if rank == 0 and not args.no_cpu_baseline and not (sharded and args.exchange == "sliced"):
         # oracle on a bounded sample of the LAST timed batch: the cpu_baseline,
         # and the parity reference for the same queries of the GPU's results
         osm = OracleSample(corpus, last_batch, k, B, budget_s=args.cpu_budget)
@@ -588,6 +617,12 @@ def main():
                     help="batches in flight on separate streams/workspaces (N=1 only); default 3")
     ap.add_argument("--reuse", default="auto", choices=["auto", "on", "off"],
                     help="batch decode-once of hot lists into an HBM arena")
+    ap.add_argument("--shard-mode", default="docid", choices=["docid", "replicate"],
+                    help="N>1: docID-range shards + exchange, or a replicated index per rank")
+    ap.add_argument("--exchange", default="allgather", choices=["allgather", "sliced"],
+                    help="docid shards: all-gather of per-shard top-k, or query-sliced all-to-all")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="N>1 process group; gloo lets ranks share a GPU (dry runs)")
     ap.add_argument("--entry-budget", type=int, default=None,
                     help="intermediate entries per workspace buffer (0 = exact bound); "
                          "default 4e8 for c4/c5, else 0")

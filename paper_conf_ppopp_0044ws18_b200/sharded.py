@@ -18,6 +18,9 @@ def gather_runs(keys: torch.Tensor, counts: torch.Tensor, group=None):
     """All-gather per-shard runs into the g-major layout the merge kernel takes:
     keys [G, nq*k] (int64 bit patterns of u64 keys), counts [G, nq]."""
     world = dist.get_world_size(group)
+    if keys.is_cuda and dist.get_backend(group) == "gloo":   # gloo: exchange through host memory
+        ak, ac = gather_runs(keys.cpu(), counts.cpu(), group)
+        return ak.to(keys.device), ac.to(counts.device)
     all_keys = torch.empty((world,) + tuple(keys.shape), dtype=keys.dtype, device=keys.device)
     all_cnts = torch.empty((world,) + tuple(counts.shape), dtype=counts.dtype, device=counts.device)
     if keys.is_cuda:
@@ -45,6 +48,9 @@ def exchange_sliced(keys: torch.Tensor, counts: torch.Tensor, k: int, group=None
     Returns (keys, counts, (q_lo, q_hi))."""
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
+    if keys.is_cuda and dist.get_backend(group) == "gloo":   # gloo: exchange through host memory
+        ak, ac, lh = exchange_sliced(keys.cpu(), counts.cpu(), k, group)
+        return ak.to(keys.device), ac.to(counts.device), lh
     nq = counts.numel()
     sl = query_slices(nq, world)
     lo, hi = sl[rank]
