@@ -24,7 +24,7 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import paper_conf_ppopp_0044ws18_b200 as g  # noqa: E402
-from synth import make_pair_workload, make_workload  # noqa: E402
+from synth import batch_of, make_pair_workload, make_workload  # noqa: E402
 
 
 def dev_batch(ix, ql, k):
@@ -121,7 +121,10 @@ def c3():
 
 def c5(nq=None):
     t0 = time.time()
-    c, ql, cfg = make_workload("c5", num_queries=nq)
+    c, ql, cfg = make_workload("c5")
+    ql = batch_of(ql, cfg, 0)
+    if nq:
+        ql = ql.slice(0, nq)
     gen_s = time.time() - t0
     k = cfg["k"]
     for B in (128, 64, 256, 512):
@@ -139,7 +142,7 @@ def c5(nq=None):
             for kq in (k, 10):   # C5 (top-1000) and the C4 per-shard workload at G = 1 (top-10)
                 run = dev_batch(ix, ql, kq)
                 ix.griffin_reset_profile()
-                ix.griffin_set_profiling(True)
+                ix.griffin_set_profiling(1)
                 ms = time_dev(run, iters=3, warmup=2)
                 ix.griffin_set_profiling(False)
                 p = ix.griffin_get_profile()
