@@ -142,7 +142,11 @@ typedef enum { GRIFFIN_MODE_AUTO = 0, GRIFFIN_MODE_MERGE = 1, GRIFFIN_MODE_GALLO
 typedef struct {
   double ms_plan, ms_intersect, ms_compact, ms_topk, ms_merge;
   uint64_t launches_intersect, launches_total;
-  uint64_t alg_bytes;        /* algorithmic bytes read+written by the intersect kernels */
+  uint64_t alg_bytes;        /* bytes the intersect kernels must read + write:
+                                compressed payload + 8-B skip/meta per block read, 4 B per
+                                decoded-arena posting, 8 B per intermediate entry, 32 B per
+                                arena probe sector, per survivor one 32-B sector per tf
+                                gather + 4-B norm + 8-B entry written */
   uint64_t payload_bytes;    /* compressed EF bytes of the blocks the method had to read */
   uint64_t decoded_postings; /* postings of those blocks */
   uint64_t survivors;        /* (docID, score) pairs emitted by intersection rounds */

@@ -203,6 +203,12 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
 
 // ------------------------------------------------------------------- intersect
 
+// SURVEY §8(d) per-survivor algorithmic bytes: each tf gather is one 32-B
+// sector, plus the doc's norm (4 B) and the (docID, score) entry written (8 B);
+// round 1 gathers two tfs (R and S), later rounds one (the previous partial
+// score comes with the intermediate entry, counted at 8 B per R element).
+constexpr uint32_t kTfSector = 32, kSurvBytes = kTfSector + 4 + 8,
+                   kSurvBytesR1 = 2 * kTfSector + 4 + 8;
 // Per-warp counters live in the warp's shared memory (lane 0 updates them),
 // not in registers: the kernel runs at the 80-register cap.
 enum : int { kCAlg = 0, kCPay, kCPost, kCSurv, kCApost, kCAcomp, kCNum };
@@ -468,7 +474,7 @@ __device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, co
     a.unit_off[u] = off;
     a.unit_cnt[u] = cnt;
     acc.ctr[kCSurv] += cnt;
-    acc.ctr[kCAlg] += (unsigned long long)cnt * (KIND == 0 ? 20u : 16u);
+    acc.ctr[kCAlg] += (unsigned long long)cnt * (KIND == 0 ? kSurvBytesR1 : kSurvBytes);
   }
 }
 
@@ -543,7 +549,7 @@ __device__ void emit_lanes(const DevIndex &ix, const RoundArgs &a, uint32_t u, c
     a.unit_off[u] = off;
     a.unit_cnt[u] = cnt;
     acc.ctr[kCSurv] += cnt;
-    acc.ctr[kCAlg] += (unsigned long long)cnt * (RC ? 20u : 16u);
+    acc.ctr[kCAlg] += (unsigned long long)cnt * (RC ? kSurvBytesR1 : kSurvBytes);
   }
 }
 
@@ -1076,7 +1082,7 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
       __syncwarp();
     }
     n = nn2;
-    if (lane == 0) acc.ctr[kCAlg] += n * 4u;
+    if (lane == 0) acc.ctr[kCAlg] += n * kTfSector;   // the kept survivors' tf gathers
   }
   // ---- emit the survivors ----
   unsigned long long off = 0;
