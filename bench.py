@@ -457,10 +457,11 @@ def run_gpu(args):
     # ---- §8(d) QPS: median wall time of one synchronous griffin_query_batch ----
     sync_ms = []
     if world == 1:
+        sync_out = (np.zeros(nq * k, np.uint32), np.zeros(nq * k, np.float32), np.zeros(nq, np.uint32))
         for i in range(2 + max(5, NB)):
             b = batches[i % NB]
             t0 = time.perf_counter()
-            ix.griffin_query_batch(b.offsets, b.terms, k)
+            ix.griffin_query_batch(b.offsets, b.terms, k, out=sync_out)
             if i >= 2:
                 sync_ms.append((time.perf_counter() - t0) * 1e3)
 
@@ -548,7 +549,8 @@ def run_gpu(args):
                      "unit": "queries/s", "median_ms": statistics.median(sync_ms) if sync_ms else None,
                      "calls": len(sync_ms),
                      "how": "SURVEY §8(d): batch size / median wall time of one synchronous "
-                            "griffin_query_batch (host buffers, H2D + D2H inside), rotating batches"},
+                            "griffin_query_batch (host buffers, H2D + D2H inside; the caller's "
+                            "output arrays reused across calls), rotating batches"},
         "latency_ms": {"p50": pct(50), "p99": pct(99), "queries": len(lat),
                        "mode": "closed-loop griffin_query (host buffers), one in flight"},
         "roofline": roof,

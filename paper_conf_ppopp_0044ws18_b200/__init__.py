@@ -324,16 +324,24 @@ class GriffinIndex:
         _check(load_library().griffin_query(self.h, _ptr(t), len(t), k, _ptr(d), _ptr(s), _ptr(c)))
         return d, s, int(c[0])
 
-    def griffin_query_batch(self, offsets, terms, k: int):
+    def griffin_query_batch(self, offsets, terms, k: int, out=None):
+        """out: optional (docids u32 >= nq*k, scores f32 >= nq*k, counts u32 >= nq)
+        arrays to fill, reused across calls (no fresh pages per batch)."""
         off = np.ascontiguousarray(offsets, np.uint32)
         t = np.ascontiguousarray(terms, np.uint32)
         nq = len(off) - 1
-        d = np.zeros(nq * k, np.uint32)
-        s = np.zeros(nq * k, np.float32)
-        c = np.zeros(max(nq, 1), np.uint32)
+        if out is None:
+            d = np.zeros(nq * k, np.uint32)
+            s = np.zeros(nq * k, np.float32)
+            c = np.zeros(max(nq, 1), np.uint32)
+        else:
+            d, s, c = (x.reshape(-1) for x in out)
+            if (d.dtype != np.uint32 or s.dtype != np.float32 or c.dtype != np.uint32
+                    or d.size < nq * k or s.size < nq * k or c.size < nq):
+                raise ValueError("out arrays: u32[nq*k], f32[nq*k], u32[nq] required")
         _check(load_library().griffin_query_batch(self.h, nq, _ptr(off), _ptr(t), k, _ptr(d),
                                                   _ptr(s), _ptr(c)))
-        return d.reshape(nq, k), s.reshape(nq, k), c[:nq]
+        return d[:nq * k].reshape(nq, k), s[:nq * k].reshape(nq, k), c[:nq]
 
     # -- device-buffer API (torch tensors carry the device memory)
     def griffin_reserve(self, offsets, terms, k: int):

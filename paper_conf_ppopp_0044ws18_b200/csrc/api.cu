@@ -7,6 +7,7 @@
 #include <cmath>
 #include <cstring>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "internal.h"
@@ -16,6 +17,28 @@ namespace griffin {
 static thread_local std::string g_err;
 void set_error(const std::string &msg) { g_err = msg; }
 
+
+void par_memcpy(void *dst, const void *src, size_t bytes) {
+  constexpr size_t kSplit = 4u << 20;   // below this, one thread
+  const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+  const size_t nt = std::min<size_t>(std::min<size_t>(8, hw), bytes / kSplit);
+  if (nt <= 1) {
+    std::memcpy(dst, src, bytes);
+    return;
+  }
+  const size_t per = (bytes / nt + 63) & ~size_t(63);
+  std::vector<std::thread> th;
+  for (size_t t = 1; t < nt; ++t) {
+    const size_t a = t * per;
+    if (a >= bytes) break;
+    th.emplace_back([=] {
+      std::memcpy(static_cast<uint8_t *>(dst) + a, static_cast<const uint8_t *>(src) + a,
+                  std::min(per, bytes - a));
+    });
+  }
+  std::memcpy(dst, src, std::min(per, bytes));
+  for (auto &t : th) t.join();
+}
 
 static griffin_status invalid(const std::string &m) {
   set_error(m);
@@ -436,8 +459,8 @@ griffin_status griffin_query_batch(griffin_index *ix, uint32_t nq, const uint32_
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho + nk * 4, w.scores.p, nk * 4, cudaMemcpyDeviceToHost, st));
   GRIFFIN_CUDA_TRY(cudaMemcpyAsync(ho + nk * 8, w.counts.p, (size_t)nq * 4, cudaMemcpyDeviceToHost, st));
   if ((s = read_status(ix, ix->ws))) return s;  // synchronises
-  std::memcpy(out_docids, ho, nk * 4);
-  std::memcpy(out_scores, ho + nk * 4, nk * 4);
+  par_memcpy(out_docids, ho, nk * 4);
+  par_memcpy(out_scores, ho + nk * 4, nk * 4);
   std::memcpy(out_counts, ho + nk * 8, (size_t)nq * 4);
   return GRIFFIN_OK;
 }
@@ -786,8 +809,8 @@ griffin_status griffin_query_batch_collect(griffin_index *ix, griffin_workspace 
     }
   }
   if (w.pend_nq && copy) {
-    std::memcpy(out_docids, ho, nk * 4);
-    std::memcpy(out_scores, ho + nk * 4, nk * 4);
+    par_memcpy(out_docids, ho, nk * 4);
+    par_memcpy(out_scores, ho + nk * 4, nk * 4);
     std::memcpy(out_counts, ho + nk * 8, (size_t)w.pend_nq * 4);
   }
   // only now may a synchronous call on this workspace reuse the staging

@@ -366,8 +366,8 @@ griffin_status cluster_query_batch(griffin_index *cx, uint32_t nq, const uint32_
     set_error("invalid query term(s) detected on the device");
     return GRIFFIN_ERR_INVALID_ARG;
   }
-  std::memcpy(out_docids, h_doc, nk * 4);
-  std::memcpy(out_scores, h_sc, nk * 4);
+  par_memcpy(out_docids, h_doc, nk * 4);
+  par_memcpy(out_scores, h_sc, nk * 4);
   std::memcpy(out_counts, h_cnt, (size_t)nq * 4);
   return GRIFFIN_OK;
 }
