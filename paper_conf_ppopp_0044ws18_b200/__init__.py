@@ -130,10 +130,29 @@ _SIGS = {
 }
 
 
+def _nccl_hint():
+    """Point the library's run-time NCCL load (NCCL exchanges only) at the copy
+    PyTorch uses (the nvidia-nccl wheel) when present: the first libnccl.so.2
+    loaded into a process is the one every later user binds to."""
+    if os.environ.get("GRIFFIN_NCCL_LIBRARY"):
+        return
+    try:
+        import importlib.util
+        spec = importlib.util.find_spec("nvidia.nccl")
+        for d in (spec.submodule_search_locations or []) if spec else []:
+            p = os.path.join(d, "lib", "libnccl.so.2")
+            if os.path.exists(p):
+                os.environ["GRIFFIN_NCCL_LIBRARY"] = p
+                return
+    except (ImportError, ValueError):
+        pass
+
+
 def load_library():
     """Load libgriffin.so (building it in-tree with nvcc if it is missing or stale)."""
     global _lib
     if _lib is None:
+        _nccl_hint()
         alt = os.environ.get("GRIFFIN_LIBRARY")   # A/B runs: another build of the same ABI
         if alt:
             lib = ctypes.CDLL(alt)

@@ -18,16 +18,18 @@
 // global top-k key has < k larger keys globally, hence in its own shard, so it
 // is in that shard's top-k.
 //
-// NCCL is loaded at run time (dlopen libnccl.so.2): the library has no link-time
-// NCCL dependency, and a missing NCCL is reported as GRIFFIN_ERR_NCCL when an
-// NCCL exchange is requested.
+// NCCL is loaded at run time (dlopen of $GRIFFIN_NCCL_LIBRARY, else
+// libnccl.so.2): the library has no link-time NCCL dependency, and a missing
+// NCCL is reported as GRIFFIN_ERR_NCCL when an NCCL exchange is requested.
 #include <dlfcn.h>
 #include <nccl.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "internal.h"
@@ -51,7 +53,12 @@ static NcclApi &nccl() {
   static NcclApi api;
   static std::once_flag once;
   std::call_once(once, [] {
-    void *h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    // GRIFFIN_NCCL_LIBRARY first: the process may later load another NCCL user
+    // (PyTorch needs its own, newer libnccl.so.2; once a libnccl.so.2 is loaded
+    // every later user binds to it), so the binding points it at that copy
+    void *h = nullptr;
+    if (const char *p = std::getenv("GRIFFIN_NCCL_LIBRARY")) h = dlopen(p, RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
     if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
     if (!h) return;
 #define GRIFFIN_NCCL_SYM(f, n)                                  \
@@ -197,8 +204,10 @@ griffin_status cluster_query_batch(griffin_index *cx, uint32_t nq, const uint32_
   float *h_sc = reinterpret_cast<float *>(hr + nk * 4);
   uint32_t *h_cnt = reinterpret_cast<uint32_t *>(hr + nk * 8);
   int *h_status = reinterpret_cast<int *>(hr + nk * 8 + (size_t)nq * 4);
-  // ---- a1-a7 on every shard (asynchronous; the devices run concurrently) ----
-  for (uint32_t g = 0; g < G; ++g) {
+  // ---- a1-a7 on every shard (asynchronous; the devices run concurrently).
+  // Each shard's ~50 launches are issued by its own host thread, so no device
+  // waits for the host to finish issuing the other shards' work.
+  auto launch_shard = [&](uint32_t g) -> griffin_status {
     griffin_index *sh = cx->shards[g];
     DeviceGuard dg(sh->device);
     Workspace &w = sh->ws;
@@ -224,6 +233,25 @@ griffin_status cluster_query_batch(griffin_index *cx, uint32_t nq, const uint32_
     GRIFFIN_CUDA_TRY(cudaMemcpyAsync(h_status + g, w.scal.as<unsigned long long>() + kScalStatus,
                                      sizeof(int), cudaMemcpyDeviceToHost, st));
     GRIFFIN_CUDA_TRY(cudaEventRecord(cl->done[g], st));
+    return GRIFFIN_OK;
+  };
+  {
+    std::vector<griffin_status> st_g(G, GRIFFIN_OK);
+    std::vector<std::string> err_g(G);
+    std::vector<std::thread> th;
+    for (uint32_t g = 1; g < G; ++g)
+      th.emplace_back([&, g] {
+        st_g[g] = launch_shard(g);
+        if (st_g[g]) err_g[g] = griffin_last_error();   // thread-local message
+      });
+    st_g[0] = launch_shard(0);
+    if (st_g[0]) err_g[0] = griffin_last_error();
+    for (auto &t : th) t.join();
+    for (uint32_t g = 0; g < G; ++g)
+      if (st_g[g]) {
+        set_error("shard " + std::to_string(g) + ": " + err_g[g]);
+        return st_g[g];
+      }
   }
   // ---- a8: exchange the per-shard top-k runs and merge them ----
   griffin_index *s0 = cx->shards[0];
