@@ -177,7 +177,7 @@ griffin_status encode_index(griffin_index *ix, const uint32_t *h_doc, const uint
   GRIFFIN_CUDA_TRY(cudaMemsetAsync(ix->d_first, 0, (nb + 1) * 4, st));
   GRIFFIN_CUDA_TRY(cudaMemsetAsync(ix->d_meta, 0, (nb + 1) * 8, st));
   if (nb) {
-    encode_size_kernel<<<(unsigned)std::min<uint64_t>((nb + 255) / 256, 148 * 64), 256, 0, st>>>(
+    encode_size_kernel<<<(unsigned)std::min<uint64_t>((nb + 255) / 256, (uint64_t)num_sms(ix->device) * 64), 256, 0, st>>>(
         d_doc.as<uint32_t>(), d_bs.as<uint64_t>(), d_bn.as<uint32_t>(), nb, ix->d_first,
         ix->d_meta, d_size.as<uint32_t>());
     GRIFFIN_CUDA_TRY(cudaGetLastError());
@@ -201,11 +201,11 @@ griffin_status encode_index(griffin_index *ix, const uint32_t *h_doc, const uint
   if (nb) {
     const uint32_t stage_words = ((B * 34u) / 32u + 16u + 3u) & ~3u;
     const size_t smem = (size_t)stage_words * 4 * 8;
-    encode_write_kernel<<<(unsigned)std::min<uint64_t>((nb + 7) / 8, 148 * 16), 256, smem, st>>>(
+    encode_write_kernel<<<(unsigned)std::min<uint64_t>((nb + 7) / 8, (uint64_t)num_sms(ix->device) * 16), 256, smem, st>>>(
         d_doc.as<uint32_t>(), d_bs.as<uint64_t>(), d_off.as<uint64_t>(), nb, stage_words,
         ix->d_meta, ix->d_payload);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
-    tf_pack_kernel<<<(unsigned)std::min<uint64_t>((nb + 7) / 8, 148 * 16), 256, 0, st>>>(
+    tf_pack_kernel<<<(unsigned)std::min<uint64_t>((nb + 7) / 8, (uint64_t)num_sms(ix->device) * 16), 256, 0, st>>>(
         d_tf.as<uint32_t>(), d_bs.as<uint64_t>(), d_bn.as<uint32_t>(), d_bt.as<uint32_t>(),
         ix->d_terms, d_p0.as<uint64_t>(), nb, ix->d_tfw);
     GRIFFIN_CUDA_TRY(cudaGetLastError());

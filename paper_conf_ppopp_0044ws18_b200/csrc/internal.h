@@ -250,6 +250,10 @@ griffin_status launch_merge_topk_peer(griffin_index *ix, uint32_t G, uint32_t nq
 griffin_status reserve_for(griffin_index *ix, Workspace &w, uint32_t nq, const uint32_t *qoffs,
                            const uint32_t *terms, uint32_t k, uint32_t *max_terms);
 griffin_status ensure_pinned_ws(Workspace &w, size_t bytes);
+// SM count of a device (cached).
+int num_sms(int dev);
+// Process-wide dynamic-smem attribute (grow-only) + cached occupancy of a kernel.
+cudaError_t launch_config(const void *fn, int dev, size_t smem, int threads, int *per_sm);
 // Host copy of results out of pinned staging: large copies (a C5 batch's
 // 80 MB of docIDs + scores) are split over a few threads.
 void par_memcpy(void *dst, const void *src, size_t bytes);

@@ -340,7 +340,7 @@ griffin_status griffin_pfd_build(const griffin_corpus *c, uint32_t block_size, i
   PFD_TRY(cudaMalloc(&p->d_meta, (nb + 1) * 8));
   uint64_t total16 = 0;
   if (nb) {
-    pfd_size_kernel<<<(unsigned)std::min<uint64_t>((nb + 127) / 128, 148 * 64), 128, 0, st>>>(
+    pfd_size_kernel<<<(unsigned)std::min<uint64_t>((nb + 127) / 128, (uint64_t)num_sms(p->device) * 64), 128, 0, st>>>(
         d_doc.as<uint32_t>(), d_bs.as<uint64_t>(), d_bn.as<uint32_t>(), nb, p->d_first,
         p->d_meta, d_size.as<uint32_t>());
     PFD_TRY(cudaGetLastError());
@@ -353,7 +353,7 @@ griffin_status griffin_pfd_build(const griffin_corpus *c, uint32_t block_size, i
   PFD_TRY(cudaMalloc(&p->d_payload, (total16 + 64) * 16));
   PFD_TRY(cudaMemsetAsync(p->d_payload, 0, (total16 + 64) * 16, st));
   if (nb) {
-    pfd_write_kernel<<<(unsigned)std::min<uint64_t>((nb + 127) / 128, 148 * 64), 128, 0, st>>>(
+    pfd_write_kernel<<<(unsigned)std::min<uint64_t>((nb + 127) / 128, (uint64_t)num_sms(p->device) * 64), 128, 0, st>>>(
         d_doc.as<uint32_t>(), d_bs.as<uint64_t>(), d_off.as<uint64_t>(), nb, p->d_meta,
         reinterpret_cast<uint32_t *>(p->d_payload), d_cnt.as<unsigned long long>());
     PFD_TRY(cudaGetLastError());
@@ -445,9 +445,8 @@ griffin_status griffin_pfd_decode_list(griffin_pfd *p, uint32_t term, uint32_t *
     if (cudaMalloc(&d, nb * p->B * 4) != cudaSuccess) {
       rc = pfd_fail("out of device memory", GRIFFIN_ERR_OOM);
     } else {
-      cudaFuncSetAttribute(pfd_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           (int)smem);
-      pfd_decode_kernel<<<(unsigned)std::min<uint64_t>((nb + 7) / 8, 148 * 4), 256, smem,
+      launch_config((const void *)pfd_decode_kernel, p->device, smem, 256, nullptr);
+      pfd_decode_kernel<<<(unsigned)std::min<uint64_t>((nb + 7) / 8, (uint64_t)num_sms(p->device) * 4), 256, smem,
                           p->stream>>>(p->d_first, p->d_meta,
                                        reinterpret_cast<const uint32_t *>(p->d_payload), b0, nb,
                                        p->B, d, nullptr);
@@ -471,9 +470,8 @@ griffin_status griffin_pfd_decode_all(griffin_pfd *p, uint32_t iters, double *ms
   unsigned long long *acc = nullptr;
   cudaEvent_t a = nullptr, b = nullptr;
   const size_t smem = (size_t)(4 * p->B + 8) * 4 * kPfdWarps;
-  int per_sm = 1, nsm = 148;
-  cudaFuncSetAttribute(pfd_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, pfd_decode_kernel, 256, smem);
+  int per_sm = 1, nsm = 1;
+  launch_config((const void *)pfd_decode_kernel, p->device, smem, 256, &per_sm);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, p->device);
   const unsigned grid = (unsigned)std::max(1, nsm * std::max(1, per_sm));
   if (cudaMalloc(&acc, 3 * 8) != cudaSuccess) {

@@ -24,6 +24,10 @@
 //                  keys (score_bits << 32 | ~docID) (§3.1.3)
 #include <algorithm>
 #include <cstdio>
+#include <atomic>
+#include <map>
+#include <mutex>
+#include <tuple>
 
 #include <nvtx3/nvToolsExt.h>
 
@@ -2311,15 +2315,19 @@ __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t 
 
 // ------------------------------------------------------------------- host side
 
-static int num_sms(int dev) {
-  static int cache[64] = {0};
-  if (dev < 0 || dev >= 64) return 148;
-  if (!cache[dev]) {
-    int v = 0;
-    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
-    cache[dev] = v > 0 ? v : 148;
+int num_sms(int dev) {
+  static std::atomic<int> cache[64];   // zero-initialised; written by any launching thread
+  int v = 0;
+  if (dev < 0 || dev >= 64) {
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev < 0 ? 0 : dev);
+    return v > 0 ? v : 1;
   }
-  return cache[dev];
+  if (!(v = cache[dev].load(std::memory_order_relaxed))) {
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+    v = v > 0 ? v : 1;
+    cache[dev].store(v, std::memory_order_relaxed);
+  }
+  return v;
 }
 
 griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t units,
@@ -2396,22 +2404,41 @@ struct StageTimer {
   }
 };
 
+// Process-wide launch configuration of a kernel on a device: the dynamic
+// shared-memory attribute only ever grows (several host threads — the multi-GPU
+// handle's per-shard launchers — configure the same kernel for different block
+// sizes; a per-thread cache could shrink it under another thread's launch), and
+// the occupancy query runs once per (kernel, device, smem), not per launch.
+cudaError_t launch_config(const void *fn, int dev, size_t smem, int threads, int *per_sm) {
+  static std::mutex mu;
+  static std::map<std::pair<const void *, int>, size_t> attr;
+  static std::map<std::tuple<const void *, int, size_t>, int> occ;
+  std::lock_guard<std::mutex> lk(mu);
+  size_t &cur = attr[{fn, dev}];
+  if (cur < smem) {
+    const cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                               (int)smem);
+    if (e != cudaSuccess) return e;
+    cur = smem;
+  }
+  const auto key = std::make_tuple(fn, dev, smem);
+  auto it = occ.find(key);
+  if (it == occ.end()) {
+    int p = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&p, fn, threads, smem);
+    it = occ.emplace(key, std::max(1, p)).first;
+  }
+  if (per_sm) *per_sm = it->second;
+  return cudaSuccess;
+}
+
 template <bool RC>
 static cudaError_t launch_intersect(griffin_index *ix, const RoundArgs &ra, cudaStream_t st) {
   const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * kWarpsPerCta;
-  static thread_local int configured_dev[2] = {-1, -1};
-  static thread_local size_t configured_smem[2] = {0, 0};
-  if (configured_dev[RC] != ix->device || configured_smem[RC] < smem) {
-    cudaError_t e = cudaFuncSetAttribute(intersect_kernel<RC>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    configured_dev[RC] = ix->device;
-    configured_smem[RC] = smem;
-  }
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, intersect_kernel<RC>, kIntersectThreads,
-                                                smem);
-  per_sm = std::max(1, per_sm);
+  int per_sm = 1;
+  const cudaError_t e = launch_config((const void *)intersect_kernel<RC>, ix->device, smem,
+                                      kIntersectThreads, &per_sm);
+  if (e != cudaSuccess) return e;
   const int grid = num_sms(ix->device) * per_sm;
   intersect_kernel<RC><<<grid, kIntersectThreads, smem, st>>>(ix->dev(), ra);
   return cudaGetLastError();
@@ -2517,16 +2544,8 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
                                                     w.run_base.as<uint64_t>(),
                                                     w.run_term.as<uint32_t>());
     const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, Dsw, false) * 4 * 8;
-    static thread_local int cfg_dev = -1;
-    static thread_local size_t cfg_smem = 0;
-    if (cfg_dev != ix->device || cfg_smem < smem) {
-      GRIFFIN_CUDA_TRY(cudaFuncSetAttribute(decode_once_kernel,
-                                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      cfg_dev = ix->device;
-      cfg_smem = smem;
-    }
-    int per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, decode_once_kernel, 256, smem);
+    int per_sm = 1;
+    GRIFFIN_CUDA_TRY(launch_config((const void *)decode_once_kernel, ix->device, smem, 256, &per_sm));
     decode_once_kernel<<<num_sms(ix->device) * std::max(1, per_sm), 256, smem, st>>>(
         di, Dsw, w.run_base.as<uint64_t>(), w.run_term.as<uint32_t>(), w.arena.as<uint32_t>(),
         scal);
@@ -2631,7 +2650,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     topk_init_kernel<<<qblocks, 256, 0, st>>>(nq, rc, ts);
     ix->launch_count += 1;
     if (ts.fmax) {
-      topk_sample_kernel<<<std::min<uint32_t>(nq, 148 * 4), kTopkThreads, 0, st>>>(
+      topk_sample_kernel<<<std::min<uint32_t>(nq, num_sms(ix->device) * 4), kTopkThreads, 0, st>>>(
           di, nq, k, rs, w.cap_off.as<uint64_t>(), w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), ts);
       topk_filter_plan_kernel<<<qblocks, 256, 0, st>>>(nq, ts, nch);
       GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(nch, cbase, nq, scan_tmp, st, &ix->launch_count));
@@ -2650,7 +2669,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
       topk_update_kernel<<<qblocks, 256, 0, st>>>(nq, k, L, ts, nch, cbase);
       ix->launch_count += 3;
     }
-    topk_final_kernel<<<std::min<uint32_t>(nq, 148 * 4), kTopkThreads, 0, st>>>(
+    topk_final_kernel<<<std::min<uint32_t>(nq, num_sms(ix->device) * 4), kTopkThreads, 0, st>>>(
         di, nq, k, rc, rs, w.cap_off.as<uint64_t>(), w.rbuf0.as<uint2>(), w.rbuf1.as<uint2>(), ts,
         cb, d_keys, d_counts);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
@@ -2665,7 +2684,7 @@ griffin_status launch_merge_topk(griffin_index *ix, uint32_t G, uint32_t nq, uin
   if (nq == 0) return GRIFFIN_OK;
   StageTimer t(ix, st, 4);
   ix->launch_count += 1;
-  merge_topk_kernel<<<std::min<uint32_t>((nq + 7) / 8, 148 * 16), 256, 0, st>>>(
+  merge_topk_kernel<<<std::min<uint32_t>((nq + 7) / 8, num_sms(ix->device) * 16), 256, 0, st>>>(
       G, nq, k, d_keys, d_counts, d_out_keys, d_out_counts);
   GRIFFIN_CUDA_TRY(cudaGetLastError());
   return GRIFFIN_OK;
@@ -2698,7 +2717,7 @@ griffin_status launch_keys_to_results(griffin_index *ix, uint32_t nq, uint32_t k
   const uint64_t n = (uint64_t)nq * k;
   if (!n) return GRIFFIN_OK;
   ix->launch_count += 1;
-  keys_to_results_kernel<<<(unsigned)std::min<uint64_t>((n + 255) / 256, 148 * 32), 256, 0, st>>>(
+  keys_to_results_kernel<<<(unsigned)std::min<uint64_t>((n + 255) / 256, (uint64_t)num_sms(ix->device) * 32), 256, 0, st>>>(
       nq, k, d_keys, d_counts, d_docids, d_scores);
   GRIFFIN_CUDA_TRY(cudaGetLastError());
   return GRIFFIN_OK;
@@ -2709,10 +2728,9 @@ griffin_status launch_decode_list(griffin_index *ix, uint32_t term, uint32_t *d_
   const TermInfo &t = ix->h_terms[term];
   if (!t.nblocks) return GRIFFIN_OK;
   const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * 8;
-  GRIFFIN_CUDA_TRY(cudaFuncSetAttribute(decode_list_kernel,
-                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  GRIFFIN_CUDA_TRY(launch_config((const void *)decode_list_kernel, ix->device, smem, 256, nullptr));
   const uint32_t runs = (t.nblocks + ix->D + 1) / (ix->D + 2);
-  decode_list_kernel<<<std::min<uint32_t>((runs + 7) / 8, 148 * 8), 256, smem, st>>>(
+  decode_list_kernel<<<std::min<uint32_t>((runs + 7) / 8, num_sms(ix->device) * 8), 256, smem, st>>>(
       ix->dev(), ix->D, t.block0, t.nblocks, d_out);
   GRIFFIN_CUDA_TRY(cudaGetLastError());
   return GRIFFIN_OK;
@@ -2722,10 +2740,8 @@ griffin_status launch_decode_all(griffin_index *ix, unsigned long long *d_acc, c
   if (!ix->nblocks) return GRIFFIN_OK;
   const uint32_t Dsw = sweep_D(ix->B);
   const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, Dsw, false) * 4 * 8;
-  GRIFFIN_CUDA_TRY(cudaFuncSetAttribute(decode_all_kernel,
-                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, decode_all_kernel, 256, smem);
+  int per_sm = 1;
+  GRIFFIN_CUDA_TRY(launch_config((const void *)decode_all_kernel, ix->device, smem, 256, &per_sm));
   ix->launch_count += 1;
   decode_all_kernel<<<num_sms(ix->device) * std::max(1, per_sm), 256, smem, st>>>(
       ix->dev(), Dsw, ix->nblocks, d_acc);

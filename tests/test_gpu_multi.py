@@ -94,3 +94,15 @@ def test_multi_gpu_distinct_devices_all_exchanges(small):
         gx = g.GriffinIndex(c, block_size=128, num_gpus=G, exchange=ex)
         _check(gx, ox, ql, 100)
         gx.close()
+
+
+def test_launch_config_shared_across_threads(small):
+    """Shard launcher threads configure kernels for their block size; that must
+    never shrink the shared-memory limit a larger configuration on another
+    thread relies on (regression: a per-thread cache did)."""
+    c, ql, ox = small
+    gx = g.GriffinIndex(c, block_size=64, num_gpus=4, devices=[0] * 4)
+    _check(gx, ox, ql, 10)   # worker threads configure B = 64
+    big = g.GriffinIndex(c, block_size=128)
+    _check(big, ox, ql, 10)  # main thread, larger shared memory per CTA
+    _check(gx, ox, ql, 10)
