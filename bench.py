@@ -423,7 +423,9 @@ def run_gpu(args):
     kernels = {
         "intersect_kernel": kern(prof["ms_intersect"], prof["alg_bytes"], prof["c8d_bytes"],
                                  prof["launches_intersect"], prof["decoded_postings"],
-                                 "fused EF decode + merge-path/gallop intersection + BM25 (all SvS rounds)"),
+                                 "SvS rounds: intersect_kernel (round 1: fused EF decode / arena tiles + "
+                                 "merge-path or gallop intersection + BM25) and probe_kernel (rounds "
+                                 "2..m-1 as one multi-list probe pass)"),
         "decode_once_kernel": kern(prof["ms_decode"], prof["dec_alg_bytes"],
                                    prof["dec_c8d_bytes"], prof["launches_decode"],
                                    prof["dec_postings"],

@@ -283,6 +283,17 @@ struct WarpSmem {
   uint32_t phase;
 };
 
+// Probe-pass kernel layout: the probe unit's tile region holds its survivor
+// chunk (tileR, scores, norms, block ids, matches: 5B words) plus, only when
+// galloping into compressed lists decodes blocks (NextGEQ off), G = D-3 decoded
+// S blocks.
+__host__ __device__ inline uint32_t probe_tile_words(uint32_t B, uint32_t D, bool nextgeq) {
+  return 5u * B + (nextgeq ? 0u : (D - 3u) * B) + kTileSlack;
+}
+__host__ __device__ inline uint32_t probe_warp_smem_words(uint32_t B, uint32_t D, bool nextgeq) {
+  return kWarpHdr + 64 + (B + 32) + stage_words(B, D) + kStgSlack + probe_tile_words(B, D, nextgeq);
+}
+
 __device__ __forceinline__ WarpSmem carve_warp_smem(uint4 *smem4, uint32_t B, uint32_t D,
                                                     bool with_tile = true) {
   uint8_t *base = reinterpret_cast<uint8_t *>(smem4);
@@ -1619,6 +1630,56 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
   }
 }
 
+// SvS rounds 2..m-1 as one multi-list probe pass: its own kernel,
+// so it carries only the probe unit's code and shared memory (no merge tiles)
+// and runs 4 CTAs of 8 warps per SM — the pass is global-latency bound
+// (skip-pointer searches and arena probes), so more resident warps hide more.
+__global__ void __launch_bounds__(kIntersectThreads, 4) probe_kernel(DevIndex ix, RoundArgs a) {
+  extern __shared__ uint4 smem4[];
+  const uint32_t lane = lane_id();
+  const uint32_t B = ix.B, D = a.D;
+  uint8_t *base = reinterpret_cast<uint8_t *>(smem4);
+  WarpSmem sm;
+  sm.lut = base;
+  uint32_t *wb = reinterpret_cast<uint32_t *>(base + kLutBytes) +
+                 (threadIdx.x >> 5) * probe_warp_smem_words(B, D, a.nextgeq != 0);
+  sm.mbar = reinterpret_cast<uint64_t *>(wb);
+  sm.cnt = wb + kWarpHdr;
+  sm.aux = sm.cnt + 64;
+  sm.stg = sm.aux + B + 32;
+  sm.tile = sm.stg + stage_words(B, D) + kStgSlack;
+  sm.phase = 0;
+  cta_smem_init(smem4, sm);
+  const uint64_t total = a.unit_base[a.nq];
+  Acc acc;
+  acc.bleft = reinterpret_cast<uint32_t *>(sm.mbar) + 2;
+  acc.boff = reinterpret_cast<unsigned long long *>(sm.mbar) + 2;
+  acc.ctr = reinterpret_cast<unsigned long long *>(sm.mbar) + 4;
+  if (lane == 0) {
+    *acc.bleft = 0;
+    *acc.boff = 0;
+#pragma unroll
+    for (int c = 0; c < kCNum; ++c) acc.ctr[c] = 0;
+  }
+  unsigned long long ticket = 0;
+  if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
+  for (;;) {
+    const uint64_t tk = __shfl_sync(0xffffffffu, ticket, 0);
+    if (tk >= total) break;
+    if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
+    const uint64_t u = a.uperm[tk];
+    const uint4 rec = a.urec[u];
+    probe_unit(ix, a, sm, u, rec.x, rec.y, acc);   // every unit of the pass is a probe unit
+  }
+  if (lane == 0) {
+    const int slot[kCNum] = {kScalCounters, kScalCounters + 1, kScalCounters + 2,
+                             kScalCounters + 3, kScalArena, kScalArena + 1};
+#pragma unroll
+    for (int c = 0; c < kCNum; ++c)
+      if (acc.ctr[c]) atomicAdd(a.scal + slot[c], acc.ctr[c]);
+  }
+}
+
 // ------------------------------------------------------------------- compaction
 
 // Global exclusive scan of the per-unit survivor counts (n = total units, read
@@ -2444,6 +2505,17 @@ static cudaError_t launch_intersect(griffin_index *ix, const RoundArgs &ra, cuda
   return cudaGetLastError();
 }
 
+static cudaError_t launch_probe(griffin_index *ix, const RoundArgs &ra, cudaStream_t st) {
+  const size_t smem = kLutBytes + (size_t)probe_warp_smem_words(ix->B, ix->D, ra.nextgeq != 0) *
+                                      4 * kWarpsPerCta;
+  int per_sm = 1;
+  const cudaError_t e = launch_config((const void *)probe_kernel, ix->device, smem,
+                                      kIntersectThreads, &per_sm);
+  if (e != cudaSuccess) return e;
+  probe_kernel<<<num_sms(ix->device) * per_sm, kIntersectThreads, smem, st>>>(ix->dev(), ra);
+  return cudaGetLastError();
+}
+
 // Top-k candidate buffers for a batch of nq queries with this k (grow-only;
 // called before a CUDA-graph capture so no allocation happens inside it).
 // Pre-filter policy: always for k > 64 (one chunk level keeps k of kTopkSmem
@@ -2598,6 +2670,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
         ix->launch_count += 1;
       }
       if (r == 1) GRIFFIN_CUDA_TRY(launch_intersect<true>(ix, ra, st));
+      else if (ra.probe) GRIFFIN_CUDA_TRY(launch_probe(ix, ra, st));   // all units are probe units
       else GRIFFIN_CUDA_TRY(launch_intersect<false>(ix, ra, st));
       ix->launch_count += 2;  // partition + intersect
     }

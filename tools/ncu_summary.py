@@ -73,7 +73,7 @@ for r in rows[2:]:
 lines.append("")
 for idx in range(len(rows) - 2):
     name = rows[2 + idx][hdr.index("Kernel Name")]
-    if "intersect" in name or "decode" in name:
+    if "intersect" in name or "decode" in name or "probe" in name:
         src = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_lines2.py"), rep,
                               str(idx), "12"], capture_output=True, text=True).stdout
         lines.append(f"## top source lines, launch {idx}: {name.split('(')[0]}")
@@ -85,9 +85,11 @@ with open(os.path.join(ROOT, "profiles", f"{tag}_ncu_kernels.txt"), "w") as f:
 summ = {"source": os.path.basename(rep), "config": config,
         "dram_bytes_per_launch": {k: sum(v) / len(v) for k, v in per_kernel.items()}}
 # bench.py keys
-summ["dram_bytes_per_launch"]["intersect_kernel"] = (
-    sum(per_kernel.get("intersect_kernel<1>", []) + per_kernel.get("intersect_kernel<0>", [])) /
-    max(1, len(per_kernel.get("intersect_kernel<1>", []) + per_kernel.get("intersect_kernel<0>", []))))
+# the intersect stage = round 1 (intersect_kernel<1>) + the later rounds (the
+# probe pass probe_kernel, or intersect_kernel<0> without it)
+_ik = (per_kernel.get("intersect_kernel<1>", []) + per_kernel.get("intersect_kernel<0>", []) +
+       per_kernel.get("probe_kernel", []))
+summ["dram_bytes_per_launch"]["intersect_kernel"] = sum(_ik) / max(1, len(_ik))
 with open(os.path.join(ROOT, "profiles", f"ncu_summary_{config}.json"), "w") as f:
     json.dump(summ, f, indent=1)
 print("\n".join(lines))
