@@ -95,7 +95,8 @@ enum : int {
   kScalDecC8d = 17,   // u64: decode-once compressed bytes read (payload + skip/meta)
   kScalRoundTot = 18, // u64: survivors of the current round (compaction scan total)
   kScalDiag = 19,     // 4 x u64 (counting mode): merge units, merged elements, gallop units, galloped elements
-  kScalCount = 23
+  kScalUnitCtr2 = 23, // u64 ticket counter of the round-1 gallop/single-term kernel
+  kScalCount = 24
 };
 
 constexpr uint32_t kBumpChunk = 256;   // bump-area entries grabbed per warp atomic

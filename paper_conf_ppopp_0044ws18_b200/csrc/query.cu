@@ -158,6 +158,7 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
   if (q == 0) {
     a.scal[kScalBump] = 0;
     a.scal[kScalUnitCtr] = 0;
+    a.scal[kScalUnitCtr2] = 0;
     a.scal[kScalPerm] = 0;
     a.scal[kScalPerm + 1] = 0;
     if (overflow) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
@@ -1119,17 +1120,48 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
 }
 
 
-template <bool RC>
+// Round-1 unit kinds run as two kernels, back to back (ROLE): 1 = the merge
+// units (the processing order puts them first: tickets [0, #merge)), 2 = the
+// gallop and single-term units (tickets [#merge, total)) with a smaller shared
+// layout (no merge tiles) and 4 CTAs/SM — they are global-latency bound
+// (skip searches, arena probes).  ROLE 0 = every unit kind in one kernel (the SvS
+// rounds without the probe pass).
 #ifndef GRIFFIN_INTERSECT_MINB
 #define GRIFFIN_INTERSECT_MINB 3
 #endif
-__global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) intersect_kernel(DevIndex ix, RoundArgs a) {
+__host__ __device__ inline uint32_t other_tile_words(uint32_t B, uint32_t D, bool nextgeq) {
+  const uint32_t G = (D - 1u) < 31u ? D - 1u : 31u;
+  return 3u * B + (nextgeq ? 0u : G * B) + kTileSlack;
+}
+__host__ __device__ inline uint32_t other_warp_smem_words(uint32_t B, uint32_t D, bool nextgeq) {
+  return kWarpHdr + 64 + (B + 32) + stage_words(B, D) + kStgSlack + other_tile_words(B, D, nextgeq);
+}
+template <int ROLE>
+struct IkMinBlocks { static constexpr int v = ROLE == 2 ? 4 : GRIFFIN_INTERSECT_MINB; };
+
+template <bool RC, int ROLE>
+__global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) intersect_kernel(DevIndex ix, RoundArgs a) {
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
   const uint32_t B = ix.B, D = a.D;
-  WarpSmem sm = carve_warp_smem(smem4, B, D);
+  WarpSmem sm;
+  if (ROLE == 2) {
+    uint8_t *base = reinterpret_cast<uint8_t *>(smem4);
+    sm.lut = base;
+    uint32_t *wb = reinterpret_cast<uint32_t *>(base + kLutBytes) +
+                   (threadIdx.x >> 5) * other_warp_smem_words(B, D, a.nextgeq != 0);
+    sm.mbar = reinterpret_cast<uint64_t *>(wb);
+    sm.cnt = wb + kWarpHdr;
+    sm.aux = sm.cnt + 64;
+    sm.stg = sm.aux + B + 32;
+    sm.tile = sm.stg + stage_words(B, D) + kStgSlack;
+    sm.phase = 0;
+  } else {
+    sm = carve_warp_smem(smem4, B, D);
+  }
   cta_smem_init(smem4, sm);
-  const uint64_t total = a.unit_base[a.nq];
+  const uint64_t nmerge = a.scal[kScalPerm];   // merge units: tickets [0, nmerge)
+  const uint64_t total = ROLE == 1 ? nmerge : a.unit_base[a.nq];
   const uint32_t G = min(D - 1u, 31u);   // gallop: S blocks staged per group
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   Acc acc;
@@ -1145,12 +1177,14 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
   // dynamic unit tickets (balances long gallop/probe units); the next ticket is
   // requested at the start of a unit so its latency overlaps the unit's work
   unsigned long long ticket = 0;
-  if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
+  unsigned long long *ctr = a.scal + (ROLE == 2 ? kScalUnitCtr2 : kScalUnitCtr);
+  const uint64_t tk0 = ROLE == 2 ? nmerge : 0ull;
+  if (lane == 0) ticket = tk0 + atomicAdd(ctr, 1ull);
   (void)nwarps;
   for (;;) {
     const uint64_t tk = __shfl_sync(0xffffffffu, ticket, 0);
     if (tk >= total) break;
-    if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
+    if (lane == 0) ticket = tk0 + atomicAdd(ctr, 1ull);
     const uint64_t u = a.uperm[tk];   // merge units first (see partition_kernel)
     const uint4 rec = a.urec[u];
     const uint4 nxt = a.urec[u + 1];
@@ -1167,7 +1201,7 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
     const bool rdec = RC && a.tdec && a.tdec[t0];
     const uint32_t *decR = rdec ? a.dec + (size_t)tR.block0 * B : nullptr;
 
-    if (RC && mode == kModeAll) {  // single-term query: the whole list is the result
+    if (ROLE != 1 && RC && mode == kModeAll) {  // single-term query: the whole list is the result
       const uint32_t n = min(B, nR - lu * B);
       if (rdec) {
         if (lane == 0) {
@@ -1198,7 +1232,7 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
       emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, 0, n, lu * B, acc);
       continue;
     }
-    if (!RC && mode == kModeProbe) {
+    if (ROLE == 0 && !RC && mode == kModeProbe) {
       probe_unit(ix, a, sm, u, q, lu, acc);
       continue;
     }
@@ -1209,7 +1243,7 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
     const bool sdec = a.tdec && a.tdec[tSid];
     const uint32_t *decS = sdec ? a.dec + (size_t)tS.block0 * B : nullptr;
 
-    if (mode == kModeMerge) {
+    if (ROLE != 2 && (ROLE == 1 || mode == kModeMerge)) {
       // ---- the unit's docID range [lo, hi) and block ranges, from the partition
       // stage's merge-path crossings (unit u and unit u+1) ----
       const uint32_t i0 = rec.y, j0 = rec.z;
@@ -1417,7 +1451,7 @@ __global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_INTERSECT_MINB) int
                           sb0 * B + sa, smem_u32(sm.tile) & 0xFFFFu,
                           smem_u32(tileS + sa) & 0xFFFFu, acc);
       __syncwarp();
-    } else {
+    } else if (ROLE != 1) {
       // ---- gallop: R chunk lu, skip-pointer search into S (Fig. 9) ----
       uint32_t *tileR = sm.tile, *kidx = sm.tile + B, *match = sm.tile + 2 * B;
       uint32_t *tileS = sm.tile + 3 * B;
@@ -2493,15 +2527,17 @@ cudaError_t launch_config(const void *fn, int dev, size_t smem, int threads, int
   return cudaSuccess;
 }
 
-template <bool RC>
+template <bool RC, int ROLE>
 static cudaError_t launch_intersect(griffin_index *ix, const RoundArgs &ra, cudaStream_t st) {
-  const size_t smem = kLutBytes + (size_t)warp_smem_words(ix->B, ix->D) * 4 * kWarpsPerCta;
+  const size_t words = ROLE == 2 ? other_warp_smem_words(ix->B, ix->D, ra.nextgeq != 0)
+                                 : warp_smem_words(ix->B, ix->D);
+  const size_t smem = kLutBytes + words * 4 * kWarpsPerCta;
   int per_sm = 1;
-  const cudaError_t e = launch_config((const void *)intersect_kernel<RC>, ix->device, smem,
+  const cudaError_t e = launch_config((const void *)intersect_kernel<RC, ROLE>, ix->device, smem,
                                       kIntersectThreads, &per_sm);
   if (e != cudaSuccess) return e;
   const int grid = num_sms(ix->device) * per_sm;
-  intersect_kernel<RC><<<grid, kIntersectThreads, smem, st>>>(ix->dev(), ra);
+  intersect_kernel<RC, ROLE><<<grid, kIntersectThreads, smem, st>>>(ix->dev(), ra);
   return cudaGetLastError();
 }
 
@@ -2669,9 +2705,15 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
         sorder_scatter_kernel<<<pgrid, 256, 0, st>>>(di, ra);
         ix->launch_count += 1;
       }
-      if (r == 1) GRIFFIN_CUDA_TRY(launch_intersect<true>(ix, ra, st));
-      else if (ra.probe) GRIFFIN_CUDA_TRY(launch_probe(ix, ra, st));   // all units are probe units
-      else GRIFFIN_CUDA_TRY(launch_intersect<false>(ix, ra, st));
+      if (r == 1) {   // merge units, then gallop / single-term units
+        GRIFFIN_CUDA_TRY((launch_intersect<true, 1>(ix, ra, st)));
+        GRIFFIN_CUDA_TRY((launch_intersect<true, 2>(ix, ra, st)));
+        ix->launch_count += 1;
+      } else if (ra.probe) {
+        GRIFFIN_CUDA_TRY(launch_probe(ix, ra, st));   // all units are probe units
+      } else {
+        GRIFFIN_CUDA_TRY((launch_intersect<false, 0>(ix, ra, st)));
+      }
       ix->launch_count += 2;  // partition + intersect
     }
     {

@@ -85,11 +85,14 @@ with open(os.path.join(ROOT, "profiles", f"{tag}_ncu_kernels.txt"), "w") as f:
 summ = {"source": os.path.basename(rep), "config": config,
         "dram_bytes_per_launch": {k: sum(v) / len(v) for k, v in per_kernel.items()}}
 # bench.py keys
-# the intersect stage = round 1 (intersect_kernel<1>) + the later rounds (the
-# probe pass probe_kernel, or intersect_kernel<0> without it)
-_ik = (per_kernel.get("intersect_kernel<1>", []) + per_kernel.get("intersect_kernel<0>", []) +
-       per_kernel.get("probe_kernel", []))
-summ["dram_bytes_per_launch"]["intersect_kernel"] = sum(_ik) / max(1, len(_ik))
+# the intersect stage = round 1 (intersect_kernel<1, 1> merge units followed by
+# intersect_kernel<1, 2> gallop/single-term units: ONE timed stage section) + the
+# later rounds (the probe pass probe_kernel, or intersect_kernel<0, 0> without
+# it). Per stage section, like bench.py's launch count (launches_intersect).
+_stage = [k for k in per_kernel if k.startswith("intersect_kernel") or k == "probe_kernel"]
+_bytes = sum(sum(per_kernel[k]) for k in _stage)
+_sections = sum(len(per_kernel[k]) for k in _stage if not k.replace(" ", "").endswith(",2>"))
+summ["dram_bytes_per_launch"]["intersect_kernel"] = _bytes / max(1, _sections)
 with open(os.path.join(ROOT, "profiles", f"ncu_summary_{config}.json"), "w") as f:
     json.dump(summ, f, indent=1)
 print("\n".join(lines))
