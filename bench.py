@@ -288,6 +288,7 @@ def run_gpu(args):
     build_s = time.time() - t0
     st = ix.griffin_index_stats()
     ix.griffin_set_reuse({"auto": 2, "on": 1, "off": 0}[args.reuse])
+    ix.griffin_set_bitmap(args.bitmap)
     # intermediate capacity per workspace buffer: packed by actual survivors, so a
     # budget well under the sum of per-query bounds holds a batch (C5: ~1e9 bound)
     budget = args.entry_budget if args.entry_budget is not None else \
@@ -404,7 +405,7 @@ def run_gpu(args):
     cnt = ix.griffin_get_profile()
     for kk in ("alg_bytes", "c8d_bytes", "payload_bytes", "decoded_postings", "survivors",
                "dec_alg_bytes", "dec_c8d_bytes", "dec_postings", "arena_postings", "merge_units",
-               "merge_elems", "gallop_units", "gallop_elems"):
+               "merge_elems", "gallop_units", "gallop_elems", "bitmap_units", "bitmap_elems"):
         prof[kk] = cnt[kk]
     ix.griffin_sync_status()
     iso_ms = sum(iso)
@@ -424,17 +425,19 @@ def run_gpu(args):
         "intersect_kernel": kern(prof["ms_intersect"], prof["alg_bytes"], prof["c8d_bytes"],
                                  prof["launches_intersect"], prof["decoded_postings"],
                                  "SvS rounds: intersect_kernel (round 1: fused EF decode / arena tiles + "
-                                 "merge-path or gallop intersection + BM25) and probe_kernel (rounds "
+                                 "merge-path, gallop or bitvector-lookup intersection + BM25) and probe_kernel (rounds "
                                  "2..m-1 as one multi-list probe pass)"),
         "decode_once_kernel": kern(prof["ms_decode"], prof["dec_alg_bytes"],
                                    prof["dec_c8d_bytes"], prof["launches_decode"],
                                    prof["dec_postings"],
-                                   "batch decode-once: Para-EF decode of hot lists into the HBM arena"),
+                                   "batch decode-once: Para-EF decode of hot lists into the HBM arena "
+                                   "(dense lists into a bitvector + rank)"),
     }
     kernels["intersect_kernel"]["survivors_per_step"] = prof["survivors"] / n_iso
     kernels["intersect_kernel"]["arena_postings_per_step"] = prof["arena_postings"] / n_iso
     kernels["intersect_kernel"]["units_per_step"] = {
-        kk: prof[kk] / n_iso for kk in ("merge_units", "merge_elems", "gallop_units", "gallop_elems")}
+        kk: prof[kk] / n_iso for kk in ("merge_units", "merge_elems", "gallop_units", "gallop_elems",
+                                        "bitmap_units", "bitmap_elems")}
     stage_ms = {kk: prof[kk] / n_iso for kk in
                 ("ms_plan", "ms_decode", "ms_intersect", "ms_compact", "ms_topk", "ms_merge")}
     dom = max(kernels, key=lambda n: kernels[n]["ms_per_step"])
@@ -545,7 +548,8 @@ def run_gpu(args):
         "batches_in_flight": len(slots),
         "index": {"bytes_per_shard": st["payload_bytes"] + st["skip_bytes"] + st["tf_bytes"],
                   "payload_bytes": st["payload_bytes"], "build_s": build_s,
-                  "corpus_load_s": gen_s, "reuse": args.reuse, "entry_budget": budget},
+                  "corpus_load_s": gen_s, "reuse": args.reuse, "bitmap_inv": args.bitmap,
+                  "entry_budget": budget},
         "decoded_postings_per_s": decoded_ps * world,
         "sync_qps": {"value": nq / (statistics.median(sync_ms) / 1e3) if sync_ms else None,
                      "unit": "queries/s", "median_ms": statistics.median(sync_ms) if sync_ms else None,
@@ -621,6 +625,8 @@ def main():
                     help="batches in flight on separate streams/workspaces (N=1 only); default 3")
     ap.add_argument("--reuse", default="auto", choices=["auto", "on", "off"],
                     help="batch decode-once of hot lists into an HBM arena")
+    ap.add_argument("--bitmap", type=int, default=32,
+                    help="dense lists (density >= 1/INV) decoded once per batch into a bitvector; 0 = off")
     ap.add_argument("--shard-mode", default="docid", choices=["docid", "replicate"],
                     help="N>1: docID-range shards + exchange, or a replicated index per rank")
     ap.add_argument("--exchange", default="allgather", choices=["allgather", "sliced"],

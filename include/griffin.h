@@ -166,6 +166,8 @@ typedef struct {
   /* unit shapes (counters mode): merge units and the elements they merged (R+S
    * inside their docID ranges), gallop units and their R elements */
   uint64_t merge_units, merge_elems, gallop_units, gallop_elems;
+  /* bitvector units (griffin_set_bitmap) and their R elements looked up */
+  uint64_t bitmap_units, bitmap_elems;
 } griffin_profile;
 
 /* ---- index ------------------------------------------------------------------
@@ -293,6 +295,17 @@ griffin_status griffin_set_profiling(griffin_index *ix, int on);
  * EF-decoded once per batch into an HBM arena (the paper's decompress-then-
  * intersect pipeline, Alg. 1 output `decmp_array`) and intersected from there. */
 griffin_status griffin_set_reuse(griffin_index *ix, int mode);
+/* Dense lists in the decode-once stage: a list selected for decode-once whose
+ * density in the shard is >= 1/inv (df_local * inv >= shard docs) is decoded
+ * into a docID bitvector with rank — per 32 docs one u64 word {bits, position
+ * of the word's first posting} — instead of the docID arena (for density >=
+ * 1/32 it is the smaller of the two).  An intersection round whose longer
+ * list S has one then looks each R element up in O(1) (bit test; the rank
+ * gives the posting position for S's tf) instead of merging or galloping
+ * through S: the SvS result set and every score are unchanged,
+ * only the work differs.  Default inv = 32; 0 turns the bitvectors off.
+ * Forced merge / gallop modes (griffin_set_mode) never use them. */
+griffin_status griffin_set_bitmap(griffin_index *ix, uint32_t inv);
 /* Galloping into a compressed (not arena-decoded) list: 1 = EF NextGEQ (default;
  * select0 over the staged block's unary high stream finds the bucket of the
  * probe's high part, only that bucket's few elements are decoded — SURVEY

@@ -76,7 +76,8 @@ class Profile(ctypes.Structure):
                 ("c8d_bytes", ctypes.c_uint64), ("dec_c8d_bytes", ctypes.c_uint64),
                 ("arena_postings", ctypes.c_uint64), ("merge_units", ctypes.c_uint64),
                 ("merge_elems", ctypes.c_uint64), ("gallop_units", ctypes.c_uint64),
-                ("gallop_elems", ctypes.c_uint64)]
+                ("gallop_elems", ctypes.c_uint64),
+                ("bitmap_units", ctypes.c_uint64), ("bitmap_elems", ctypes.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -108,6 +109,7 @@ _SIGS = {
     "griffin_set_profiling": [_vp, ctypes.c_int],
     "griffin_set_reuse": [_vp, ctypes.c_int],
     "griffin_set_nextgeq": [_vp, ctypes.c_int],
+    "griffin_set_bitmap": [_vp, _u32],
     "griffin_set_probe_chunk": [_vp, _u32],
     "griffin_set_entry_budget": [_vp, _u64],
     "griffin_pfd_build": [_vp, _u32, ctypes.c_int, _vp],
@@ -412,6 +414,11 @@ class GriffinIndex:
     def griffin_set_reuse(self, mode: int):
         """0 off (fused decode every round), 1 on (decode hot lists once per batch), 2 auto."""
         _check(load_library().griffin_set_reuse(self.h, mode))
+
+    def griffin_set_bitmap(self, inv: int):
+        """Dense lists (density >= 1/inv) decoded once per batch into a bitvector
+        + rank instead of the docID arena; 0 off, default 32."""
+        _check(load_library().griffin_set_bitmap(self.h, inv))
 
     def griffin_set_nextgeq(self, on: bool):
         """Gallop into compressed lists by EF NextGEQ (True, default) or block decode."""

@@ -363,6 +363,8 @@ void griffin_index_destroy(griffin_index *ix) {
     cudaFree(ix->d_payload);
     cudaFree(ix->d_tfw);
     cudaFree(ix->d_norm);
+    cudaFree(ix->d_bm_slot);
+    cudaFree(ix->d_bm_term);
     for (Workspace *xw : ix->extra_ws) {
       free_workspace(*xw);
       delete xw;
@@ -472,7 +474,7 @@ static uint64_t ws_identity(const Workspace &w) {
                           &w.qmode, &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.uperm,
                           &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys,
                           &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand,
-                          &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.run_term, &w.arena})
+                          &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.run_term, &w.arena, &w.bmap})
     h = (h ^ (uint64_t)(uintptr_t)b->p) * 1099511628211ull;
   // capacities are baked into a captured graph's kernel arguments too
   for (const uint64_t v : {(uint64_t)w.nq_cap, (uint64_t)w.unit_cap, (uint64_t)w.entry_cap,
@@ -639,7 +641,7 @@ static void free_workspace(Workspace &w) {
                     &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.uperm, &w.rbuf0,
                     &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys, &w.counts,
                     &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand, &w.tdec, &w.runs,
-                    &w.run_base, &w.vtmp, &w.run_term, &w.arena, &w.sbkt_cnt, &w.sbkt_pos,
+                    &w.run_base, &w.vtmp, &w.run_term, &w.arena, &w.bmap, &w.sbkt_cnt, &w.sbkt_pos,
                     &w.sbkt_tmp, &w.flt, &w.fstate})
     b->release();
   if (w.h_pinned) cudaFreeHost(w.h_pinned);
@@ -872,6 +874,20 @@ griffin_status griffin_set_reuse(griffin_index *ix, int mode) {
   return GRIFFIN_OK;
 }
 
+griffin_status griffin_set_bitmap(griffin_index *ix, uint32_t inv) {
+  if (ix && ix->cl) {   // multi-GPU handle: every shard
+    for (griffin_index *sh : ix->shards) {
+      griffin_status s = griffin_set_bitmap(sh, inv);
+      if (s) return s;
+    }
+    return GRIFFIN_OK;
+  }
+  if (!ix) return invalid("null index");
+  std::lock_guard<std::mutex> lk(ix->mu);
+  ix->bm_inv = inv;
+  return GRIFFIN_OK;
+}
+
 griffin_status griffin_set_nextgeq(griffin_index *ix, int on) {
   if (ix && ix->cl) {   // multi-GPU handle: every shard
     for (griffin_index *sh : ix->shards) {
@@ -955,6 +971,7 @@ griffin_status griffin_reset_profile(griffin_index *ix) {
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDec, 0, 3 * 8));
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalArena, 0, 3 * 8));
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDiag, 0, 4 * 8));
+      GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDiag2, 0, 2 * 8));
     }
   return GRIFFIN_OK;
 }
@@ -985,6 +1002,7 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
   out->dec_alg_bytes = out->dec_payload_bytes = out->dec_postings = 0;
   out->c8d_bytes = out->dec_c8d_bytes = out->arena_postings = 0;
   out->merge_units = out->merge_elems = out->gallop_units = out->gallop_elems = 0;
+  out->bitmap_units = out->bitmap_elems = 0;
   for (Workspace *w : all) {
     if (!w->scal.p) continue;
     unsigned long long c[kScalCount];
@@ -1003,6 +1021,8 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
     out->merge_elems += c[kScalDiag + 1];
     out->gallop_units += c[kScalDiag + 2];
     out->gallop_elems += c[kScalDiag + 3];
+    out->bitmap_units += c[kScalDiag2];
+    out->bitmap_elems += c[kScalDiag2 + 1];
   }
   return GRIFFIN_OK;
 }

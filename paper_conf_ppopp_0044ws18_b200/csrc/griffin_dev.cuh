@@ -152,6 +152,63 @@ struct XorSink {
   __device__ __forceinline__ void put4(uint32_t *, uint4 v) { x ^= v.x ^ v.y ^ v.z ^ v.w; }
   __device__ __forceinline__ void put(uint32_t *, uint32_t v) { x ^= v; }
 };
+// BitSink writes a list's decoded docIDs into its bitvector with rank: word
+// w = {bits of docs [32w, 32w+32), ~(list position of the word's first
+// posting)} (the rank is only read where a bit is set).  The decoder hands
+// each lane its elements in list order; a lane ORs a run of elements that
+// share a word into a register and writes the word once.  A run whose
+// neighbours on both sides were decoded by this lane, in other words, owns
+// the word outright (plain 64-bit store); any other run may share its word
+// with another lane: atomicOr for the bits, atomicMax of ~position (= the
+// smallest position) for the rank — the area is zeroed first.  Positions come
+// from the output pointer: the decoder writes element i of the run at tile + i.
+struct BitSink {
+  uint2 *bm;              // the list's bitvector
+  const uint32_t *tile;   // decoder destination base
+  uint32_t pos0;          // list position of tile[0]
+  uint32_t cw = 0xFFFFFFFFu, bits = 0, fpos = 0, lpos = 0;
+  bool cf = false;        // the run's predecessor was seen here (in another word)
+  __device__ __forceinline__ void flush(bool cl) {
+    if (cw == 0xFFFFFFFFu) return;
+    if (cf && cl) {
+      bm[cw] = make_uint2(bits, ~fpos);
+    } else {
+      atomicOr(&bm[cw].x, bits);
+      atomicMax(&bm[cw].y, ~fpos);
+    }
+  }
+  __device__ __forceinline__ void add(uint32_t pos, uint32_t v) {
+    const uint32_t w = v >> 5;
+    const bool contig = cw != 0xFFFFFFFFu && pos == lpos + 1u;
+    if (w != cw || !contig) {
+      flush(contig);   // the successor (this element) is here, in another word
+      cf = contig;
+      cw = w;
+      bits = 0;
+      fpos = pos;
+    }
+    bits |= 1u << (v & 31u);
+    lpos = pos;
+  }
+  __device__ __forceinline__ void put4(uint32_t *p, uint4 v) {
+    const uint32_t pos = pos0 + (uint32_t)(p - tile);
+    add(pos, v.x);
+    add(pos + 1u, v.y);
+    add(pos + 2u, v.z);
+    add(pos + 3u, v.w);
+  }
+  __device__ __forceinline__ void put(uint32_t *p, uint32_t v) { add(pos0 + (uint32_t)(p - tile), v); }
+  // end of this lane's elements: its last run may share its word
+  __device__ __forceinline__ void finish() {
+    flush(false);
+    cw = 0xFFFFFFFFu;
+  }
+};
+// Bitvector lookup of docID x: its list position, or kNone if absent.
+__device__ __forceinline__ uint32_t bitvec_pos(uint2 w, uint32_t x) {
+  const uint32_t bit = x & 31u;
+  return ((w.x >> bit) & 1u) ? ~w.y + __popc(w.x & ((1u << bit) - 1u)) : 0xFFFFFFFFu;
+}
 
 // ---- eight consecutive elements of a staged block (one lane) ----------------------
 // Elements k .. k+ne-1 (ne <= 8) given p = the high-stream position of element

@@ -28,7 +28,11 @@ void set_error(const std::string &msg);
 enum : int { kStatusBadTerm = 1, kStatusOverflow = 2, kStatusTooManyTerms = 4 };
 
 // Query modes per (query, round).
-enum : uint32_t { kModeNone = 0, kModeMerge = 1, kModeGallop = 2, kModeAll = 3, kModeProbe = 4 };
+enum : uint32_t { kModeNone = 0, kModeMerge = 1, kModeGallop = 2, kModeAll = 3, kModeProbe = 4,
+                  kModeBitmap = 5 };
+// Per-term batch decode-once kind (Workspace::tdec): not decoded, decoded into
+// the docID arena, or decoded into a docID bitvector with rank (dense lists).
+enum : uint8_t { kDecNone = 0, kDecArena = 1, kDecBitmap = 2 };
 
 // Grow-only device buffer.
 struct DevBuf {
@@ -64,6 +68,7 @@ struct Workspace {
   DevBuf keys, counts, docids, scores, qoffs, qterms;  // host-API staging on device
   DevBuf demand, tdec, runs, run_base, vtmp, run_term; // per term / run (batch reuse)
   DevBuf arena;                                        // decoded lists, nblocks * B u32
+  DevBuf bmap;                                         // decoded dense lists: bitvector + rank
   DevBuf sbkt_cnt, sbkt_pos, sbkt_tmp;                 // S-locality unit order buckets
   size_t nq_cap = 0, unit_cap = 0, entry_cap = 0;
   // pinned host staging; a grown buffer's predecessors stay allocated until the
@@ -96,10 +101,12 @@ enum : int {
   kScalRoundTot = 18, // u64: survivors of the current round (compaction scan total)
   kScalDiag = 19,     // 4 x u64 (counting mode): merge units, merged elements, gallop units, galloped elements
   kScalUnitCtr2 = 23, // u64 ticket counter of the round-1 gallop/single-term kernel
-  kScalCount = 24
+  kScalDiag2 = 24,    // 2 x u64 (counting mode): bitvector units, their R elements
+  kScalCount = 26
 };
 
-constexpr uint32_t kBumpChunk = 256;   // bump-area entries grabbed per warp atomic
+constexpr uint32_t kBumpChunk = 256;
+constexpr uint32_t kBmBucketShift = 13;   // 8192 docs (2 KB of bitvector) per bucket   // bump-area entries grabbed per warp atomic
 
 struct RoundArgs {
   uint32_t nq, round, D, T, Tdec;
@@ -132,8 +139,16 @@ struct RoundArgs {
   uint32_t *sbkt_cnt;     // S-locality order: merge units per bucket of S blocks (or null)
   unsigned long long *sbkt_pos;   // bucket cursors (exclusive scan of sbkt_cnt)
   uint32_t sbkt_shift;    // bucket = global S block of the unit's start >> shift
+  // bitvector units follow the merge buckets: bucket = sbkt_nm + S slot * sbkt_nbb
+  // + (first R docID >> kBmBucketShift), so units probing the same bitvector
+  // region run together (L2 reuse across queries)
+  uint64_t sbkt_nm;
+  uint32_t sbkt_nbb;
   const uint32_t *dec;    // batch decoded arena (global block * B + i), or null
-  const uint8_t *tdec;    // per term: 1 = decoded in the arena this batch
+  const uint8_t *tdec;    // per term: kDecArena / kDecBitmap this batch (else kDecNone)
+  const uint2 *bm;        // bitvector area: slot s at bm + s * bm_words
+  const uint32_t *bm_slot;   // per term: its bitvector slot (kNone: not eligible)
+  uint32_t bm_words;      // words per bitvector = ceil(n_docs / 32)
 };
 
 }  // namespace griffin
@@ -186,6 +201,11 @@ struct griffin_index {
   int sorder = 1;   // merge units ordered by the S blocks they read (L2 reuse across queries)
   uint32_t sorder_shift = 6;
   uint32_t P = 0;   // probe chunk (0 = B)
+  // dense lists decoded once per batch into a bitvector + rank (kDecBitmap):
+  // eligible iff df_local * bm_inv >= n_docs (density >= 1 / bm_inv); 0 = off.
+  // Slots are per eligible term (host-assigned when the knob changes).
+  uint32_t bm_inv = 32, bm_slots_inv = 0, bm_nslots = 0;
+  uint32_t *d_bm_slot = nullptr, *d_bm_term = nullptr;
   uint64_t entry_budget = 0;   // griffin_set_entry_budget: intermediate entries per workspace (0 = exact bound)
   int profiling = 0;   // bit 0: per-stage CUDA events, bit 1: algorithmic-byte counters
   griffin_profile prof{};

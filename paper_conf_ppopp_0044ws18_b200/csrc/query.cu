@@ -50,7 +50,10 @@ constexpr uint32_t kTopkSmem = 4096;
 // spilled (C2 round-1+2 intersect, ms: emission depth 4 / 2 / 1 = 0.653 /
 // 0.626 / 0.607; arena probes 4 / 2 = 0.697 / 0.655; skip searches 4 / 2 =
 // 0.605 / 0.603 — profiles/r01_configs.jsonl, session 3).
-constexpr int kEmitDepth = GRIFFIN_EMIT_DEPTH;   // survivors per lane per emission pass (gathers in flight)
+constexpr int kEmitDepth = GRIFFIN_EMIT_DEPTH;
+#ifndef GRIFFIN_UNIT_EMIT_DEPTH
+#define GRIFFIN_UNIT_EMIT_DEPTH 1
+#endif   // survivors per lane per emission pass (gathers in flight)
 constexpr int kSkipDepth = GRIFFIN_SKIP_DEPTH;   // interleaved skip-pointer searches per lane
 #ifndef GRIFFIN_MERGE_UNROLL
 #define GRIFFIN_MERGE_UNROLL 4
@@ -195,11 +198,15 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
       const TermInfo tS = ix.terms[sid];
       // crossover: T for compressed S (gallop decodes one block per
       // touched block), Tdec when S sits decoded in the batch arena
-      const uint64_t T = (a.tdec && a.tdec[sid]) ? a.Tdec : a.T;
+      const uint8_t kd = a.tdec ? a.tdec[sid] : kDecNone;
+      const uint64_t T = kd == kDecArena ? a.Tdec : a.T;
       const bool gallop = a.forced_mode == 2 ||
                           (a.forced_mode == 0 && (uint64_t)tS.df_local > T * nR);
-      mode = gallop ? kModeGallop : kModeMerge;
-      units = gallop ? nbR : (nbR + tS.nblocks + a.D - 1) / a.D;
+      // S decoded into a bitvector this batch: every R element is looked up in
+      // O(1) (no merge or gallop through S), one unit per R chunk of B
+      const bool bitmap = a.forced_mode == 0 && kd == kDecBitmap;
+      mode = bitmap ? kModeBitmap : (gallop ? kModeGallop : kModeMerge);
+      units = (bitmap || gallop) ? nbR : (nbR + tS.nblocks + a.D - 1) / a.D;
     }
   }
   a.qmode[q] = mode;
@@ -435,14 +442,18 @@ __device__ __forceinline__ uint32_t load_r_chunk(const uint2 *Rq, uint32_t nR, u
   return n;
 }
 
-// Ordered emission of the matched R-tile elements [ia, ib) (two passes: count,
-// then write at a bump-allocated offset).  KIND 0: round 1 (s = w_R + w_S);
-// KIND 1: later round (s = s_prev + w_S); KIND 2: single-term (s = w_R).
+// Ordered emission of the matched R-tile elements [ia, ib).  KIND 0: round 1
+// (s = w_R + w_S); KIND 1: later round (s = s_prev + w_S); KIND 2: single-term
+// (s = w_R).  KIND 0/1 first compact the matches (R tile index -> idx[],
+// S position -> match[] in place, both in R order) so the scoring loop below
+// runs every lane on a survivor instead of one lane in ~three, with two
+// survivors' gathers (norm, tfs) in flight per lane.  idx: >= ib words of
+// scratch (unused for KIND 2).
 template <int KIND>
-__device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, const TermInfo &tR,
+__device__ __forceinline__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, const TermInfo &tR,
                           const TermInfo &tS, const uint2 *Rq, const uint32_t *tile,
-                          const uint32_t *match, uint32_t ia, uint32_t ib, uint32_t posR0,
-                          Acc &acc) {
+                          uint32_t *match, uint32_t *idx, uint32_t ia, uint32_t ib,
+                          uint32_t posR0, Acc &acc) {
   const uint32_t lane = lane_id(), lt = lanemask_lt();
   uint32_t cnt = 0;
   if (KIND == 2) {
@@ -450,8 +461,18 @@ __device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, co
   } else {
     for (uint32_t c0 = ia; c0 < ib; c0 += 32) {
       const uint32_t i = c0 + lane;
-      cnt += __popc(__ballot_sync(0xffffffffu, i < ib && match[i] != kNone));
+      const uint32_t mv = i < ib ? match[i] : kNone;
+      const bool p = mv != kNone;
+      const uint32_t bal = __ballot_sync(0xffffffffu, p);
+      __syncwarp();   // every lane has read its match[i] before any compacted write
+      if (p) {
+        const uint32_t o = cnt + __popc(bal & lt);   // o <= i: in place is safe
+        idx[o] = i;
+        match[o] = mv;
+      }
+      cnt += __popc(bal);
     }
+    __syncwarp();
   }
   unsigned long long off = 0;
   if (lane == 0 && cnt) off = bump_alloc(a, acc, cnt);
@@ -460,32 +481,46 @@ __device__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, co
     if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
     cnt = 0;
   }
-  if (cnt) {
-    uint32_t run = 0;
-    for (uint32_t c0 = ia; c0 < ib; c0 += 32) {
-      const uint32_t i = c0 + lane;
-      const bool p = i < ib && (KIND == 2 || match[i] != kNone);
-      const uint32_t bal = __ballot_sync(0xffffffffu, p);
-      if (p) {
-        const uint32_t doc = tile[i];
-        const float nrm = __ldg(ix.norm + doc);
+  constexpr int kDep = KIND == 2 ? 1 : GRIFFIN_UNIT_EMIT_DEPTH;
+  for (uint32_t j0 = 0; j0 < cnt; j0 += 32u * kDep) {
+    uint32_t doc[kDep], t1[kDep], t2[kDep];
+    float nrm[kDep];
+#pragma unroll
+    for (int t = 0; t < kDep; ++t) {
+      const uint32_t j = j0 + 32u * t + lane;
+      if (j < cnt) {
+        const uint32_t i = KIND == 2 ? ia + j : idx[j];
+        doc[t] = tile[i];
+        nrm[t] = __ldg(ix.norm + doc[t]);
+        if (KIND == 2) {
+          t1[t] = tf_lookup(ix, tR, posR0 + i);
+        } else {
+          t1[t] = tf_lookup(ix, tS, match[j]);
+          t2[t] = KIND == 0 ? tf_lookup(ix, tR, posR0 + i) : Rq[posR0 + i].y;
+        }
+      }
+    }
+#pragma unroll
+    for (int t = 0; t < kDep; ++t) {
+      const uint32_t j = j0 + 32u * t + lane;
+      if (j < cnt) {
         float s;
         if (KIND == 2) {
-          s = bm25_w(tR.idf, tf_lookup(ix, tR, posR0 + i), nrm, ix.k1p1);
+          s = bm25_w(tR.idf, t1[t], nrm[t], ix.k1p1);
         } else {
-          const float wS = bm25_w(tS.idf, tf_lookup(ix, tS, match[i]), nrm, ix.k1p1);
+          const float wS = bm25_w(tS.idf, t1[t], nrm[t], ix.k1p1);
           if (KIND == 0) {
-            s = bm25_w(tR.idf, tf_lookup(ix, tR, posR0 + i), nrm, ix.k1p1);  // first term: s = w
+            s = bm25_w(tR.idf, t2[t], nrm[t], ix.k1p1);  // first term: s = w
             s = __fadd_rn(s, wS);
           } else {
-            s = __fadd_rn(__uint_as_float(Rq[posR0 + i].y), wS);
+            s = __fadd_rn(__uint_as_float(t2[t]), wS);
           }
         }
-        a.bump[off + run + __popc(bal & lt)] = make_uint2(doc, __float_as_uint(s));
+        a.bump[off + j] = make_uint2(doc[t], __float_as_uint(s));
       }
-      run += __popc(bal);
     }
   }
+  __syncwarp();
   if (lane == 0) {
     a.unit_off[u] = off;
     a.unit_cnt[u] = cnt;
@@ -627,6 +662,19 @@ __device__ __forceinline__ uint32_t merge_unit_bucket(const DevIndex &ix, const 
   return (ix.terms[sid].block0 + rec.z) >> a.sbkt_shift;
 }
 
+// bucket of bitvector unit u (R chunk lu of query q): its S bitvector slot and
+// the chunk's first R docID
+template <bool RC>
+__device__ __forceinline__ uint64_t bitmap_unit_bucket(const DevIndex &ix, const RoundArgs &a,
+                                                       uint64_t u) {
+  const uint4 rec = a.urec[u];
+  const uint32_t q = rec.x, lu = rec.y;
+  const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
+  const uint32_t x0 = RC ? __ldg(ix.first + ix.terms[pt[0]].block0 + lu)
+                         : a.rprev[a.roff_prev[q] + (size_t)lu * ix.B].x;
+  return a.sbkt_nm + (uint64_t)a.bm_slot[pt[a.round]] * a.sbkt_nbb + (x0 >> kBmBucketShift);
+}
+
 template <bool RC>
 __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
   const uint64_t total = a.unit_base[a.nq];
@@ -648,7 +696,10 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
     uint32_t q = 0;
     if (valid) q = a.urec[u].x;
     const bool mg = valid && a.qmode[q] == kModeMerge;
-    const uint32_t bm = __ballot_sync(0xffffffffu, mg), bo = __ballot_sync(0xffffffffu, valid && !mg);
+    // bitvector units are bucketed too when the order is on (after the merge units)
+    const bool bu = valid && a.sbkt_cnt && a.sbkt_nbb && a.qmode[q] == kModeBitmap;
+    const uint32_t bm = __ballot_sync(0xffffffffu, mg),
+                   bo = __ballot_sync(0xffffffffu, valid && !mg && !bu);
     const uint32_t lane = threadIdx.x & 31u, lt = (1u << lane) - 1u;
     unsigned long long hm = 0, ho = 0;
     if (lane == 0) {
@@ -660,6 +711,8 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
     if (mg) {
       if (a.sbkt_cnt) atomicAdd(a.sbkt_cnt + merge_unit_bucket(ix, a, u), 1u);
       else a.uperm[hm + __popc(bm & lt)] = (uint32_t)u;
+    } else if (bu) {
+      atomicAdd(a.sbkt_cnt + bitmap_unit_bucket<RC>(ix, a, u), 1u);
     } else if (valid) {
       a.uperm[total - 1 - (ho + __popc(bo & lt))] = (uint32_t)u;
     }
@@ -676,13 +729,16 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
 // postings of 39M distinct ones, C5 2.66 B of 455M).  Order inside a bucket is
 // arbitrary; results do not depend on processing order.
 constexpr uint32_t kSorderMinQueries = 4096;
+template <bool RC>
 __global__ void sorder_scatter_kernel(DevIndex ix, RoundArgs a) {
   const uint64_t total = a.unit_base[a.nq];
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < total; u += stride) {
     const uint32_t q = a.urec[u].x;
-    if (a.qmode[q] != kModeMerge) continue;
-    const unsigned long long slot = atomicAdd(a.sbkt_pos + merge_unit_bucket(ix, a, u), 1ull);
+    const uint32_t md = a.qmode[q];
+    if (md != kModeMerge && !(md == kModeBitmap && a.sbkt_nbb)) continue;
+    const uint64_t bk = md == kModeMerge ? merge_unit_bucket(ix, a, u) : bitmap_unit_bucket<RC>(ix, a, u);
+    const unsigned long long slot = atomicAdd(a.sbkt_pos + bk, 1ull);
     a.uperm[slot] = (uint32_t)u;
   }
 }
@@ -942,6 +998,40 @@ __device__ __forceinline__ uint32_t arena_probe_slice(const uint32_t *__restrict
   return chunks;
 }
 
+// Bitvector lookups of the elements x = tileR[0..n): match[e] = x's position
+// in S, or kNone (4 independent 8-B loads in flight per lane).  Counting pass:
+// one 32-B sector per distinct sector the warp reads in list order (SURVEY
+// §8(d) charges gathers by sector).
+__device__ __forceinline__ void bitvec_probe(const uint2 *__restrict__ bm,
+                                             const uint32_t *tileR, uint32_t *match, uint32_t n,
+                                             int count, Acc &acc) {
+  const uint32_t lane = lane_id();
+  uint32_t sectors = 0;
+  for (uint32_t base = 0; base < n; base += 128u) {
+    uint32_t x[4];
+    uint2 wv[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t e = base + lane + 32u * j;
+      x[j] = e < n ? tileR[e] : 0u;
+      wv[j] = e < n ? __ldg(bm + (x[j] >> 5)) : make_uint2(0, 0);
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t e = base + lane + 32u * j;
+      if (e < n) {
+        match[e] = bitvec_pos(wv[j], x[j]);
+        if (count) sectors += (e == 0 || (tileR[e - 1] >> 7) != (x[j] >> 7)) ? 1u : 0u;
+      }
+    }
+  }
+  if (count) {
+    const uint32_t sp = __reduce_add_sync(0xffffffffu, sectors);
+    if (lane == 0) acc.ctr[kCAlg] += sp * 32ull;
+  }
+  __syncwarp();
+}
+
 // Multi-list probe (SvS rounds 2..m-1 in one pass): every round-1 survivor is
 // looked up in each remaining list in canonical order — skip-pointer search,
 // then an in-place binary search of the decoded-arena block or a staged EF
@@ -974,8 +1064,13 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
     const uint32_t sid = pt[r];
     const TermInfo tS = ix.terms[sid];
     const uint32_t *fS = ix.first + tS.block0;
-    const bool sdec = a.tdec && a.tdec[sid];
+    const uint8_t kd = a.tdec ? a.tdec[sid] : kDecNone;
+    const bool sdec = kd == kDecArena;
     const uint32_t *decS = sdec ? a.dec + (size_t)tS.block0 * B : nullptr;
+    if (kd == kDecBitmap) {
+      // ---- S decoded into a bitvector: O(1) lookups, then the shared drop/score step ----
+      bitvec_probe(a.bm + (size_t)a.bm_slot[sid] * a.bm_words, tileR, match, n, a.count, acc);
+    } else {
     // skip pointers this chunk can touch: [ub(first survivor) - 1, ub(last)),
     // found by a warp-cooperative 16-ary search; a chunk usually spans few
     // enough of them to be searched from one coalesced smem window
@@ -1075,6 +1170,7 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
         g0 += ng;
       }
     }
+    }   // compressed / arena S
     __syncwarp();
     // ---- add w_t to the members, drop the rest (stable in-place compaction) ----
     uint32_t nn2 = 0;
@@ -1198,7 +1294,7 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
     const uint32_t nR = RC ? tR.df_local : a.rcount[q];
     const uint32_t nbR = RC ? tR.nblocks : (nR + B - 1) / B;
     // R source: compressed EF, the batch's decoded arena, or the intermediate
-    const bool rdec = RC && a.tdec && a.tdec[t0];
+    const bool rdec = RC && a.tdec && a.tdec[t0] == kDecArena;
     const uint32_t *decR = rdec ? a.dec + (size_t)tR.block0 * B : nullptr;
 
     if (ROLE != 1 && RC && mode == kModeAll) {  // single-term query: the whole list is the result
@@ -1229,7 +1325,7 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
           acc.ctr[kCAlg] += sz * 16u + 8u;
         }
       }
-      emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, 0, n, lu * B, acc);
+      emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, nullptr, 0, n, lu * B, acc);
       continue;
     }
     if (ROLE == 0 && !RC && mode == kModeProbe) {
@@ -1240,7 +1336,7 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
     const TermInfo tS = ix.terms[tSid];
     const uint32_t *fS = ix.first + tS.block0;
     const uint32_t nbS = tS.nblocks;
-    const bool sdec = a.tdec && a.tdec[tSid];
+    const bool sdec = a.tdec && a.tdec[tSid] == kDecArena;
     const uint32_t *decS = sdec ? a.dec + (size_t)tS.block0 * B : nullptr;
 
     if (ROLE != 2 && (ROLE == 1 || mode == kModeMerge)) {
@@ -1488,6 +1584,20 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
         if (lane == 0) acc.ctr[kCAlg] += n * 8u;
       }
       __syncwarp();
+      if (mode == kModeBitmap) {
+        // S decoded into a bitvector this batch: O(1) lookups of the R chunk
+        if (a.count && lane == 0) {
+          atomicAdd(a.scal + kScalDiag2, 1ull);
+          atomicAdd(a.scal + kScalDiag2 + 1, (unsigned long long)n);
+        }
+        bitvec_probe(a.bm + (size_t)a.bm_slot[tSid] * a.bm_words, tileR, match, n, a.count, acc);
+        if (RC)
+          emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
+        else
+          emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
+        __syncwarp();
+        continue;
+      }
       const uint32_t k_lo = rec.z, k_hi = rec.w;   // from the partition stage
       if (a.count && lane == 0) {
         atomicAdd(a.scal + kScalDiag + 2, 1ull);
@@ -1528,9 +1638,9 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
         if (lane == 0) acc.ctr[kCAlg] += sp * 32ull;
         __syncwarp();
         if (RC)
-          emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
+          emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
         else
-          emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
+          emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
         __syncwarp();
         continue;
       }
@@ -1649,9 +1759,9 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
         g0 += ng;
       }
       if (RC)
-        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
+        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
       else
-        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, 0, n, lu * B, acc);
+        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
       __syncwarp();
     }
   }
@@ -2263,7 +2373,7 @@ __device__ __forceinline__ uint32_t decode_run(const DevIndex &ix, WarpSmem &w, 
     f = ix.first[k0 + lane];
     sz = block_size16(m.y);
   }
-  if (sink) stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, w.tile, *sink);
+  if (sink) stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, dst ? dst : w.tile, *sink);
   else stage_decode_lanes(ix, w, stage_words(ix.B, D) / 4u, 0, nb, m, f, sz, dst ? dst : w.tile);
   const uint32_t tot = __reduce_add_sync(0xffffffffu, lane < nb ? meta_n(m.y) : 0u);
   *pay_bytes = __reduce_add_sync(0xffffffffu, sz) * 16u;
@@ -2347,15 +2457,29 @@ __global__ void demand_kernel(DevIndex ix, RoundArgs a, uint32_t *demand) {
   }
 }
 
-__global__ void select_kernel(DevIndex ix, const uint32_t *demand, uint8_t *tdec, uint32_t *runs,
-                              uint32_t run_len) {
+// bm_slot (or null: bitvectors off): a selected term with a bitvector slot is
+// decoded into it (kDecBitmap), any other selected term into the arena.
+__global__ void select_kernel(DevIndex ix, const uint32_t *demand, const uint32_t *bm_slot,
+                              uint8_t *tdec, uint32_t *runs, uint32_t run_len) {
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
   if (t >= ix.num_terms) return;
   const uint32_t nb = ix.terms[t].nblocks;
   // decode once if the batch would otherwise decode >= 1.5x the list's blocks
   const bool sel = nb > 0 && 2ull * demand[t] >= 3ull * nb;
-  tdec[t] = sel ? 1 : 0;
+  tdec[t] = sel ? ((bm_slot && bm_slot[t] != kNone) ? kDecBitmap : kDecArena) : kDecNone;
   runs[t] = sel ? (nb + run_len - 1) / run_len : 0u;
+}
+
+// Zero the bitvector slots of this batch's kDecBitmap terms (slot-major grid).
+__global__ void bm_zero_kernel(const uint8_t *tdec, const uint32_t *bm_term, uint32_t nslots,
+                               uint32_t words, uint4 *bm) {
+  const uint32_t per = (words + 1u) / 2u;   // uint4 = two words
+  for (uint32_t s = blockIdx.y; s < nslots; s += gridDim.y) {
+    if (tdec[bm_term[s]] != kDecBitmap) continue;
+    uint4 *p = bm + (size_t)s * per;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < per; i += gridDim.x * blockDim.x)
+      p[i] = make_uint4(0, 0, 0, 0);
+  }
 }
 
 // Para-EF decode of every block of the selected terms into the arena
@@ -2371,9 +2495,11 @@ __global__ void run_map_kernel(uint32_t V, const uint32_t *runs, const uint64_t 
   for (uint32_t i = lane_id(); i < nr; i += 32) run_term[b + i] = t;
 }
 
-__global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t D,
+__global__ void __launch_bounds__(256, 3) decode_once_kernel(DevIndex ix, uint32_t D,
                                                           const uint64_t *run_base,
                                                           const uint32_t *run_term, uint32_t *arena,
+                                                          const uint8_t *tdec, uint2 *bm,
+                                                          const uint32_t *bm_slot, uint32_t bm_words,
                                                           unsigned long long *scal) {
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
@@ -2390,13 +2516,24 @@ __global__ void __launch_bounds__(256) decode_once_kernel(DevIndex ix, uint32_t 
     const uint32_t ri = (uint32_t)(r - run_base[lo]);
     const uint32_t k0 = ri * run, nb = min(run, t.nblocks - k0);
     const uint64_t gb = (uint64_t)t.block0 + k0;
-    uint32_t p;
-    // decoded straight into the arena (128-bit stores, coalesced per half-warp)
-    const uint32_t n = decode_run(ix, w, D, gb, nb, &p, nullptr, arena + gb * B);
+    uint32_t p, n;
+    if (tdec[lo] == kDecBitmap) {
+      // dense list: into its bitvector + rank (arena + gb * B only names positions)
+      BitSink bs;
+      bs.bm = bm + (size_t)bm_slot[lo] * bm_words;
+      bs.tile = arena + gb * B;
+      bs.pos0 = k0 * B;
+      n = decode_run(ix, w, D, gb, nb, &p, nullptr, arena + gb * B, &bs);
+      bs.finish();
+      if (lane == 0) alg += p + 8ull * nb + (uint64_t)bm_words * 8ull * nb / t.nblocks;
+    } else {
+      // decoded straight into the arena (128-bit stores, coalesced per half-warp)
+      n = decode_run(ix, w, D, gb, nb, &p, nullptr, arena + gb * B);
+      if (lane == 0) alg += p + 8ull * nb + 4ull * n;
+    }
     if (lane == 0) {
       pay += p;
       post += n;
-      alg += p + 8ull * nb + 4ull * n;
       c8d += p + 8ull * nb;
     }
   }
@@ -2425,6 +2562,18 @@ int num_sms(int dev) {
   return v;
 }
 
+static griffin_status ensure_bm_slots(griffin_index *ix);
+// S-locality buckets: merge units by S block, then bitvector units by (S slot, R docID)
+static uint64_t sorder_merge_buckets(const griffin_index *ix) {
+  return (ix->nblocks >> ix->sorder_shift) + 1;
+}
+static uint32_t sorder_bm_per_slot(const griffin_index *ix) {
+  return ((ix->doc_end - ix->doc_base) >> kBmBucketShift) + 1;
+}
+static uint64_t sorder_buckets(const griffin_index *ix) {
+  return sorder_merge_buckets(ix) + (uint64_t)ix->bm_nslots * sorder_bm_per_slot(ix);
+}
+
 griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t units,
                           uint64_t entries) {
   // `entries` is the exact per-batch bound (sum over queries of min(df0, df1));
@@ -2446,7 +2595,9 @@ griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t
   GRIFFIN_CUDA_TRY(w.uperm.reserve((units + 2) * 4));
   GRIFFIN_CUDA_TRY(w.unit_dst.reserve((units + 2) * 8 + (units / kScanTile + 2) * 8));
   if (ix->sorder && nq >= kSorderMinQueries) {   // S-locality buckets (no allocation in run_batch)
-    const size_t nbkt = (ix->nblocks >> ix->sorder_shift) + 1;
+    griffin_status bs = ensure_bm_slots(ix);
+    if (bs) return bs;
+    const size_t nbkt = sorder_buckets(ix);
     GRIFFIN_CUDA_TRY(w.sbkt_cnt.reserve(nbkt * 4));
     GRIFFIN_CUDA_TRY(w.sbkt_pos.reserve((nbkt + 1) * 8));
     GRIFFIN_CUDA_TRY(w.sbkt_tmp.reserve((nbkt / kScanTile + 4) * 8));
@@ -2577,6 +2728,34 @@ griffin_status reserve_topk(griffin_index *ix, Workspace &w, uint32_t nq, uint32
   return GRIFFIN_OK;
 }
 
+// Bitvector slots of the terms eligible for kDecBitmap (griffin_set_bitmap):
+// df_local * bm_inv >= shard docs; recomputed when the knob changes.
+static griffin_status ensure_bm_slots(griffin_index *ix) {
+  if (ix->bm_slots_inv == ix->bm_inv && (ix->d_bm_slot || !ix->bm_inv)) return GRIFFIN_OK;
+  cudaFree(ix->d_bm_slot);
+  cudaFree(ix->d_bm_term);
+  ix->d_bm_slot = ix->d_bm_term = nullptr;
+  ix->bm_nslots = 0;
+  ix->bm_slots_inv = ix->bm_inv;
+  if (!ix->bm_inv) return GRIFFIN_OK;
+  const uint64_t nd = ix->doc_end - ix->doc_base;
+  std::vector<uint32_t> slot(ix->V, kNone), term;
+  for (uint32_t t = 0; t < ix->V; ++t) {
+    const uint64_t df = ix->h_terms[t].df_local;
+    if (df > 0 && df * ix->bm_inv >= nd) {
+      slot[t] = (uint32_t)term.size();
+      term.push_back(t);
+    }
+  }
+  ix->bm_nslots = (uint32_t)term.size();
+  GRIFFIN_CUDA_TRY(cudaMalloc(&ix->d_bm_slot, (size_t)ix->V * 4 + 4));
+  GRIFFIN_CUDA_TRY(cudaMalloc(&ix->d_bm_term, term.size() * 4 + 4));
+  GRIFFIN_CUDA_TRY(cudaMemcpy(ix->d_bm_slot, slot.data(), (size_t)ix->V * 4, cudaMemcpyHostToDevice));
+  if (!term.empty())
+    GRIFFIN_CUDA_TRY(cudaMemcpy(ix->d_bm_term, term.data(), term.size() * 4, cudaMemcpyHostToDevice));
+  return GRIFFIN_OK;
+}
+
 griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uint32_t *d_qoffs,
                          const uint32_t *d_terms, uint32_t max_terms, uint32_t k, uint64_t *d_keys,
                          uint32_t *d_counts, cudaStream_t st, bool final_topk, int forced_mode) {
@@ -2640,12 +2819,33 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     const uint32_t Dsw = sweep_D(ix->B);
     GRIFFIN_CUDA_TRY(w.run_term.reserve((ix->nblocks / (Dsw + 2) + (size_t)V + 2) * 4));
     GRIFFIN_CUDA_TRY(w.arena.reserve((ix->nblocks * ix->B + 64) * 4));
+    // dense lists: bitvector slots (forced modes never read them)
+    const bool bitmaps = ix->bm_inv && forced_mode == 0 && ix->h_terms.size() == V;
+    const uint32_t bm_words = (ix->doc_end - ix->doc_base + 31u) / 32u;
+    if (bitmaps) {
+      griffin_status bs = ensure_bm_slots(ix);
+      if (bs) return bs;
+      GRIFFIN_CUDA_TRY(w.bmap.reserve((size_t)ix->bm_nslots * ((bm_words + 1u) & ~1u) * 8 + 16));
+    }
+    const bool use_bm = bitmaps && ix->bm_nslots > 0;
     GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.demand.p, 0, (size_t)V * 4, st));
     ra.T = ix->T;
     demand_kernel<<<qblocks, 256, 0, st>>>(di, ra, w.demand.as<uint32_t>());
     select_kernel<<<(V + 255) / 256, 256, 0, st>>>(di, w.demand.as<uint32_t>(),
+                                                   use_bm ? ix->d_bm_slot : nullptr,
                                                    w.tdec.as<uint8_t>(), w.runs.as<uint32_t>(),
                                                    Dsw + 2);
+    if (use_bm) {
+      // slots are padded to an even word count (uint4 zeroing)
+      const uint32_t words = (bm_words + 1u) & ~1u;
+      dim3 zg(std::max(1u, std::min(64u, (words / 2 + 255) / 256)), std::min(ix->bm_nslots, 1024u));
+      bm_zero_kernel<<<zg, 256, 0, st>>>(w.tdec.as<uint8_t>(), ix->d_bm_term, ix->bm_nslots, words,
+                                         w.bmap.as<uint4>());
+      ix->launch_count += 1;
+    }
+    ra.bm = use_bm ? w.bmap.as<uint2>() : nullptr;
+    ra.bm_slot = use_bm ? ix->d_bm_slot : nullptr;
+    ra.bm_words = (bm_words + 1u) & ~1u;
     GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(w.runs.as<uint32_t>(), w.run_base.as<uint64_t>(), V,
                                               w.vtmp.as<uint64_t>(), st, &ix->launch_count));
     run_map_kernel<<<(uint32_t)(((uint64_t)V * 32 + 255) / 256), 256, 0, st>>>(V, w.runs.as<uint32_t>(),
@@ -2656,7 +2856,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
     GRIFFIN_CUDA_TRY(launch_config((const void *)decode_once_kernel, ix->device, smem, 256, &per_sm));
     decode_once_kernel<<<num_sms(ix->device) * std::max(1, per_sm), 256, smem, st>>>(
         di, Dsw, w.run_base.as<uint64_t>(), w.run_term.as<uint32_t>(), w.arena.as<uint32_t>(),
-        scal);
+        w.tdec.as<uint8_t>(), const_cast<uint2 *>(ra.bm), ra.bm_slot, ra.bm_words, scal);
     GRIFFIN_CUDA_TRY(cudaGetLastError());
     ix->launch_count += 4;
     ra.dec = w.arena.as<uint32_t>();
@@ -2691,7 +2891,14 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
       uint64_t nbkt = 0;
       if (ix->sorder && nq >= kSorderMinQueries && (r == 1 || !ra.probe) && w.sbkt_cnt.p) {
         ra.sbkt_shift = ix->sorder_shift;
-        nbkt = (ix->nblocks >> ra.sbkt_shift) + 1;   // buffers sized in reserve_ws
+        ra.sbkt_nm = sorder_merge_buckets(ix);
+        ra.sbkt_nbb = sorder_bm_per_slot(ix);
+        // bitvector buckets only when this batch uses bitvectors and the buffers
+        // (sized in reserve_ws) hold them; else those units join the tail
+        const bool bmb = ra.bm && sorder_buckets(ix) * 4 <= w.sbkt_cnt.bytes &&
+                         (sorder_buckets(ix) + 1) * 8 <= w.sbkt_pos.bytes;
+        if (!bmb) ra.sbkt_nbb = 0;
+        nbkt = bmb ? sorder_buckets(ix) : ra.sbkt_nm;
         GRIFFIN_CUDA_TRY(cudaMemsetAsync(w.sbkt_cnt.p, 0, nbkt * 4, st));
         ra.sbkt_cnt = w.sbkt_cnt.as<uint32_t>();
         ra.sbkt_pos = w.sbkt_pos.as<unsigned long long>();
@@ -2702,7 +2909,8 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
         GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(ra.sbkt_cnt, w.sbkt_pos.as<uint64_t>(), nbkt,
                                                   w.sbkt_tmp.as<uint64_t>(), st,
                                                   &ix->launch_count));
-        sorder_scatter_kernel<<<pgrid, 256, 0, st>>>(di, ra);
+        if (r == 1) sorder_scatter_kernel<true><<<pgrid, 256, 0, st>>>(di, ra);
+        else sorder_scatter_kernel<false><<<pgrid, 256, 0, st>>>(di, ra);
         ix->launch_count += 1;
       }
       if (r == 1) {   // merge units, then gallop / single-term units

@@ -343,12 +343,16 @@ def test_c2_full_size_all_queries_timed_config():
             assert_topk_equal(gd, gs, gc, od, os_, oc)
 
 
-def test_large_batch_s_locality_order():
-    """Batches of >= 4096 queries hand out merge units in S-locality order
-    (sorder_scatter_kernel); the results must not depend on it."""
+@pytest.mark.parametrize("inv", [0, 32, 1 << 24])
+def test_large_batch_s_locality_order(inv):
+    """Batches of >= 4096 queries hand out merge units (and bitvector units, by
+    S slot and R docID) in S-locality order (sorder_scatter_kernel); the results
+    must not depend on it."""
     import torch
     c, ql, cfg = make_workload("small", num_queries=5000)
     gx = g.GriffinIndex(c, block_size=128)
+    gx.griffin_set_bitmap(inv)
+    gx.griffin_set_profiling(3)
     ox = oracle.OracleIndex(c, block_size=128)
     k, nq = 10, ql.num_queries
     # device API: one batch of all 5000 queries (the host API would slice it)
@@ -367,6 +371,11 @@ def test_large_batch_s_locality_order():
     od, os_, oc = ox.query_batch(ql, k, nthreads=4)
     assert_topk_equal(dd.cpu().numpy().view(np.uint32).reshape(nq, k), ds.cpu().numpy().reshape(nq, k),
                       cnt.cpu().numpy().view(np.uint32), od, os_, oc)
+    prof = gx.griffin_get_profile()
+    if inv == 0:
+        assert prof["bitmap_units"] == 0
+    if inv == 1 << 24:
+        assert prof["bitmap_units"] > 0
 
 
 @pytest.mark.slow
@@ -479,6 +488,72 @@ def test_reuse_random_batches_and_single_terms():
         od, os_, oc = ox.query_batch(ql, 50)
         gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 50)
         assert_topk_equal(gd, gs, gc, od, os_, oc)
+
+
+@pytest.mark.parametrize("inv", [0, 32, 1 << 24])
+def test_bitmap_decode_once_bit_exact(tiny, inv):
+    """Dense lists decoded once into a bitvector + rank (griffin_set_bitmap):
+    off, the default density threshold, and every decoded list — identical to
+    the oracle, and the bitvector units really ran when enabled."""
+    c, ql, ox = tiny
+    gx = g.GriffinIndex(c, block_size=128)
+    gx.griffin_set_reuse(1)
+    gx.griffin_set_bitmap(inv)
+    gx.griffin_set_profiling(3)
+    for k in (10, 300):
+        od, os_, oc = ox.query_batch(ql, k)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+    prof = gx.griffin_get_profile()
+    if inv == 1 << 24:
+        assert prof["bitmap_units"] > 0 and prof["bitmap_elems"] > 0
+    if inv == 0:
+        assert prof["bitmap_units"] == 0
+    gx.close()
+
+
+@pytest.mark.parametrize("B", [64, 96, 128, 256, 512])
+def test_bitmap_dense_runs_and_edges(B):
+    """Bitvector construction edge cases: lists of consecutive docIDs (whole
+    words owned by one lane: plain stores), near-complete lists, docID 0 and
+    N-1, word boundaries shared by lanes and blocks, multi-term queries (probe
+    pass / later SvS rounds against bitvectors), every block size."""
+    rng = np.random.default_rng(B)
+    N = 70_003
+    lists = [
+        np.arange(0, N, dtype=np.uint32),                                   # every doc
+        np.arange(5, N - 3, dtype=np.uint32)[rng.random(N - 8) < 0.97],     # near complete
+        np.nonzero(rng.random(N) < 0.5)[0].astype(np.uint32),
+        np.nonzero(rng.random(N) < 0.06)[0].astype(np.uint32),
+        np.unique(np.concatenate([[0, 31, 32, 63, 64, N - 33, N - 32, N - 1],
+                                  rng.integers(0, N, 3000)])).astype(np.uint32),
+        np.arange(1000, 9000, dtype=np.uint32),                             # one run
+        np.nonzero(rng.random(N) < 0.002)[0].astype(np.uint32),
+    ]
+    tfs = [rng.integers(1, 9, size=len(l)).astype(np.uint32) for l in lists]
+    dl = rng.integers(1, 3000, size=N).astype(np.uint32)
+    c = corpus_from_lists(N, lists, tfs, dl)
+    ox = oracle.OracleIndex(c, block_size=B)
+    gx = g.GriffinIndex(c, block_size=B)
+    gx.griffin_set_reuse(1)
+    gx.griffin_set_bitmap(1 << 24)
+    V = len(lists)
+    offs, terms = [0], []
+    for _ in range(3):
+        for a in range(V):
+            for b in range(V):
+                terms.extend([a, b])
+                offs.append(len(terms))
+    for _ in range(40):
+        m = int(rng.integers(3, 7))
+        terms.extend(int(t) for t in rng.choice(V, size=m, replace=False))
+        offs.append(len(terms))
+    ql = QueryLog(offsets=np.array(offs, np.uint32), terms=np.array(terms, np.uint32))
+    for k in (7, 1000):
+        od, os_, oc = ox.query_batch(ql, k)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+    gx.close()
 
 
 @pytest.mark.parametrize("k", [64, 65, 1000, 2048])

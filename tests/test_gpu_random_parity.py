@@ -1,7 +1,8 @@
 """Randomised parity (hypothesis): random small corpora (list lengths from empty
 to dense, docIDs near 0 and N-1, tf up to 2^32-1), random block sizes and
 batches of 1-8 term queries with repeats and empty-list terms, k from 1 to 600,
-each index mode — the GPU top-k (docIDs, order, score bits, counts) must equal
+each index mode and decode-once representation (docID arena or dense-list
+bitvector) — the GPU top-k (docIDs, order, score bits, counts) must equal
 the oracle's.  Shapes are kept small so every example runs in well under a
 second; the examples together exercise partial blocks, b = 0 runs, single-block
 lists, merge and gallop rounds, the probe pass and the top-k levels."""
@@ -57,17 +58,19 @@ def workloads(draw):
     k = draw(st.sampled_from([1, 3, 10, 100, 600]))
     mode = draw(st.sampled_from([g.MODE_AUTO, g.MODE_MERGE, g.MODE_GALLOP]))
     reuse = draw(st.sampled_from([0, 1, 2]))
-    return corpus_from_lists(N, lists, tfs, dl), ql, B, k, mode, reuse
+    bitmap = draw(st.sampled_from([0, 32, 1 << 24]))   # dense-list bitvectors: off / default / every decoded list
+    return corpus_from_lists(N, lists, tfs, dl), ql, B, k, mode, reuse, bitmap
 
 
 @settings(max_examples=150, deadline=None, derandomize=True,
           suppress_health_check=list(HealthCheck))
 @given(workloads())
 def test_random_workloads_bit_exact(w):
-    c, ql, B, k, mode, reuse = w
+    c, ql, B, k, mode, reuse, bitmap = w
     gx = g.GriffinIndex(c, block_size=B)
     gx.griffin_set_mode(mode)
     gx.griffin_set_reuse(reuse)
+    gx.griffin_set_bitmap(bitmap)
     ox = oracle.OracleIndex(c, block_size=B)
     gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
     od, os_, oc = ox.query_batch(ql, k)
