@@ -105,8 +105,11 @@ enum : int {
   kScalCount = 26
 };
 
-constexpr uint32_t kBumpChunk = 256;
-constexpr uint32_t kBmBucketShift = 13;   // 8192 docs (2 KB of bitvector) per bucket   // bump-area entries grabbed per warp atomic
+#ifndef GRIFFIN_BUMP_CHUNK
+#define GRIFFIN_BUMP_CHUNK 1024
+#endif
+constexpr uint32_t kBumpChunk = GRIFFIN_BUMP_CHUNK;   // bump-area entries grabbed per warp atomic
+constexpr uint32_t kBmBucketShift = 13;   // 8192 docs (2 KB of bitvector) per bucket
 
 struct RoundArgs {
   uint32_t nq, round, D, T, Tdec;

@@ -64,6 +64,7 @@ constexpr int kMergeUnroll = GRIFFIN_MERGE_UNROLL;
 #endif
 constexpr bool kIkPair = GRIFFIN_IK_PAIR;   // intersect kernel: two-blocks-per-warp decoder at B = 128
 constexpr int kTopkThreads = 512;
+constexpr uint32_t kTileSlackC = 64;   // = kTileSlack (read slack after a tile), needed early
 
 // ------------------------------------------------------------------- planning
 
@@ -152,6 +153,55 @@ __global__ void plan_totals_kernel(DevIndex ix, uint32_t nq, const uint32_t *pla
   }
 }
 
+// R blocks (or B-entry intermediate chunks) per bitvector unit, U, and where
+// its three U*B-word arrays live: the R tile at the start of the tile region,
+// the compacted R indices at the start of the staging area (free after
+// decoding), the compacted S positions after the R tile when the tile holds
+// both, else after the indices in the staging area.  Bitvector units run in
+// the round-1 gallop kernel (ROLE 2 layout, whose staging area is sized for
+// 2*Umax*B words) and, for later SvS rounds without the probe pass, in the
+// all-kinds kernel (ROLE 0 layout); U must fit both.  Fewer, larger units
+// amortise the per-unit work (ticket, records, a TMA round trip, the output
+// allocation) over up to U*B lookups.
+#ifndef GRIFFIN_BM_UNIT_ELEMS
+#define GRIFFIN_BM_UNIT_ELEMS 384
+#endif
+// most R elements per unit: Umax(B) = clamp(GRIFFIN_BM_UNIT_ELEMS / B, 1, 4)
+__host__ __device__ inline uint32_t bm_unit_max(uint32_t B) {
+  const uint32_t u = GRIFFIN_BM_UNIT_ELEMS / B;
+  return u < 1u ? 1u : (u > 4u ? 4u : u);
+}
+__host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D);
+__host__ __device__ inline uint32_t other_tile_words(uint32_t B, uint32_t D, bool nextgeq);
+__host__ __device__ inline uint32_t other_stage_words(uint32_t B, uint32_t D) {
+  const uint32_t s = stage_words(B, D), w = 2u * bm_unit_max(B) * B;
+  return s > w ? s : w;
+}
+// tile / staging words of the layout bitvector units run in (role2: ROLE 2)
+__host__ __device__ inline void bm_layout(uint32_t B, uint32_t D, bool nextgeq, bool role2,
+                                          uint32_t *tile, uint32_t *stg) {
+  *tile = (role2 ? other_tile_words(B, D, nextgeq) : (D + 2u) * B + kTileSlackC) - kTileSlackC;
+  *stg = role2 ? other_stage_words(B, D) : stage_words(B, D);
+}
+__host__ __device__ inline bool bm_spos_in_tile(uint32_t B, uint32_t D, bool nextgeq, bool role2,
+                                                uint32_t U) {
+  uint32_t tile, stg;
+  bm_layout(B, D, nextgeq, role2, &tile, &stg);
+  return 2u * U * B <= tile;
+}
+__host__ __device__ inline uint32_t bm_unit_blocks(uint32_t B, uint32_t D, bool nextgeq) {
+  for (uint32_t U = bm_unit_max(B); U > 1u; --U) {
+    bool ok = true;
+    for (int r = 0; r < 2; ++r) {
+      uint32_t tile, stg;
+      bm_layout(B, D, nextgeq, r == 1, &tile, &stg);
+      ok = ok && U * B <= tile && (2u * U * B <= tile || 2u * U * B <= stg);
+    }
+    if (ok) return U;
+  }
+  return 1u;
+}
+
 __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
   const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
   // units must fit their arrays; intermediates are checked at compaction time
@@ -206,7 +256,8 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
       // O(1) (no merge or gallop through S), one unit per R chunk of B
       const bool bitmap = a.forced_mode == 0 && kd == kDecBitmap;
       mode = bitmap ? kModeBitmap : (gallop ? kModeGallop : kModeMerge);
-      units = (bitmap || gallop) ? nbR : (nbR + tS.nblocks + a.D - 1) / a.D;
+      const uint32_t U = bm_unit_blocks(ix.B, a.D, a.nextgeq != 0);
+      units = bitmap ? (nbR + U - 1) / U : (gallop ? nbR : (nbR + tS.nblocks + a.D - 1) / a.D);
     }
   }
   a.qmode[q] = mode;
@@ -239,10 +290,13 @@ struct Acc {
 // are located by unit_off/unit_cnt, so chunk order and gaps do not matter.
 __device__ __forceinline__ unsigned long long bump_alloc(const RoundArgs &a, Acc &acc,
                                                          uint32_t cnt) {
+  // a unit bigger than a quarter chunk gets its own exact allocation (so a
+  // refill never throws away more than a quarter chunk of the previous one)
+  if (cnt > kBumpChunk / 4u) return atomicAdd(a.scal + kScalBump, (unsigned long long)cnt);
   unsigned long long off = *acc.boff;
   uint32_t left = *acc.bleft;
   if (cnt > left) {
-    left = cnt > kBumpChunk ? cnt : kBumpChunk;
+    left = kBumpChunk;
     off = atomicAdd(a.scal + kScalBump, (unsigned long long)left);
   }
   *acc.boff = off + cnt;
@@ -263,7 +317,7 @@ __host__ __device__ inline uint32_t stage_words(uint32_t B, uint32_t D) {
 }
 // read slack after the tile: the uniform-trip merge loop may read up to L =
 // ceil((D+2)*B/32) words past a lane's segment (D <= 8 at B = 128 -> 40)
-constexpr uint32_t kTileSlack = 64;
+constexpr uint32_t kTileSlack = kTileSlackC;
 // read slack after the staging area: decoders read a word or two past a block's
 // high stream (look-ahead windows), also when it ends the staging area
 constexpr uint32_t kStgSlack = kRunSlack;   // >= the run decoder's over-read
@@ -442,26 +496,72 @@ __device__ __forceinline__ uint32_t load_r_chunk(const uint2 *Rq, uint32_t nR, u
   return n;
 }
 
-// Ordered emission of the matched R-tile elements [ia, ib).  KIND 0: round 1
-// (s = w_R + w_S); KIND 1: later round (s = s_prev + w_S); KIND 2: single-term
-// (s = w_R).  KIND 0/1 first compact the matches (R tile index -> idx[],
-// S position -> match[] in place, both in R order) so the scoring loop below
-// runs every lane on a survivor instead of one lane in ~three, with two
-// survivors' gathers (norm, tfs) in flight per lane.  idx: >= ib words of
-// scratch (unused for KIND 2).
+// Emission of a unit's survivors, already compacted in R order: survivor j is
+// R tile element idx[j] (list position posR0 + idx[j]), found at S position
+// spos[j].  KIND 0: round 1 (s = w_R + w_S); KIND 1: later round (s = s_prev +
+// w_S); KIND 2: single-term (s = w_R; survivor j is tile element j, no idx).
+// Every lane scores a survivor (gathers: norm, tf of S, tf of R or the previous
+// partial score) and the unit's entries are written contiguously.
 template <int KIND>
-__device__ __forceinline__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u, const TermInfo &tR,
-                          const TermInfo &tS, const uint2 *Rq, const uint32_t *tile,
-                          uint32_t *match, uint32_t *idx, uint32_t ia, uint32_t ib,
-                          uint32_t posR0, Acc &acc) {
+__device__ __forceinline__ void emit_compact(const DevIndex &ix, const RoundArgs &a, uint32_t u,
+                                             const TermInfo &tR, const TermInfo &tS,
+                                             const uint2 *Rq, const uint32_t *tile,
+                                             const uint32_t *idx, const uint32_t *spos,
+                                             uint32_t cnt, uint32_t posR0, Acc &acc) {
+  const uint32_t lane = lane_id();
+  unsigned long long off = 0;
+  if (lane == 0 && cnt) off = bump_alloc(a, acc, cnt);
+  off = __shfl_sync(0xffffffffu, off, 0);
+  if (off + cnt > a.bump_cap) {
+    if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
+    cnt = 0;
+  }
+  for (uint32_t j = lane; j < cnt; j += 32u) {
+    const uint32_t i = KIND == 2 ? j : idx[j];
+    const uint32_t doc = tile[i];
+    const float nrm = __ldg(ix.norm + doc);
+    float s;
+    if (KIND == 2) {
+      s = bm25_w(tR.idf, tf_lookup(ix, tR, posR0 + i), nrm, ix.k1p1);
+    } else {
+      const uint32_t t1 = tf_lookup(ix, tS, spos[j]);
+      const uint32_t t2 = KIND == 0 ? tf_lookup(ix, tR, posR0 + i) : Rq[posR0 + i].y;
+      const float wS = bm25_w(tS.idf, t1, nrm, ix.k1p1);
+      if (KIND == 0) {
+        s = bm25_w(tR.idf, t2, nrm, ix.k1p1);  // first term: s = w
+        s = __fadd_rn(s, wS);
+      } else {
+        s = __fadd_rn(__uint_as_float(t2), wS);
+      }
+    }
+    a.bump[off + j] = make_uint2(doc, __float_as_uint(s));
+  }
+  __syncwarp();
+  if (lane == 0) {
+    a.unit_off[u] = off;
+    a.unit_cnt[u] = cnt;
+    acc.ctr[kCSurv] += cnt;
+    acc.ctr[kCAlg] += (unsigned long long)cnt * (KIND == 0 ? kSurvBytesR1 : kSurvBytes);
+  }
+}
+
+// Emission of the matched R-tile elements [0, n) (match[i] = S position or
+// kNone): compact the matches first (R tile index -> idx[], S position ->
+// match[] in place, in R order), so the scoring loop runs every lane on a
+// survivor instead of one lane in ~three.  idx: >= n words of scratch.
+template <int KIND>
+__device__ __forceinline__ void emit_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u,
+                                          const TermInfo &tR, const TermInfo &tS, const uint2 *Rq,
+                                          const uint32_t *tile, uint32_t *match, uint32_t *idx,
+                                          uint32_t n, uint32_t posR0, Acc &acc) {
   const uint32_t lane = lane_id(), lt = lanemask_lt();
   uint32_t cnt = 0;
   if (KIND == 2) {
-    cnt = ib - ia;
+    cnt = n;
   } else {
-    for (uint32_t c0 = ia; c0 < ib; c0 += 32) {
+    for (uint32_t c0 = 0; c0 < n; c0 += 32) {
       const uint32_t i = c0 + lane;
-      const uint32_t mv = i < ib ? match[i] : kNone;
+      const uint32_t mv = i < n ? match[i] : kNone;
       const bool p = mv != kNone;
       const uint32_t bal = __ballot_sync(0xffffffffu, p);
       __syncwarp();   // every lane has read its match[i] before any compacted write
@@ -474,59 +574,7 @@ __device__ __forceinline__ void emit_unit(const DevIndex &ix, const RoundArgs &a
     }
     __syncwarp();
   }
-  unsigned long long off = 0;
-  if (lane == 0 && cnt) off = bump_alloc(a, acc, cnt);
-  off = __shfl_sync(0xffffffffu, off, 0);
-  if (off + cnt > a.bump_cap) {
-    if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
-    cnt = 0;
-  }
-  constexpr int kDep = KIND == 2 ? 1 : GRIFFIN_UNIT_EMIT_DEPTH;
-  for (uint32_t j0 = 0; j0 < cnt; j0 += 32u * kDep) {
-    uint32_t doc[kDep], t1[kDep], t2[kDep];
-    float nrm[kDep];
-#pragma unroll
-    for (int t = 0; t < kDep; ++t) {
-      const uint32_t j = j0 + 32u * t + lane;
-      if (j < cnt) {
-        const uint32_t i = KIND == 2 ? ia + j : idx[j];
-        doc[t] = tile[i];
-        nrm[t] = __ldg(ix.norm + doc[t]);
-        if (KIND == 2) {
-          t1[t] = tf_lookup(ix, tR, posR0 + i);
-        } else {
-          t1[t] = tf_lookup(ix, tS, match[j]);
-          t2[t] = KIND == 0 ? tf_lookup(ix, tR, posR0 + i) : Rq[posR0 + i].y;
-        }
-      }
-    }
-#pragma unroll
-    for (int t = 0; t < kDep; ++t) {
-      const uint32_t j = j0 + 32u * t + lane;
-      if (j < cnt) {
-        float s;
-        if (KIND == 2) {
-          s = bm25_w(tR.idf, t1[t], nrm[t], ix.k1p1);
-        } else {
-          const float wS = bm25_w(tS.idf, t1[t], nrm[t], ix.k1p1);
-          if (KIND == 0) {
-            s = bm25_w(tR.idf, t2[t], nrm[t], ix.k1p1);  // first term: s = w
-            s = __fadd_rn(s, wS);
-          } else {
-            s = __fadd_rn(__uint_as_float(t2[t]), wS);
-          }
-        }
-        a.bump[off + j] = make_uint2(doc[t], __float_as_uint(s));
-      }
-    }
-  }
-  __syncwarp();
-  if (lane == 0) {
-    a.unit_off[u] = off;
-    a.unit_cnt[u] = cnt;
-    acc.ctr[kCSurv] += cnt;
-    acc.ctr[kCAlg] += (unsigned long long)cnt * (KIND == 0 ? kSurvBytesR1 : kSurvBytes);
-  }
+  emit_compact<KIND>(ix, a, u, tR, tS, Rq, tile, idx, match, cnt, posR0, acc);
 }
 
 // Ordered emission of per-lane match lists (merge units): lane l found c
@@ -670,8 +718,9 @@ __device__ __forceinline__ uint64_t bitmap_unit_bucket(const DevIndex &ix, const
   const uint4 rec = a.urec[u];
   const uint32_t q = rec.x, lu = rec.y;
   const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
-  const uint32_t x0 = RC ? __ldg(ix.first + ix.terms[pt[0]].block0 + lu)
-                         : a.rprev[a.roff_prev[q] + (size_t)lu * ix.B].x;
+  const uint32_t b0 = lu * bm_unit_blocks(ix.B, a.D, a.nextgeq != 0);
+  const uint32_t x0 = RC ? __ldg(ix.first + ix.terms[pt[0]].block0 + b0)
+                         : a.rprev[a.roff_prev[q] + (size_t)b0 * ix.B].x;
   return a.sbkt_nm + (uint64_t)a.bm_slot[pt[a.round]] * a.sbkt_nbb + (x0 >> kBmBucketShift);
 }
 
@@ -1032,6 +1081,46 @@ __device__ __forceinline__ void bitvec_probe(const uint2 *__restrict__ bm,
   __syncwarp();
 }
 
+// Bitvector lookups of the elements x = tileR[0..n), compacted in R order:
+// the j-th hit is tile element idx[j] at S position spos[j]; returns the
+// number of hits.  4 independent 8-B loads in flight per lane.
+__device__ __forceinline__ uint32_t bitvec_probe_compact(const uint2 *__restrict__ bm,
+                                                         const uint32_t *tileR, uint32_t n,
+                                                         uint32_t *idx, uint32_t *spos, int count,
+                                                         Acc &acc) {
+  const uint32_t lane = lane_id(), lt = lanemask_lt();
+  uint32_t sectors = 0, cnt = 0;
+  for (uint32_t base = 0; base < n; base += 128u) {
+    uint32_t x[4];
+    uint2 wv[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t e = base + lane + 32u * j;
+      x[j] = e < n ? tileR[e] : 0u;
+      wv[j] = e < n ? __ldg(bm + (x[j] >> 5)) : make_uint2(0, 0);
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t e = base + lane + 32u * j;
+      const uint32_t p = e < n ? bitvec_pos(wv[j], x[j]) : kNone;
+      const uint32_t bal = __ballot_sync(0xffffffffu, p != kNone);
+      if (p != kNone) {
+        const uint32_t o = cnt + __popc(bal & lt);
+        idx[o] = e;
+        spos[o] = p;
+      }
+      cnt += __popc(bal);
+      if (count && e < n) sectors += (e == 0 || (tileR[e - 1] >> 7) != (x[j] >> 7)) ? 1u : 0u;
+    }
+  }
+  if (count) {
+    const uint32_t sp = __reduce_add_sync(0xffffffffu, sectors);
+    if (lane == 0) acc.ctr[kCAlg] += sp * 32ull;
+  }
+  __syncwarp();
+  return cnt;
+}
+
 // Multi-list probe (SvS rounds 2..m-1 in one pass): every round-1 survivor is
 // looked up in each remaining list in canonical order — skip-pointer search,
 // then an in-place binary search of the decoded-arena block or a staged EF
@@ -1230,7 +1319,7 @@ __host__ __device__ inline uint32_t other_tile_words(uint32_t B, uint32_t D, boo
   return 3u * B + (nextgeq ? 0u : G * B) + kTileSlack;
 }
 __host__ __device__ inline uint32_t other_warp_smem_words(uint32_t B, uint32_t D, bool nextgeq) {
-  return kWarpHdr + 64 + (B + 32) + stage_words(B, D) + kStgSlack + other_tile_words(B, D, nextgeq);
+  return kWarpHdr + 64 + (B + 32) + other_stage_words(B, D) + kStgSlack + other_tile_words(B, D, nextgeq);
 }
 template <int ROLE>
 struct IkMinBlocks { static constexpr int v = ROLE == 2 ? 4 : GRIFFIN_INTERSECT_MINB; };
@@ -1250,7 +1339,7 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
     sm.cnt = wb + kWarpHdr;
     sm.aux = sm.cnt + 64;
     sm.stg = sm.aux + B + 32;
-    sm.tile = sm.stg + stage_words(B, D) + kStgSlack;
+    sm.tile = sm.stg + other_stage_words(B, D) + kStgSlack;
     sm.phase = 0;
   } else {
     sm = carve_warp_smem(smem4, B, D);
@@ -1325,7 +1414,7 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
           acc.ctr[kCAlg] += sz * 16u + 8u;
         }
       }
-      emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, nullptr, 0, n, lu * B, acc);
+      emit_unit<2>(ix, a, (uint32_t)u, tR, tR, nullptr, sm.tile, nullptr, nullptr, n, lu * B, acc);
       continue;
     }
     if (ROLE == 0 && !RC && mode == kModeProbe) {
@@ -1547,6 +1636,67 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
                           sb0 * B + sa, smem_u32(sm.tile) & 0xFFFFu,
                           smem_u32(tileS + sa) & 0xFFFFu, acc);
       __syncwarp();
+    } else if (ROLE != 1 && mode == kModeBitmap) {
+      // ---- S decoded into a bitvector this batch: R blocks [b0, b0+nb) (or
+      // intermediate chunks) looked up in O(1), hits compacted, then scored ----
+      const uint32_t U = bm_unit_blocks(B, D, a.nextgeq != 0);
+      const uint32_t b0 = lu * U, nb = min(U, nbR - b0), s0 = b0 * B;
+      const uint32_t n = min(U * B, nR - s0);
+      uint32_t *tileR = sm.tile, *idx = sm.stg;   // idx: the staging area, free after decode
+      uint32_t *spos = bm_spos_in_tile(B, D, a.nextgeq != 0, ROLE == 2, U) ? sm.tile + U * B
+                                                                             : sm.stg + U * B;
+      if (RC && rdec) {
+        const uint32_t by = ((n + 3u) & ~3u) * 4u;
+        if (lane == 0) {
+          fence_proxy_async();
+          mbar_expect_tx(sm.mbar, by);
+          bulk_g2s(tileR, decR + s0, by, sm.mbar);
+        }
+        mbar_wait(sm.mbar, sm.phase);
+        sm.phase ^= 1u;
+        if (a.count) {
+          const uint32_t c = lane < nb ? block_size16(ix.meta[(uint64_t)tR.block0 + b0 + lane].y) * 16u + 8u : 0u;
+          const uint32_t sc = __reduce_add_sync(0xffffffffu, c);
+          if (lane == 0) {
+            acc.ctr[kCAlg] += n * 4u;
+            acc.ctr[kCApost] += n;
+            acc.ctr[kCAcomp] += sc;
+          }
+        }
+      } else if (RC) {
+        uint2 m = make_uint2(0, 0);
+        uint32_t f = 0, sz = 0;
+        if (lane < nb) {
+          const uint64_t gb = (uint64_t)tR.block0 + b0 + lane;
+          m = ix.meta[gb];
+          f = ix.first[gb];
+          sz = block_size16(m.y);
+        }
+        stage_decode_lanes<kIkPair>(ix, sm, stage_words(B, D) / 4u, 0, nb, m, f, sz, tileR);
+        if (a.count) {
+          const uint32_t sp = __reduce_add_sync(0xffffffffu, sz) * 16u;
+          if (lane == 0) {
+            acc.ctr[kCPay] += sp;
+            acc.ctr[kCPost] += n;
+            acc.ctr[kCAlg] += sp + 8u * nb;
+          }
+        }
+      } else {
+        for (uint32_t i = lane; i < n; i += 32) tileR[i] = Rq[s0 + i].x;
+        if (a.count && lane == 0) acc.ctr[kCAlg] += n * 8u;
+      }
+      __syncwarp();
+      if (a.count && lane == 0) {
+        atomicAdd(a.scal + kScalDiag2, 1ull);
+        atomicAdd(a.scal + kScalDiag2 + 1, (unsigned long long)n);
+      }
+      const uint32_t cnt = bitvec_probe_compact(a.bm + (size_t)a.bm_slot[tSid] * a.bm_words, tileR,
+                                                n, idx, spos, a.count, acc);
+      if (RC)
+        emit_compact<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, idx, spos, cnt, s0, acc);
+      else
+        emit_compact<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, idx, spos, cnt, s0, acc);
+      __syncwarp();
     } else if (ROLE != 1) {
       // ---- gallop: R chunk lu, skip-pointer search into S (Fig. 9) ----
       uint32_t *tileR = sm.tile, *kidx = sm.tile + B, *match = sm.tile + 2 * B;
@@ -1584,20 +1734,6 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
         if (lane == 0) acc.ctr[kCAlg] += n * 8u;
       }
       __syncwarp();
-      if (mode == kModeBitmap) {
-        // S decoded into a bitvector this batch: O(1) lookups of the R chunk
-        if (a.count && lane == 0) {
-          atomicAdd(a.scal + kScalDiag2, 1ull);
-          atomicAdd(a.scal + kScalDiag2 + 1, (unsigned long long)n);
-        }
-        bitvec_probe(a.bm + (size_t)a.bm_slot[tSid] * a.bm_words, tileR, match, n, a.count, acc);
-        if (RC)
-          emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
-        else
-          emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
-        __syncwarp();
-        continue;
-      }
       const uint32_t k_lo = rec.z, k_hi = rec.w;   // from the partition stage
       if (a.count && lane == 0) {
         atomicAdd(a.scal + kScalDiag + 2, 1ull);
@@ -1638,9 +1774,9 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
         if (lane == 0) acc.ctr[kCAlg] += sp * 32ull;
         __syncwarp();
         if (RC)
-          emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
+          emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, n, lu * B, acc);
         else
-          emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
+          emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, n, lu * B, acc);
         __syncwarp();
         continue;
       }
@@ -1759,9 +1895,9 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
         g0 += ng;
       }
       if (RC)
-        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
+        emit_unit<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, n, lu * B, acc);
       else
-        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, 0, n, lu * B, acc);
+        emit_unit<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, match, kidx, n, lu * B, acc);
       __syncwarp();
     }
   }
