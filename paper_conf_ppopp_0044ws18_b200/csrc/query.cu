@@ -710,17 +710,29 @@ __device__ __forceinline__ uint32_t merge_unit_bucket(const DevIndex &ix, const 
   return (ix.terms[sid].block0 + rec.z) >> a.sbkt_shift;
 }
 
-// bucket of bitvector unit u (R chunk lu of query q): its S bitvector slot and
-// the chunk's first R docID
+// Units handed out in bitvector order (after the merge buckets): bitvector
+// units, and probe-pass units whose first remaining list is a bitvector.
+__device__ __forceinline__ bool bm_bucketed(const RoundArgs &a, uint32_t q) {
+  const uint32_t md = a.qmode[q];
+  return a.sbkt_nbb && (md == kModeBitmap ||
+                        (md == kModeProbe && a.tdec &&
+                         a.tdec[a.plan_terms[(size_t)q * kMaxTerms + a.round]] == kDecBitmap));
+}
+// its bucket: the bitvector's slot and the unit's first R docID
 template <bool RC>
 __device__ __forceinline__ uint64_t bitmap_unit_bucket(const DevIndex &ix, const RoundArgs &a,
                                                        uint64_t u) {
   const uint4 rec = a.urec[u];
   const uint32_t q = rec.x, lu = rec.y;
   const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
-  const uint32_t b0 = lu * bm_unit_blocks(ix.B, a.D, a.nextgeq != 0);
-  const uint32_t x0 = RC ? __ldg(ix.first + ix.terms[pt[0]].block0 + b0)
-                         : a.rprev[a.roff_prev[q] + (size_t)b0 * ix.B].x;
+  uint32_t x0;
+  if (a.qmode[q] == kModeProbe) {
+    x0 = a.rprev[a.roff_prev[q] + (size_t)lu * a.pchunk].x;
+  } else {
+    const uint32_t b0 = lu * bm_unit_blocks(ix.B, a.D, a.nextgeq != 0);
+    x0 = RC ? __ldg(ix.first + ix.terms[pt[0]].block0 + b0)
+            : a.rprev[a.roff_prev[q] + (size_t)b0 * ix.B].x;
+  }
   return a.sbkt_nm + (uint64_t)a.bm_slot[pt[a.round]] * a.sbkt_nbb + (x0 >> kBmBucketShift);
 }
 
@@ -746,7 +758,7 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
     if (valid) q = a.urec[u].x;
     const bool mg = valid && a.qmode[q] == kModeMerge;
     // bitvector units are bucketed too when the order is on (after the merge units)
-    const bool bu = valid && a.sbkt_cnt && a.sbkt_nbb && a.qmode[q] == kModeBitmap;
+    const bool bu = valid && a.sbkt_cnt && bm_bucketed(a, q);
     const uint32_t bm = __ballot_sync(0xffffffffu, mg),
                    bo = __ballot_sync(0xffffffffu, valid && !mg && !bu);
     const uint32_t lane = threadIdx.x & 31u, lt = (1u << lane) - 1u;
@@ -785,7 +797,7 @@ __global__ void sorder_scatter_kernel(DevIndex ix, RoundArgs a) {
   for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < total; u += stride) {
     const uint32_t q = a.urec[u].x;
     const uint32_t md = a.qmode[q];
-    if (md != kModeMerge && !(md == kModeBitmap && a.sbkt_nbb)) continue;
+    if (md != kModeMerge && !bm_bucketed(a, q)) continue;
     const uint64_t bk = md == kModeMerge ? merge_unit_bucket(ix, a, u) : bitmap_unit_bucket<RC>(ix, a, u);
     const unsigned long long slot = atomicAdd(a.sbkt_pos + bk, 1ull);
     a.uperm[slot] = (uint32_t)u;
@@ -3025,7 +3037,9 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
       ra.sbkt_cnt = nullptr;
       ra.sbkt_pos = nullptr;
       uint64_t nbkt = 0;
-      if (ix->sorder && nq >= kSorderMinQueries && (r == 1 || !ra.probe) && w.sbkt_cnt.p) {
+      // (the probe pass has no merge units; it orders its units by their first
+      // remaining list's bitvector when that list has one)
+      if (ix->sorder && nq >= kSorderMinQueries && (r == 1 || !ra.probe || ra.bm) && w.sbkt_cnt.p) {
         ra.sbkt_shift = ix->sorder_shift;
         ra.sbkt_nm = sorder_merge_buckets(ix);
         ra.sbkt_nbb = sorder_bm_per_slot(ix);
