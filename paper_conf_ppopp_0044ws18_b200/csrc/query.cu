@@ -502,12 +502,16 @@ __device__ __forceinline__ uint32_t load_r_chunk(const uint2 *Rq, uint32_t nR, u
 // w_S); KIND 2: single-term (s = w_R; survivor j is tile element j, no idx).
 // Every lane scores a survivor (gathers: norm, tf of S, tf of R or the previous
 // partial score) and the unit's entries are written contiguously.
+// rtf (KIND 0, optional): R's packed tf words from bit rtf_bit0 on, staged in
+// shared memory, so R's tf is read there instead of gathered.
 template <int KIND>
 __device__ __forceinline__ void emit_compact(const DevIndex &ix, const RoundArgs &a, uint32_t u,
                                              const TermInfo &tR, const TermInfo &tS,
                                              const uint2 *Rq, const uint32_t *tile,
                                              const uint32_t *idx, const uint32_t *spos,
-                                             uint32_t cnt, uint32_t posR0, Acc &acc) {
+                                             uint32_t cnt, uint32_t posR0, Acc &acc,
+                                             const uint32_t *rtf = nullptr,
+                                             uint64_t rtf_bit0 = 0) {
   const uint32_t lane = lane_id();
   unsigned long long off = 0;
   if (lane == 0 && cnt) off = bump_alloc(a, acc, cnt);
@@ -525,7 +529,14 @@ __device__ __forceinline__ void emit_compact(const DevIndex &ix, const RoundArgs
       s = bm25_w(tR.idf, tf_lookup(ix, tR, posR0 + i), nrm, ix.k1p1);
     } else {
       const uint32_t t1 = tf_lookup(ix, tS, spos[j]);
-      const uint32_t t2 = KIND == 0 ? tf_lookup(ix, tR, posR0 + i) : Rq[posR0 + i].y;
+      uint32_t t2;
+      if (KIND == 0 && rtf) {
+        const uint32_t bit = (uint32_t)((uint64_t)(posR0 + i) * tR.tf_w - rtf_bit0);
+        t2 = (__funnelshift_r(rtf[bit >> 5], rtf[(bit >> 5) + 1], bit) &
+              (0xFFFFFFFFu >> (32u - tR.tf_w))) + 1u;
+      } else {
+        t2 = KIND == 0 ? tf_lookup(ix, tR, posR0 + i) : Rq[posR0 + i].y;
+      }
       const float wS = bm25_w(tS.idf, t1, nrm, ix.k1p1);
       if (KIND == 0) {
         s = bm25_w(tR.idf, t2, nrm, ix.k1p1);  // first term: s = w
@@ -1096,36 +1107,52 @@ __device__ __forceinline__ void bitvec_probe(const uint2 *__restrict__ bm,
 // Bitvector lookups of the elements x = tileR[0..n), compacted in R order:
 // the j-th hit is tile element idx[j] at S position spos[j]; returns the
 // number of hits.  4 independent 8-B loads in flight per lane.
+// 128 elements from base (4 per lane, independent loads in flight); FULL: no
+// bounds checks (every element < n)
+template <bool FULL>
+__device__ __forceinline__ void bitvec_chunk(const uint2 *__restrict__ bm, const uint32_t *tileR,
+                                             uint32_t base, uint32_t n, uint32_t *idx,
+                                             uint32_t *spos, uint32_t &cnt) {
+  const uint32_t lane = lane_id(), lt = lanemask_lt();
+  uint32_t x[4];
+  uint2 wv[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const uint32_t e = base + lane + 32u * j;
+    const bool in = FULL || e < n;
+    x[j] = in ? tileR[e] : 0u;
+    wv[j] = in ? __ldg(bm + (x[j] >> 5)) : make_uint2(0, 0);
+  }
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const uint32_t bit = x[j] & 31u;
+    const bool hit = (wv[j].x >> bit) & 1u;   // (0 for out-of-range lanes: word 0 loaded as zero)
+    const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+    if (hit) {
+      const uint32_t o = cnt + __popc(bal & lt);
+      idx[o] = base + lane + 32u * j;
+      spos[o] = ~wv[j].y + __popc(wv[j].x & ((1u << bit) - 1u));
+    }
+    cnt += __popc(bal);
+  }
+}
+
+// Bitvector lookups of the elements x = tileR[0..n), compacted in R order:
+// the j-th hit is tile element idx[j] at S position spos[j]; returns the
+// number of hits.  Counting pass: one 32-B sector per distinct sector the
+// warp reads in list order (SURVEY §8(d) charges gathers by sector).
 __device__ __forceinline__ uint32_t bitvec_probe_compact(const uint2 *__restrict__ bm,
                                                          const uint32_t *tileR, uint32_t n,
                                                          uint32_t *idx, uint32_t *spos, int count,
                                                          Acc &acc) {
-  const uint32_t lane = lane_id(), lt = lanemask_lt();
-  uint32_t sectors = 0, cnt = 0;
-  for (uint32_t base = 0; base < n; base += 128u) {
-    uint32_t x[4];
-    uint2 wv[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const uint32_t e = base + lane + 32u * j;
-      x[j] = e < n ? tileR[e] : 0u;
-      wv[j] = e < n ? __ldg(bm + (x[j] >> 5)) : make_uint2(0, 0);
-    }
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const uint32_t e = base + lane + 32u * j;
-      const uint32_t p = e < n ? bitvec_pos(wv[j], x[j]) : kNone;
-      const uint32_t bal = __ballot_sync(0xffffffffu, p != kNone);
-      if (p != kNone) {
-        const uint32_t o = cnt + __popc(bal & lt);
-        idx[o] = e;
-        spos[o] = p;
-      }
-      cnt += __popc(bal);
-      if (count && e < n) sectors += (e == 0 || (tileR[e - 1] >> 7) != (x[j] >> 7)) ? 1u : 0u;
-    }
-  }
+  const uint32_t lane = lane_id();
+  uint32_t cnt = 0, base = 0;
+  for (; base + 128u <= n; base += 128u) bitvec_chunk<true>(bm, tileR, base, n, idx, spos, cnt);
+  if (base < n) bitvec_chunk<false>(bm, tileR, base, n, idx, spos, cnt);
   if (count) {
+    uint32_t sectors = 0;
+    for (uint32_t e = lane; e < n; e += 32u)
+      sectors += (e == 0 || (tileR[e - 1] >> 7) != (tileR[e] >> 7)) ? 1u : 0u;
     const uint32_t sp = __reduce_add_sync(0xffffffffu, sectors);
     if (lane == 0) acc.ctr[kCAlg] += sp * 32ull;
   }
@@ -1702,10 +1729,25 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
         atomicAdd(a.scal + kScalDiag2, 1ull);
         atomicAdd(a.scal + kScalDiag2 + 1, (unsigned long long)n);
       }
+      // round 1: R's tf words for positions [s0, s0+n) staged (coalesced) in
+      // the aux area when they fit — survivors read R's tf there
+      const uint32_t *rtf = nullptr;
+      uint64_t rtf_bit0 = 0;
+      if (RC && tR.tf_w) {
+        const uint64_t b0w = ((uint64_t)s0 * tR.tf_w) >> 5;
+        const uint64_t b1w = ((uint64_t)(s0 + n) * tR.tf_w + 31u) >> 5;
+        const uint32_t nw = (uint32_t)(b1w - b0w) + 1u;   // + the funnel's look-ahead word
+        if (nw <= B + 32u) {
+          for (uint32_t i = lane; i < nw; i += 32u) sm.aux[i] = __ldg(ix.tfw + tR.tf_off + b0w + i);
+          rtf = sm.aux;
+          rtf_bit0 = b0w * 32u;
+        }
+      }
       const uint32_t cnt = bitvec_probe_compact(a.bm + (size_t)a.bm_slot[tSid] * a.bm_words, tileR,
                                                 n, idx, spos, a.count, acc);
       if (RC)
-        emit_compact<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, idx, spos, cnt, s0, acc);
+        emit_compact<0>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, idx, spos, cnt, s0, acc, rtf,
+                        rtf_bit0);
       else
         emit_compact<1>(ix, a, (uint32_t)u, tR, tS, Rq, tileR, idx, spos, cnt, s0, acc);
       __syncwarp();
