@@ -166,42 +166,48 @@ struct BitSink {
   uint2 *bm;              // the list's bitvector
   const uint32_t *tile;   // decoder destination base
   uint32_t pos0;          // list position of tile[0]
-  uint32_t cw = 0xFFFFFFFFu, bits = 0, fpos = 0, lpos = 0;
+  uint32_t cw = 0xFFFFFFFFu, bits = 0, fpos = 0, lpos = 0xFFFFFFFEu;
   bool cf = false;        // the run's predecessor was seen here (in another word)
-  __device__ __forceinline__ void flush(bool cl) {
-    if (cw == 0xFFFFFFFFu) return;
-    if (cf && cl) {
-      bm[cw] = make_uint2(bits, ~fpos);
-    } else {
+  // flush the current run if `fl`; cl = its successor was seen here.  Written
+  // as predicated code: lanes break runs at different elements, so a branch
+  // would serialise the flush for almost every element of a warp.
+  __device__ __forceinline__ void flush_if(bool fl, bool cl) {
+    const bool own = fl && cf && cl;
+    if (own) bm[cw] = make_uint2(bits, ~fpos);
+    if (fl && !own) {
       atomicOr(&bm[cw].x, bits);
       atomicMax(&bm[cw].y, ~fpos);
     }
   }
-  __device__ __forceinline__ void add(uint32_t pos, uint32_t v) {
+  // element v at list position pos; contig = pos follows the previous element
+  __device__ __forceinline__ void add(uint32_t pos, uint32_t v, bool contig) {
     const uint32_t w = v >> 5;
-    const bool contig = cw != 0xFFFFFFFFu && pos == lpos + 1u;
-    if (w != cw || !contig) {
-      flush(contig);   // the successor (this element) is here, in another word
-      cf = contig;
-      cw = w;
-      bits = 0;
-      fpos = pos;
-    }
-    bits |= 1u << (v & 31u);
-    lpos = pos;
+    const bool brk = w != cw || !contig;
+    flush_if(brk && cw != 0xFFFFFFFFu, contig);
+    cf = brk ? contig : cf;
+    fpos = brk ? pos : fpos;
+    bits = (brk ? 0u : bits) | (1u << (v & 31u));
+    cw = w;
   }
   __device__ __forceinline__ void put4(uint32_t *p, uint4 v) {
     const uint32_t pos = pos0 + (uint32_t)(p - tile);
-    add(pos, v.x);
-    add(pos + 1u, v.y);
-    add(pos + 2u, v.z);
-    add(pos + 3u, v.w);
+    const bool c0 = pos == lpos + 1u;   // the four are consecutive positions
+    add(pos, v.x, c0);
+    add(pos + 1u, v.y, true);
+    add(pos + 2u, v.z, true);
+    add(pos + 3u, v.w, true);
+    lpos = pos + 3u;
   }
-  __device__ __forceinline__ void put(uint32_t *p, uint32_t v) { add(pos0 + (uint32_t)(p - tile), v); }
+  __device__ __forceinline__ void put(uint32_t *p, uint32_t v) {
+    const uint32_t pos = pos0 + (uint32_t)(p - tile);
+    add(pos, v, pos == lpos + 1u);
+    lpos = pos;
+  }
   // end of this lane's elements: its last run may share its word
   __device__ __forceinline__ void finish() {
-    flush(false);
+    flush_if(cw != 0xFFFFFFFFu, false);
     cw = 0xFFFFFFFFu;
+    lpos = 0xFFFFFFFEu;   // the next element never continues this run
   }
 };
 // Bitvector lookup of docID x: its list position, or kNone if absent.

@@ -2672,6 +2672,9 @@ __global__ void bm_zero_kernel(const uint8_t *tdec, const uint32_t *bm_term, uin
   }
 }
 
+#ifndef GRIFFIN_DECODE_ONCE_MINB
+#define GRIFFIN_DECODE_ONCE_MINB 3
+#endif
 // Para-EF decode of every block of the selected terms into the arena
 // (slot = global block * B + i): warp per run of <= D+2 consecutive blocks,
 // TMA-staged payloads, decoded tile written back with 128-bit stores.
@@ -2685,7 +2688,7 @@ __global__ void run_map_kernel(uint32_t V, const uint32_t *runs, const uint64_t 
   for (uint32_t i = lane_id(); i < nr; i += 32) run_term[b + i] = t;
 }
 
-__global__ void __launch_bounds__(256, 3) decode_once_kernel(DevIndex ix, uint32_t D,
+__global__ void __launch_bounds__(256, GRIFFIN_DECODE_ONCE_MINB) decode_once_kernel(DevIndex ix, uint32_t D,
                                                           const uint64_t *run_base,
                                                           const uint32_t *run_term, uint32_t *arena,
                                                           const uint8_t *tdec, uint2 *bm,
