@@ -2088,19 +2088,50 @@ __global__ void __launch_bounds__(256) compact_copy_kernel(RoundArgs a, const ui
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); u < total;
        u += nwarps) {
-    const uint32_t q = a.urec[u].x;   // the partition stage's record
     const uint64_t my = udst[u];
-    const uint64_t base = udst[ubase[q]];
     const uint32_t cnt = a.unit_cnt[u];
     const uint2 *src = a.bump + a.unit_off[u];
-    uint2 *dst = a.rnext + (packed ? my : a.roff_next[q] + (my - base));
-    for (uint32_t i = lane; i < cnt; i += 32) dst[i] = src[i];
-    if (lane == 0 && u + 1 == ubase[q + 1]) {
-      a.rcount[q] = (uint32_t)(my + cnt - base);
-      a.rsel[q] = (uint8_t)(a.round & 1u);
-      if (packed) a.roff_next[q] = base;
+    uint2 *dst;
+    if (packed) {   // rounds 1-2: the packed offset (per-query bookkeeping: compact_queries_kernel)
+      dst = a.rnext + my;
+    } else {
+      const uint32_t q = a.urec[u].x;   // the partition stage's record
+      const uint64_t base = udst[ubase[q]];
+      dst = a.rnext + a.roff_next[q] + (my - base);
+      if (lane == 0 && u + 1 == ubase[q + 1]) {
+        a.rcount[q] = (uint32_t)(my + cnt - base);
+        a.rsel[q] = (uint8_t)(a.round & 1u);
+      }
+    }
+    // four entries per lane in flight
+    for (uint32_t i0 = 0; i0 < cnt; i0 += 128u) {
+      uint2 v[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t i = i0 + 32u * j + lane;
+        if (i < cnt) v[j] = src[i];
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t i = i0 + 32u * j + lane;
+        if (i < cnt) dst[i] = v[j];
+      }
     }
   }
+}
+
+// Packed rounds: per query, its survivors' count, buffer and packed offset
+// (the exclusive scan of its units' counts; rtot = the round's total).
+__global__ void compact_queries_kernel(RoundArgs a, const uint64_t *udst) {
+  const uint32_t q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q >= a.nq || a.scal[kScalRoundTot] > a.entry_cap) return;
+  const uint64_t total = a.unit_base[a.nq], rtot = a.scal[kScalRoundTot];
+  const uint64_t u0 = a.unit_base[q], u1 = a.unit_base[q + 1];
+  if (u0 == u1) return;   // no units this round: the query's count stays as planned (0)
+  const uint64_t b0 = udst[u0], b1 = u1 < total ? udst[u1] : rtot;
+  a.rcount[q] = (uint32_t)(b1 - b0);
+  a.rsel[q] = (uint8_t)(a.round & 1u);
+  a.roff_next[q] = b0;
 }
 
 // Query q's final intermediate: buffer rsel[q] at q's offset in that buffer
@@ -3130,6 +3161,10 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
       unit_scan_apply<<<tiles, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum,
                                                       w.unit_dst.as<uint64_t>());
       compact_copy_kernel<<<num_sms(ix->device) * 8, 256, 0, st>>>(ra, w.unit_dst.as<uint64_t>());
+      if (r <= 2) {
+        compact_queries_kernel<<<qblocks, 256, 0, st>>>(ra, w.unit_dst.as<uint64_t>());
+        ix->launch_count += 1;
+      }
       GRIFFIN_CUDA_TRY(cudaGetLastError());
       ix->launch_count += 4;  // sums, single, apply, copy
     }
