@@ -138,7 +138,8 @@ struct RoundArgs {
   uint64_t bump_cap;      // entries of the bump area (entry_cap + per-warp chunk slack)
   unsigned long long *scal;
   uint4 *urec;            // per unit: {q, i0|lu, j0, lo docID} (partition stage)
-  uint32_t *uperm;        // processing order of the units: merge units first, then the rest
+  uint4 *uperm;           // processing order of the units (merge units first, then the rest):
+                          // {unit, query | mode << 29, R term, S term} (uperm_entry)
   uint32_t *sbkt_cnt;     // S-locality order: merge units per bucket of S blocks (or null)
   unsigned long long *sbkt_pos;   // bucket cursors (exclusive scan of sbkt_cnt)
   uint32_t sbkt_shift;    // bucket = global S block of the unit's start >> shift

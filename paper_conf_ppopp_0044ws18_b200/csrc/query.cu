@@ -721,6 +721,14 @@ __device__ __forceinline__ uint32_t merge_unit_bucket(const DevIndex &ix, const 
   return (ix.terms[sid].block0 + rec.z) >> a.sbkt_shift;
 }
 
+// Processing-order entry of unit u of query q: {u, q | mode << 29, R term,
+// this round's S term}, so a kernel's unit head needs one dependent load (this
+// entry) before it can fetch the unit record and both TermInfos in parallel.
+__device__ __forceinline__ uint4 uperm_entry(const RoundArgs &a, uint64_t u, uint32_t q) {
+  const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
+  return make_uint4((uint32_t)u, q | (a.qmode[q] << 29), pt[0], pt[a.round % kMaxTerms]);
+}
+
 // Units handed out in bitvector order (after the merge buckets): bitvector
 // units, and probe-pass units whose first remaining list is a bitvector.
 __device__ __forceinline__ bool bm_bucketed(const RoundArgs &a, uint32_t q) {
@@ -782,11 +790,11 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
     ho = __shfl_sync(0xffffffffu, ho, 0);
     if (mg) {
       if (a.sbkt_cnt) atomicAdd(a.sbkt_cnt + merge_unit_bucket(ix, a, u), 1u);
-      else a.uperm[hm + __popc(bm & lt)] = (uint32_t)u;
+      else a.uperm[hm + __popc(bm & lt)] = uperm_entry(a, u, q);
     } else if (bu) {
       atomicAdd(a.sbkt_cnt + bitmap_unit_bucket<RC>(ix, a, u), 1u);
     } else if (valid) {
-      a.uperm[total - 1 - (ho + __popc(bo & lt))] = (uint32_t)u;
+      a.uperm[total - 1 - (ho + __popc(bo & lt))] = uperm_entry(a, u, q);
     }
   }
 }
@@ -811,7 +819,7 @@ __global__ void sorder_scatter_kernel(DevIndex ix, RoundArgs a) {
     if (md != kModeMerge && !bm_bucketed(a, q)) continue;
     const uint64_t bk = md == kModeMerge ? merge_unit_bucket(ix, a, u) : bitmap_unit_bucket<RC>(ix, a, u);
     const unsigned long long slot = atomicAdd(a.sbkt_pos + bk, 1ull);
-    a.uperm[slot] = (uint32_t)u;
+    a.uperm[slot] = uperm_entry(a, u, q);
   }
 }
 
@@ -1409,14 +1417,12 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
     const uint64_t tk = __shfl_sync(0xffffffffu, ticket, 0);
     if (tk >= total) break;
     if (lane == 0) ticket = tk0 + atomicAdd(ctr, 1ull);
-    const uint64_t u = a.uperm[tk];   // merge units first (see partition_kernel)
+    const uint4 pe = a.uperm[tk];   // merge units first (see partition_kernel)
+    const uint64_t u = pe.x;
+    const uint32_t q = pe.y & 0x1FFFFFFFu, mode = pe.y >> 29, t0 = pe.z, tSid = pe.w;
     const uint4 rec = a.urec[u];
     const uint4 nxt = a.urec[u + 1];
-    const uint32_t q = rec.x;
     const uint32_t lu = rec.y;   // gallop/all: unit index within the query
-    const uint32_t mode = a.qmode[q];
-    const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
-    const uint32_t t0 = pt[0];
     const TermInfo tR = ix.terms[t0];
     const uint2 *Rq = RC ? nullptr : a.rprev + a.roff_prev[q];
     const uint32_t nR = RC ? tR.df_local : a.rcount[q];
@@ -1460,7 +1466,6 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
       probe_unit(ix, a, sm, u, q, lu, acc);
       continue;
     }
-    const uint32_t tSid = pt[a.round];
     const TermInfo tS = ix.terms[tSid];
     const uint32_t *fS = ix.first + tS.block0;
     const uint32_t nbS = tS.nblocks;
@@ -2001,7 +2006,7 @@ __global__ void __launch_bounds__(kIntersectThreads, 4) probe_kernel(DevIndex ix
     const uint64_t tk = __shfl_sync(0xffffffffu, ticket, 0);
     if (tk >= total) break;
     if (lane == 0) ticket = atomicAdd(a.scal + kScalUnitCtr, 1ull);
-    const uint64_t u = a.uperm[tk];
+    const uint64_t u = a.uperm[tk].x;
     const uint4 rec = a.urec[u];
     probe_unit(ix, a, sm, u, rec.x, rec.y, acc);   // every unit of the pass is a probe unit
   }
@@ -2816,7 +2821,7 @@ griffin_status reserve_ws(griffin_index *ix, Workspace &w, uint32_t nq, uint64_t
   GRIFFIN_CUDA_TRY(w.unit_off.reserve((units + 1) * 8));
   GRIFFIN_CUDA_TRY(w.unit_cnt.reserve((units + 1) * 4));
   GRIFFIN_CUDA_TRY(w.urec.reserve((units + 2) * 16));
-  GRIFFIN_CUDA_TRY(w.uperm.reserve((units + 2) * 4));
+  GRIFFIN_CUDA_TRY(w.uperm.reserve((units + 2) * 16));
   GRIFFIN_CUDA_TRY(w.unit_dst.reserve((units + 2) * 8 + (units / kScanTile + 2) * 8));
   if (ix->sorder && nq >= kSorderMinQueries) {   // S-locality buckets (no allocation in run_batch)
     griffin_status bs = ensure_bm_slots(ix);
@@ -2984,6 +2989,10 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
                          const uint32_t *d_terms, uint32_t max_terms, uint32_t k, uint64_t *d_keys,
                          uint32_t *d_counts, cudaStream_t st, bool final_topk, int forced_mode) {
   if (nq == 0) return GRIFFIN_OK;
+  if (nq >= (1u << 29)) {   // unit order entries pack the query index in 29 bits
+    set_error("a batch holds at most 2^29 - 1 queries");
+    return GRIFFIN_ERR_INVALID_ARG;
+  }
   if (nq > w.nq_cap || !w.scal.p) {
     set_error("workspace not reserved for this batch (call griffin_reserve)");
     return GRIFFIN_ERR_INVALID_ARG;
@@ -3009,7 +3018,7 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
   ra.unit_off = w.unit_off.as<uint64_t>();
   ra.unit_cnt = w.unit_cnt.as<uint32_t>();
   ra.urec = w.urec.as<uint4>();
-  ra.uperm = w.uperm.as<uint32_t>();
+  ra.uperm = w.uperm.as<uint4>();
   ra.unit_cap = w.unit_cap;
   ra.bump = w.bump.as<uint2>();
   ra.entry_cap = w.entry_cap;
