@@ -405,7 +405,7 @@ def run_gpu(args):
     cnt = ix.griffin_get_profile()
     for kk in ("alg_bytes", "c8d_bytes", "payload_bytes", "decoded_postings", "survivors",
                "dec_alg_bytes", "dec_c8d_bytes", "dec_postings", "arena_postings", "merge_units",
-               "merge_elems", "gallop_units", "gallop_elems", "bitmap_units", "bitmap_elems"):
+               "merge_elems", "gallop_units", "gallop_elems", "bitmap_units", "bitmap_elems", "bitand_units", "bitand_words"):
         prof[kk] = cnt[kk]
     ix.griffin_sync_status()
     iso_ms = sum(iso)
@@ -437,7 +437,8 @@ def run_gpu(args):
     kernels["intersect_kernel"]["arena_postings_per_step"] = prof["arena_postings"] / n_iso
     kernels["intersect_kernel"]["units_per_step"] = {
         kk: prof[kk] / n_iso for kk in ("merge_units", "merge_elems", "gallop_units", "gallop_elems",
-                                        "bitmap_units", "bitmap_elems")}
+                                        "bitmap_units", "bitmap_elems", "bitand_units",
+                                        "bitand_words")}
     stage_ms = {kk: prof[kk] / n_iso for kk in
                 ("ms_plan", "ms_decode", "ms_intersect", "ms_compact", "ms_topk", "ms_merge")}
     dom = max(kernels, key=lambda n: kernels[n]["ms_per_step"])

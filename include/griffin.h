@@ -166,8 +166,9 @@ typedef struct {
   /* unit shapes (counters mode): merge units and the elements they merged (R+S
    * inside their docID ranges), gallop units and their R elements */
   uint64_t merge_units, merge_elems, gallop_units, gallop_elems;
-  /* bitvector units (griffin_set_bitmap) and their R elements looked up */
-  uint64_t bitmap_units, bitmap_elems;
+  /* bitvector units (griffin_set_bitmap) and their R elements looked up;
+   * word-AND units (both lists of a round-1 pair are bitvectors) and their words */
+  uint64_t bitmap_units, bitmap_elems, bitand_units, bitand_words;
 } griffin_profile;
 
 /* ---- index ------------------------------------------------------------------

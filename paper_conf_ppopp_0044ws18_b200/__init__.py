@@ -77,7 +77,8 @@ class Profile(ctypes.Structure):
                 ("arena_postings", ctypes.c_uint64), ("merge_units", ctypes.c_uint64),
                 ("merge_elems", ctypes.c_uint64), ("gallop_units", ctypes.c_uint64),
                 ("gallop_elems", ctypes.c_uint64),
-                ("bitmap_units", ctypes.c_uint64), ("bitmap_elems", ctypes.c_uint64)]
+                ("bitmap_units", ctypes.c_uint64), ("bitmap_elems", ctypes.c_uint64),
+                ("bitand_units", ctypes.c_uint64), ("bitand_words", ctypes.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

@@ -971,7 +971,7 @@ griffin_status griffin_reset_profile(griffin_index *ix) {
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDec, 0, 3 * 8));
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalArena, 0, 3 * 8));
       GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDiag, 0, 4 * 8));
-      GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDiag2, 0, 2 * 8));
+      GRIFFIN_CUDA_TRY(cudaMemset(w->scal.as<unsigned long long>() + kScalDiag2, 0, 4 * 8));
     }
   return GRIFFIN_OK;
 }
@@ -1002,7 +1002,7 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
   out->dec_alg_bytes = out->dec_payload_bytes = out->dec_postings = 0;
   out->c8d_bytes = out->dec_c8d_bytes = out->arena_postings = 0;
   out->merge_units = out->merge_elems = out->gallop_units = out->gallop_elems = 0;
-  out->bitmap_units = out->bitmap_elems = 0;
+  out->bitmap_units = out->bitmap_elems = out->bitand_units = out->bitand_words = 0;
   for (Workspace *w : all) {
     if (!w->scal.p) continue;
     unsigned long long c[kScalCount];
@@ -1023,6 +1023,8 @@ griffin_status griffin_get_profile(griffin_index *ix, griffin_profile *out) {
     out->gallop_elems += c[kScalDiag + 3];
     out->bitmap_units += c[kScalDiag2];
     out->bitmap_elems += c[kScalDiag2 + 1];
+    out->bitand_units += c[kScalDiag2 + 2];
+    out->bitand_words += c[kScalDiag2 + 3];
   }
   return GRIFFIN_OK;
 }

@@ -29,7 +29,9 @@ enum : int { kStatusBadTerm = 1, kStatusOverflow = 2, kStatusTooManyTerms = 4 };
 
 // Query modes per (query, round).
 enum : uint32_t { kModeNone = 0, kModeMerge = 1, kModeGallop = 2, kModeAll = 3, kModeProbe = 4,
-                  kModeBitmap = 5 };
+                  kModeBitmap = 5, kModeBitAnd = 6 };
+// word-AND units (both lists of a round-1 pair decoded into bitvectors): words per unit
+constexpr uint32_t kAndWords = 512;
 // Per-term batch decode-once kind (Workspace::tdec): not decoded, decoded into
 // the docID arena, or decoded into a docID bitvector with rank (dense lists).
 enum : uint8_t { kDecNone = 0, kDecArena = 1, kDecBitmap = 2 };
@@ -101,8 +103,8 @@ enum : int {
   kScalRoundTot = 18, // u64: survivors of the current round (compaction scan total)
   kScalDiag = 19,     // 4 x u64 (counting mode): merge units, merged elements, gallop units, galloped elements
   kScalUnitCtr2 = 23, // u64 ticket counter of the round-1 gallop/single-term kernel
-  kScalDiag2 = 24,    // 2 x u64 (counting mode): bitvector units, their R elements
-  kScalCount = 26
+  kScalDiag2 = 24,    // 4 x u64 (counting mode): bitvector units, their R elements, word-AND units, their words
+  kScalCount = 28
 };
 
 #ifndef GRIFFIN_BUMP_CHUNK

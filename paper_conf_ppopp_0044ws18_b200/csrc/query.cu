@@ -255,9 +255,21 @@ __global__ void plan_round_kernel(DevIndex ix, RoundArgs a, uint32_t *qunits) {
       // S decoded into a bitvector this batch: every R element is looked up in
       // O(1) (no merge or gallop through S), one unit per R chunk of B
       const bool bitmap = a.forced_mode == 0 && kd == kDecBitmap;
-      mode = bitmap ? kModeBitmap : (gallop ? kModeGallop : kModeMerge);
+      // ... and so is R (round 1): AND the two bitvectors word by word over
+      // R's docID range, kAndWords words per unit (no R decode, no lookups)
+#ifdef GRIFFIN_NO_BITAND   // A/B builds
+      const bool band = false;
+#else
+      const bool band = bitmap && a.round == 1 && a.tdec[a.plan_terms[q * kMaxTerms]] == kDecBitmap;
+#endif
+      mode = band ? kModeBitAnd : (bitmap ? kModeBitmap : (gallop ? kModeGallop : kModeMerge));
       const uint32_t U = bm_unit_blocks(ix.B, a.D, a.nextgeq != 0);
-      units = bitmap ? (nbR + U - 1) / U : (gallop ? nbR : (nbR + tS.nblocks + a.D - 1) / a.D);
+      if (band) {
+        const uint32_t w0 = __ldg(ix.first + t0.block0) >> 5;
+        units = (a.bm_words - w0 + kAndWords - 1) / kAndWords;
+      } else {
+        units = bitmap ? (nbR + U - 1) / U : (gallop ? nbR : (nbR + tS.nblocks + a.D - 1) / a.D);
+      }
     }
   }
   a.qmode[q] = mode;
@@ -733,7 +745,7 @@ __device__ __forceinline__ uint4 uperm_entry(const RoundArgs &a, uint64_t u, uin
 // units, and probe-pass units whose first remaining list is a bitvector.
 __device__ __forceinline__ bool bm_bucketed(const RoundArgs &a, uint32_t q) {
   const uint32_t md = a.qmode[q];
-  return a.sbkt_nbb && (md == kModeBitmap ||
+  return a.sbkt_nbb && (md == kModeBitmap || md == kModeBitAnd ||
                         (md == kModeProbe && a.tdec &&
                          a.tdec[a.plan_terms[(size_t)q * kMaxTerms + a.round]] == kDecBitmap));
 }
@@ -747,6 +759,8 @@ __device__ __forceinline__ uint64_t bitmap_unit_bucket(const DevIndex &ix, const
   uint32_t x0;
   if (a.qmode[q] == kModeProbe) {
     x0 = a.rprev[a.roff_prev[q] + (size_t)lu * a.pchunk].x;
+  } else if (a.qmode[q] == kModeBitAnd) {
+    x0 = (((__ldg(ix.first + ix.terms[pt[0]].block0) >> 5) + lu * kAndWords) << 5);
   } else {
     const uint32_t b0 = lu * bm_unit_blocks(ix.B, a.D, a.nextgeq != 0);
     x0 = RC ? __ldg(ix.first + ix.terms[pt[0]].block0 + b0)
@@ -1352,6 +1366,100 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
 }
 
 
+// Word-AND unit (round 1, both lists decoded into bitvectors this batch):
+// words [w0, w1) of R's docID range.  Pass 1 counts the unit's survivors
+// (popc of the ANDed words) for its output allocation; pass 2 walks 32 words
+// per step (one per lane): each set bit of R.bits & S.bits is a survivor, its
+// positions in R and S are the words' ranks + popc of the bits below it.  The
+// survivors are buffered in shared memory (docID, R position, S position; at
+// most C = cap of them, in docID order) and scored with every lane busy — w_R
+// + w_S, SURVEY O6 — when the buffer fills; a 32-word step with more than C
+// survivors is scored straight from the lanes.
+__device__ __forceinline__ void bitand_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u,
+                                            uint32_t lu, uint32_t t0, uint32_t tSid,
+                                            const TermInfo &tR, const TermInfo &tS,
+                                            uint32_t *sdoc, uint32_t *srp, uint32_t *ssp,
+                                            uint32_t cap, Acc &acc) {
+  const uint32_t lane = lane_id();
+  const uint2 *bR = a.bm + (size_t)a.bm_slot[t0] * a.bm_words;
+  const uint2 *bS = a.bm + (size_t)a.bm_slot[tSid] * a.bm_words;
+  const uint32_t w0 = (__ldg(ix.first + tR.block0) >> 5) + lu * kAndWords;
+  const uint32_t w1 = min(w0 + kAndWords, a.bm_words);
+  uint32_t c = 0;
+  for (uint32_t w = w0 + lane; w < w1; w += 32u) c += __popc(__ldg(&bR[w].x) & __ldg(&bS[w].x));
+  uint32_t cnt = __reduce_add_sync(0xffffffffu, c);
+  unsigned long long off = 0;
+  if (lane == 0 && cnt) off = bump_alloc(a, acc, cnt);
+  off = __shfl_sync(0xffffffffu, off, 0);
+  if (off + cnt > a.bump_cap) {
+    if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
+    cnt = 0;
+  }
+  auto score = [&](uint32_t doc, uint32_t rpos, uint32_t spos) -> uint2 {
+    const float nrm = __ldg(ix.norm + doc);
+    const float wS = bm25_w(tS.idf, tf_lookup(ix, tS, spos), nrm, ix.k1p1);
+    float sc = bm25_w(tR.idf, tf_lookup(ix, tR, rpos), nrm, ix.k1p1);   // first term: s = w
+    return make_uint2(doc, __float_as_uint(__fadd_rn(sc, wS)));
+  };
+  if (cnt) {
+    uint64_t run = off;    // next output slot
+    uint32_t fb = 0;       // buffered survivors
+    auto flush = [&]() {
+      __syncwarp();
+      for (uint32_t j = lane; j < fb; j += 32u) a.bump[run + j] = score(sdoc[j], srp[j], ssp[j]);
+      run += fb;
+      fb = 0;
+      __syncwarp();
+    };
+    for (uint32_t wb = w0; wb < w1; wb += 32u) {
+      const uint32_t w = wb + lane;
+      const uint2 ra = w < w1 ? __ldg(bR + w) : make_uint2(0, 0);
+      const uint2 sa = w < w1 ? __ldg(bS + w) : make_uint2(0, 0);
+      uint32_t m = ra.x & sa.x;
+      const uint32_t k = __popc(m);
+      const uint32_t incl = warp_incl_scan(k);
+      const uint32_t T = __shfl_sync(0xffffffffu, incl, 31);
+      if (T == 0) continue;
+      if (fb + T > cap) flush();
+      if (T <= cap) {
+        uint32_t o = fb + incl - k;
+        while (m) {
+          const uint32_t bit = __ffs(m) - 1u;
+          m &= m - 1u;
+          const uint32_t below = (1u << bit) - 1u;
+          sdoc[o] = (w << 5) | bit;
+          srp[o] = ~ra.y + __popc(ra.x & below);
+          ssp[o] = ~sa.y + __popc(sa.x & below);
+          ++o;
+        }
+        fb += T;
+      } else {   // more survivors in 32 words than the buffer holds: score from the lanes
+        uint64_t o = run + incl - k;
+        while (m) {
+          const uint32_t bit = __ffs(m) - 1u;
+          m &= m - 1u;
+          const uint32_t below = (1u << bit) - 1u;
+          a.bump[o++] = score((w << 5) | bit, ~ra.y + __popc(ra.x & below),
+                              ~sa.y + __popc(sa.x & below));
+        }
+        run += T;
+      }
+    }
+    flush();
+  }
+  __syncwarp();
+  if (lane == 0) {
+    a.unit_off[u] = off;
+    a.unit_cnt[u] = cnt;
+    acc.ctr[kCSurv] += cnt;
+    acc.ctr[kCAlg] += (unsigned long long)cnt * kSurvBytesR1 + 16ull * (w1 > w0 ? w1 - w0 : 0u);
+    if (a.count) {
+      atomicAdd(a.scal + kScalDiag2 + 2, 1ull);
+      atomicAdd(a.scal + kScalDiag2 + 3, (unsigned long long)(w1 > w0 ? w1 - w0 : 0u));
+    }
+  }
+}
+
 // Round-1 unit kinds run as two kernels, back to back (ROLE): 1 = the merge
 // units (the processing order puts them first: tickets [0, #merge)), 2 = the
 // gallop and single-term units (tickets [#merge, total)) with a smaller shared
@@ -1680,6 +1788,12 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
                           sb0 * B + sa, smem_u32(sm.tile) & 0xFFFFu,
                           smem_u32(tileS + sa) & 0xFFFFu, acc);
       __syncwarp();
+    } else if (ROLE != 1 && mode == kModeBitAnd) {
+      // survivor buffer: docIDs in the tile, R / S positions in the staging area
+      uint32_t tw, sw;
+      bm_layout(B, D, a.nextgeq != 0, ROLE == 2, &tw, &sw);
+      const uint32_t cap = min(tw, sw / 2u);
+      bitand_unit(ix, a, (uint32_t)u, lu, t0, tSid, tR, tS, sm.tile, sm.stg, sm.stg + cap, cap, acc);
     } else if (ROLE != 1 && mode == kModeBitmap) {
       // ---- S decoded into a bitvector this batch: R blocks [b0, b0+nb) (or
       // intermediate chunks) looked up in O(1), hits compacted, then scored ----

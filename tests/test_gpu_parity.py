@@ -514,7 +514,7 @@ def test_bitmap_decode_once_bit_exact(tiny, inv):
 
 @pytest.mark.parametrize("B", [64, 96, 128, 256, 512])
 def test_bitmap_dense_runs_and_edges(B):
-    """Bitvector construction edge cases: lists of consecutive docIDs (whole
+    """Bitvector construction and word-AND edge cases: lists of consecutive docIDs (whole
     words owned by one lane: plain stores), near-complete lists, docID 0 and
     N-1, word boundaries shared by lanes and blocks, multi-term queries (probe
     pass / later SvS rounds against bitvectors), every block size."""
@@ -537,6 +537,7 @@ def test_bitmap_dense_runs_and_edges(B):
     gx = g.GriffinIndex(c, block_size=B)
     gx.griffin_set_reuse(1)
     gx.griffin_set_bitmap(1 << 24)
+    gx.griffin_set_profiling(3)
     V = len(lists)
     offs, terms = [0], []
     for _ in range(3):
@@ -553,6 +554,9 @@ def test_bitmap_dense_runs_and_edges(B):
         od, os_, oc = ox.query_batch(ql, k)
         gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
         assert_topk_equal(gd, gs, gc, od, os_, oc)
+    prof = gx.griffin_get_profile()
+    # every decoded list is a bitvector here: pairs of two of them are ANDed
+    assert prof["bitand_units"] > 0
     gx.close()
 
 
