@@ -2138,50 +2138,56 @@ __global__ void __launch_bounds__(kIntersectThreads, 4) probe_kernel(DevIndex ix
 // Global exclusive scan of the per-unit survivor counts (n = total units, read
 // on the device; CTAs past n exit).  Units of one query are contiguous, so a
 // query's output offset of unit u is udst[u] - udst[first unit of q].
+// (grid-stride over the `ntiles` tiles of the reserved unit capacity: the
+// grid is sized for the device, not for the capacity, and tiles past the
+// round's unit count only write a zero sum)
 __global__ void __launch_bounds__(kScanThreads) unit_scan_sums(const uint32_t *cnt,
                                                                const uint64_t *n_dev,
-                                                               uint64_t *tsum) {
+                                                               uint64_t *tsum, uint32_t ntiles) {
   __shared__ uint64_t ws[32];
   __shared__ uint64_t tot;
   const uint64_t n = *n_dev;
-  const uint64_t t0 = (uint64_t)blockIdx.x * kScanTile;
-  if (t0 >= n) {
-    if (threadIdx.x == 0) tsum[blockIdx.x] = 0;
-    return;
-  }
-  uint64_t s = 0;
+  for (uint32_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const uint64_t t0 = (uint64_t)tile * kScanTile;
+    if (t0 >= n) {
+      if (threadIdx.x == 0) tsum[tile] = 0;
+      continue;
+    }
+    uint64_t s = 0;
 #pragma unroll
-  for (int i = 0; i < kScanItems; ++i) {
-    const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
-    if (idx < n) s += cnt[idx];
+    for (int i = 0; i < kScanItems; ++i) {
+      const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
+      if (idx < n) s += cnt[idx];
+    }
+    block_excl_scan<uint64_t>(s, ws, &tot);
+    if (threadIdx.x == 0) tsum[tile] = tot;
   }
-  block_excl_scan<uint64_t>(s, ws, &tot);
-  if (threadIdx.x == 0) tsum[blockIdx.x] = tot;
 }
-
 __global__ void __launch_bounds__(kScanThreads) unit_scan_apply(const uint32_t *cnt,
                                                                 const uint64_t *n_dev,
                                                                 const uint64_t *toff,
-                                                                uint64_t *out) {
+                                                                uint64_t *out, uint32_t ntiles) {
   __shared__ uint64_t ws[32];
   __shared__ uint64_t tot;
   const uint64_t n = *n_dev;
-  const uint64_t t0 = (uint64_t)blockIdx.x * kScanTile;
-  if (t0 >= n) return;
-  uint64_t loc[kScanItems];
-  uint64_t s = 0;
+  for (uint32_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const uint64_t t0 = (uint64_t)tile * kScanTile;
+    if (t0 >= n) break;   // tiles are visited in increasing order per block
+    uint64_t loc[kScanItems];
+    uint64_t s = 0;
 #pragma unroll
-  for (int i = 0; i < kScanItems; ++i) {
-    const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
-    loc[i] = idx < n ? cnt[idx] : 0;
-    s += loc[i];
-  }
-  uint64_t run = toff[blockIdx.x] + block_excl_scan<uint64_t>(s, ws, &tot);
+    for (int i = 0; i < kScanItems; ++i) {
+      const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
+      loc[i] = idx < n ? cnt[idx] : 0;
+      s += loc[i];
+    }
+    uint64_t run = toff[tile] + block_excl_scan<uint64_t>(s, ws, &tot);
 #pragma unroll
-  for (int i = 0; i < kScanItems; ++i) {
-    const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
-    if (idx < n) out[idx] = run;
-    run += loc[i];
+    for (int i = 0; i < kScanItems; ++i) {
+      const uint64_t idx = t0 + (uint64_t)threadIdx.x * kScanItems + i;
+      if (idx < n) out[idx] = run;
+      run += loc[i];
+    }
   }
 }
 
@@ -3278,11 +3284,12 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
       const uint64_t *n_dev = w.unit_base.as<uint64_t>() + nq;
       const unsigned tiles = (unsigned)(w.unit_cap / kScanTile + 1);
       uint64_t *tsum = w.unit_dst.as<uint64_t>() + (w.unit_cap + 2);
-      unit_scan_sums<<<tiles, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum);
+      const unsigned sgrid = std::min<unsigned>(tiles, num_sms(ix->device) * 2);
+      unit_scan_sums<<<sgrid, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum, tiles);
       scan_single_kernel<uint64_t><<<1, kScanThreads, 0, st>>>(tsum, tsum, tiles,
                                                                reinterpret_cast<uint64_t *>(scal + kScalRoundTot));
-      unit_scan_apply<<<tiles, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum,
-                                                      w.unit_dst.as<uint64_t>());
+      unit_scan_apply<<<sgrid, kScanThreads, 0, st>>>(ra.unit_cnt, n_dev, tsum,
+                                                      w.unit_dst.as<uint64_t>(), tiles);
       compact_copy_kernel<<<num_sms(ix->device) * 8, 256, 0, st>>>(ra, w.unit_dst.as<uint64_t>());
       if (r <= 2) {
         compact_queries_kernel<<<qblocks, 256, 0, st>>>(ra, w.unit_dst.as<uint64_t>());
