@@ -2470,17 +2470,32 @@ __global__ void __launch_bounds__(256) topk_filter_kernel(
     const uint64_t tau = ts.ftau[q];
     const uint32_t slot = ts.fslot[q];
     uint64_t *out = ts.flt + (size_t)slot * kFiltCap;
-    for (uint32_t i0 = threadIdx.x - lane; i0 < len; i0 += blockDim.x) {
-      const uint32_t i = i0 + lane;
-      const uint64_t x = i < len ? make_key(R[i], ix.doc_base) : 0ull;
-      const bool keep = i < len && x >= tau;
-      const uint32_t bal = __ballot_sync(0xffffffffu, keep);
-      if (bal) {
+    // four entries per lane in flight; one output reservation per 128 entries
+    for (uint32_t i0 = (threadIdx.x - lane) * 4u; i0 < len; i0 += blockDim.x * 4u) {
+      uint64_t x[4];
+      bool keep[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t i = i0 + 32u * j + lane;
+        x[j] = i < len ? make_key(R[i], ix.doc_base) : 0ull;
+        keep[j] = i < len && x[j] >= tau;
+      }
+      uint32_t bal[4], tot = 0;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        bal[j] = __ballot_sync(0xffffffffu, keep[j]);
+        tot += __popc(bal[j]);
+      }
+      if (tot) {
         uint32_t base = 0;
-        if (lane == 0) base = atomicAdd(ts.fcnt + slot, (uint32_t)__popc(bal));
+        if (lane == 0) base = atomicAdd(ts.fcnt + slot, tot);
         base = __shfl_sync(0xffffffffu, base, 0);
-        const uint32_t pos = base + __popc(bal & lanemask_lt());
-        if (keep && pos < kFiltCap) out[pos] = x;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const uint32_t pos = base + __popc(bal[j] & lanemask_lt());
+          if (keep[j] && pos < kFiltCap) out[pos] = x[j];
+          base += __popc(bal[j]);
+        }
       }
     }
   }
