@@ -289,6 +289,8 @@ def run_gpu(args):
     st = ix.griffin_index_stats()
     ix.griffin_set_reuse({"auto": 2, "on": 1, "off": 0}[args.reuse])
     ix.griffin_set_bitmap(args.bitmap)
+    if args.probe_chunk:
+        ix.griffin_set_probe_chunk(args.probe_chunk)
     # intermediate capacity per workspace buffer: packed by actual survivors, so a
     # budget well under the sum of per-query bounds holds a batch (C5: ~1e9 bound)
     budget = args.entry_budget if args.entry_budget is not None else \
@@ -628,6 +630,8 @@ def main():
                     help="batch decode-once of hot lists into an HBM arena")
     ap.add_argument("--bitmap", type=int, default=32,
                     help="dense lists (density >= 1/INV) decoded once per batch into a bitvector; 0 = off")
+    ap.add_argument("--probe-chunk", type=int, default=0,
+                    help="probe-pass survivors per unit (0 = library default)")
     ap.add_argument("--shard-mode", default="docid", choices=["docid", "replicate"],
                     help="N>1: docID-range shards + exchange, or a replicated index per rank")
     ap.add_argument("--exchange", default="allgather", choices=["allgather", "sliced"],

@@ -135,3 +135,21 @@ def test_multi_gpu_options_rejected_on_host():
     with pytest.raises(g.GriffinError) as e:   # a multi handle builds its shards itself
         g.GriffinIndex(c, num_gpus=2, num_shards=2)
     assert e.value.status == 1
+
+
+def test_profile_struct_layout_matches_header(tmp_path):
+    """The binding's ctypes mirror of griffin_profile has the C struct's size
+    and field offsets (compiled from include/griffin.h with the host gcc)."""
+    fields = [f for f, _ in g.Profile._fields_]
+    src = tmp_path / "layout.c"
+    src.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "griffin.h"\n'
+                   'int main(void) {\n  printf("%zu\\n", sizeof(griffin_profile));\n' +
+                   "".join(f'  printf("%zu\\n", offsetof(griffin_profile, {f}));\n' for f in fields) +
+                   "  return 0;\n}\n")
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)],
+                   check=True)
+    out = [int(x) for x in subprocess.run([str(exe)], capture_output=True, text=True,
+                                          check=True).stdout.split()]
+    assert out[0] == ctypes.sizeof(g.Profile)
+    assert out[1:] == [getattr(g.Profile, f).offset for f in fields]
