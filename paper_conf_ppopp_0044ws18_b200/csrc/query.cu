@@ -822,7 +822,10 @@ __global__ void partition_kernel(DevIndex ix, RoundArgs a) {
 // out together and their S tiles come from L2 (a C2 batch merges 92M S
 // postings of 39M distinct ones, C5 2.66 B of 455M).  Order inside a bucket is
 // arbitrary; results do not depend on processing order.
-constexpr uint32_t kSorderMinQueries = 4096;
+#ifndef GRIFFIN_SORDER_MIN_QUERIES
+#define GRIFFIN_SORDER_MIN_QUERIES 4096
+#endif
+constexpr uint32_t kSorderMinQueries = GRIFFIN_SORDER_MIN_QUERIES;
 template <bool RC>
 __global__ void sorder_scatter_kernel(DevIndex ix, RoundArgs a) {
   const uint64_t total = a.unit_base[a.nq];
