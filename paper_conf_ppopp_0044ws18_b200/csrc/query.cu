@@ -1209,10 +1209,10 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
     const uint2 v = Rq[s0 + e];
     tileR[e] = v.x;
     sc[e] = v.y;
-    nrm[e] = __float_as_uint(__ldg(ix.norm + v.x));
+    nrm[e] = 0xFFFFFFFFu;   // gathered when the survivor first passes a list (most are dropped)
   }
   __syncwarp();
-  if (lane == 0) acc.ctr[kCAlg] += n * 12u;
+  if (lane == 0) acc.ctr[kCAlg] += n * 8u;
   for (uint32_t r = 2; r < m && n > 0; ++r) {
     const uint32_t sid = pt[r];
     const TermInfo tS = ix.terms[sid];
@@ -1331,9 +1331,15 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
       const uint32_t e = c0 + lane;
       const bool in = e < n;
       const uint32_t x = in ? tileR[e] : 0u, mt = in ? match[e] : kNone;
-      const uint32_t nm = in ? nrm[e] : 0u;
+      uint32_t nm = in ? nrm[e] : 0u;
       float s = in ? __uint_as_float(sc[e]) : 0.f;
       const bool keep = in && mt != kNone;
+      const bool gather = keep && nm == 0xFFFFFFFFu;
+      if (gather) nm = __float_as_uint(__ldg(ix.norm + x));   // (norms are finite)
+      if (a.count) {
+        const uint32_t ng = __popc(__ballot_sync(0xffffffffu, gather));
+        if (lane == 0) acc.ctr[kCAlg] += ng * 4u;   // the doc's norm, once
+      }
       if (keep) s = __fadd_rn(s, bm25_w(tS.idf, tf_lookup(ix, tS, mt), __uint_as_float(nm), ix.k1p1));
       const uint32_t bal = __ballot_sync(0xffffffffu, keep);
       __syncwarp();
