@@ -474,7 +474,7 @@ static uint64_t ws_identity(const Workspace &w) {
                           &w.qmode, &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.uperm,
                           &w.rbuf0, &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys,
                           &w.counts, &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand,
-                          &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.run_term, &w.arena, &w.bmap})
+                          &w.tdec, &w.runs, &w.run_base, &w.vtmp, &w.run_term, &w.arena, &w.bmap, &w.qtau})
     h = (h ^ (uint64_t)(uintptr_t)b->p) * 1099511628211ull;
   // capacities are baked into a captured graph's kernel arguments too
   for (const uint64_t v : {(uint64_t)w.nq_cap, (uint64_t)w.unit_cap, (uint64_t)w.entry_cap,
@@ -641,7 +641,7 @@ static void free_workspace(Workspace &w) {
                     &w.unit_base, &w.unit_off, &w.unit_cnt, &w.unit_dst, &w.urec, &w.uperm, &w.rbuf0,
                     &w.rbuf1, &w.bump, &w.cand, &w.tkstate, &w.scal, &w.keys, &w.counts,
                     &w.docids, &w.scores, &w.qoffs, &w.qterms, &w.demand, &w.tdec, &w.runs,
-                    &w.run_base, &w.vtmp, &w.run_term, &w.arena, &w.bmap, &w.sbkt_cnt, &w.sbkt_pos,
+                    &w.run_base, &w.vtmp, &w.run_term, &w.arena, &w.bmap, &w.qtau, &w.sbkt_cnt, &w.sbkt_pos,
                     &w.sbkt_tmp, &w.flt, &w.fstate})
     b->release();
   if (w.h_pinned) cudaFreeHost(w.h_pinned);

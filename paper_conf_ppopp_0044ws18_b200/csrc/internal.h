@@ -71,6 +71,7 @@ struct Workspace {
   DevBuf demand, tdec, runs, run_base, vtmp, run_term; // per term / run (batch reuse)
   DevBuf arena;                                        // decoded lists, nblocks * B u32
   DevBuf bmap;                                         // decoded dense lists: bitvector + rank
+  DevBuf qtau;                                         // per query: top-k key threshold (bitand_tau_kernel)
   DevBuf sbkt_cnt, sbkt_pos, sbkt_tmp;                 // S-locality unit order buckets
   size_t nq_cap = 0, unit_cap = 0, entry_cap = 0;
   // pinned host staging; a grown buffer's predecessors stay allocated until the
@@ -155,6 +156,7 @@ struct RoundArgs {
   const uint2 *bm;        // bitvector area: slot s at bm + s * bm_words
   const uint32_t *bm_slot;   // per term: its bitvector slot (kNone: not eligible)
   uint32_t bm_words;      // words per bitvector = ceil(n_docs / 32)
+  const uint64_t *qtau;   // per query: round-1 key threshold of 2-term word-AND queries (or null)
 };
 
 }  // namespace griffin

@@ -1384,16 +1384,20 @@ __device__ void probe_unit(const DevIndex &ix, const RoundArgs &a, WarpSmem &sm,
 // most C = cap of them, in docID order) and scored with every lane busy — w_R
 // + w_S, SURVEY O6 — when the buffer fills; a 32-word step with more than C
 // survivors is scored straight from the lanes.
+__device__ __forceinline__ uint64_t make_key(uint2 e, uint32_t doc_base);
 __device__ __forceinline__ void bitand_unit(const DevIndex &ix, const RoundArgs &a, uint32_t u,
-                                            uint32_t lu, uint32_t t0, uint32_t tSid,
+                                            uint32_t q, uint32_t lu, uint32_t t0, uint32_t tSid,
                                             const TermInfo &tR, const TermInfo &tS,
                                             uint32_t *sdoc, uint32_t *srp, uint32_t *ssp,
                                             uint32_t cap, Acc &acc) {
-  const uint32_t lane = lane_id();
+  const uint32_t lane = lane_id(), lt = lanemask_lt();
   const uint2 *bR = a.bm + (size_t)a.bm_slot[t0] * a.bm_words;
   const uint2 *bS = a.bm + (size_t)a.bm_slot[tSid] * a.bm_words;
   const uint32_t w0 = (__ldg(ix.first + tR.block0) >> 5) + lu * kAndWords;
   const uint32_t w1 = min(w0 + kAndWords, a.bm_words);
+  // a 2-term query's keys below its subset threshold cannot reach its top-k
+  // (bitand_tau_kernel): they are scored but not written
+  const uint64_t tau = a.qtau ? a.qtau[q] : 0ull;
   uint32_t c = 0;
   for (uint32_t w = w0 + lane; w < w1; w += 32u) c += __popc(__ldg(&bR[w].x) & __ldg(&bS[w].x));
   uint32_t cnt = __reduce_add_sync(0xffffffffu, c);
@@ -1404,19 +1408,29 @@ __device__ __forceinline__ void bitand_unit(const DevIndex &ix, const RoundArgs 
     if (lane == 0) atomicOr(reinterpret_cast<int *>(a.scal + kScalStatus), kStatusOverflow);
     cnt = 0;
   }
-  auto score = [&](uint32_t doc, uint32_t rpos, uint32_t spos) -> uint2 {
-    const float nrm = __ldg(ix.norm + doc);
-    const float wS = bm25_w(tS.idf, tf_lookup(ix, tS, spos), nrm, ix.k1p1);
-    float sc = bm25_w(tR.idf, tf_lookup(ix, tR, rpos), nrm, ix.k1p1);   // first term: s = w
-    return make_uint2(doc, __float_as_uint(__fadd_rn(sc, wS)));
-  };
+  uint32_t kept = 0;   // survivors written (all of them when tau = 0)
+  uint32_t gsmall = 1;   // largest power of two <= min(8, cap / 32) (cap >= 32 in every layout)
+  while (gsmall < 8u && 64u * gsmall <= cap) gsmall <<= 1;
   if (cnt) {
-    uint64_t run = off;    // next output slot
     uint32_t fb = 0;       // buffered survivors
     auto flush = [&]() {
       __syncwarp();
-      for (uint32_t j = lane; j < fb; j += 32u) a.bump[run + j] = score(sdoc[j], srp[j], ssp[j]);
-      run += fb;
+      for (uint32_t j0 = 0; j0 < fb; j0 += 32u) {
+        const uint32_t j = j0 + lane;
+        uint2 e = make_uint2(0, 0);
+        bool keep = false;
+        if (j < fb) {
+          const uint32_t doc = sdoc[j];
+          const float nrm = __ldg(ix.norm + doc);
+          const float wS = bm25_w(tS.idf, tf_lookup(ix, tS, ssp[j]), nrm, ix.k1p1);
+          const float wR = bm25_w(tR.idf, tf_lookup(ix, tR, srp[j]), nrm, ix.k1p1);   // first term: s = w
+          e = make_uint2(doc, __float_as_uint(__fadd_rn(wR, wS)));
+          keep = make_key(e, ix.doc_base) >= tau;
+        }
+        const uint32_t bal = __ballot_sync(0xffffffffu, keep);
+        if (keep) a.bump[off + kept + __popc(bal & lt)] = e;
+        kept += __popc(bal);
+      }
       fb = 0;
       __syncwarp();
     };
@@ -1424,50 +1438,52 @@ __device__ __forceinline__ void bitand_unit(const DevIndex &ix, const RoundArgs 
       const uint32_t w = wb + lane;
       const uint2 ra = w < w1 ? __ldg(bR + w) : make_uint2(0, 0);
       const uint2 sa = w < w1 ? __ldg(bS + w) : make_uint2(0, 0);
-      uint32_t m = ra.x & sa.x;
-      const uint32_t k = __popc(m);
-      const uint32_t incl = warp_incl_scan(k);
+      const uint32_t mm = ra.x & sa.x;
+      const uint32_t k = __popc(mm);
+      const uint32_t incl = warp_incl_scan(k), excl = incl - k;
       const uint32_t T = __shfl_sync(0xffffffffu, incl, 31);
       if (T == 0) continue;
-      if (fb + T > cap) flush();
-      if (T <= cap) {
-        uint32_t o = fb + incl - k;
-        while (m) {
-          const uint32_t bit = __ffs(m) - 1u;
-          m &= m - 1u;
-          const uint32_t below = (1u << bit) - 1u;
-          sdoc[o] = (w << 5) | bit;
-          srp[o] = ~ra.y + __popc(ra.x & below);
-          ssp[o] = ~sa.y + __popc(sa.x & below);
-          ++o;
+      // buffered in groups of lanes that fit the buffer: the whole warp, or
+      // gsmall lanes (<= 32 docs each, <= cap in all) when one step holds
+      // more survivors than `cap`
+      const uint32_t gl = T <= cap ? 32u : gsmall;
+      for (uint32_t g = 0; g < 32u; g += gl) {
+        const uint32_t gb = __shfl_sync(0xffffffffu, excl, g);
+        const uint32_t gT = __shfl_sync(0xffffffffu, incl, g + gl - 1u) - gb;
+        if (gT == 0) continue;
+        if (fb + gT > cap) flush();
+        if (lane >= g && lane < g + gl) {
+          uint32_t m = mm, o = fb + excl - gb;
+          while (m) {
+            const uint32_t bit = __ffs(m) - 1u;
+            m &= m - 1u;
+            const uint32_t below = (1u << bit) - 1u;
+            sdoc[o] = (w << 5) | bit;
+            srp[o] = ~ra.y + __popc(ra.x & below);
+            ssp[o] = ~sa.y + __popc(sa.x & below);
+            ++o;
+          }
         }
-        fb += T;
-      } else {   // more survivors in 32 words than the buffer holds: score from the lanes
-        uint64_t o = run + incl - k;
-        while (m) {
-          const uint32_t bit = __ffs(m) - 1u;
-          m &= m - 1u;
-          const uint32_t below = (1u << bit) - 1u;
-          a.bump[o++] = score((w << 5) | bit, ~ra.y + __popc(ra.x & below),
-                              ~sa.y + __popc(sa.x & below));
-        }
-        run += T;
+        fb += gT;
       }
     }
     flush();
   }
   __syncwarp();
   if (lane == 0) {
+    const uint32_t nw = w1 > w0 ? w1 - w0 : 0u;
     a.unit_off[u] = off;
-    a.unit_cnt[u] = cnt;
-    acc.ctr[kCSurv] += cnt;
-    acc.ctr[kCAlg] += (unsigned long long)cnt * kSurvBytesR1 + 16ull * (w1 > w0 ? w1 - w0 : 0u);
+    a.unit_cnt[u] = kept;
+    acc.ctr[kCSurv] += kept;
+    // 16 B per word pair; per scored survivor two tf sectors + the norm, per kept one the entry
+    acc.ctr[kCAlg] += (unsigned long long)cnt * (2u * kTfSector + 4u) + 8ull * kept + 16ull * nw;
     if (a.count) {
       atomicAdd(a.scal + kScalDiag2 + 2, 1ull);
-      atomicAdd(a.scal + kScalDiag2 + 3, (unsigned long long)(w1 > w0 ? w1 - w0 : 0u));
+      atomicAdd(a.scal + kScalDiag2 + 3, (unsigned long long)nw);
     }
   }
 }
+
 
 // Round-1 unit kinds run as two kernels, back to back (ROLE): 1 = the merge
 // units (the processing order puts them first: tickets [0, #merge)), 2 = the
@@ -1802,7 +1818,7 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
       uint32_t tw, sw;
       bm_layout(B, D, a.nextgeq != 0, ROLE == 2, &tw, &sw);
       const uint32_t cap = min(tw, sw / 2u);
-      bitand_unit(ix, a, (uint32_t)u, lu, t0, tSid, tR, tS, sm.tile, sm.stg, sm.stg + cap, cap, acc);
+      bitand_unit(ix, a, (uint32_t)u, q, lu, t0, tSid, tR, tS, sm.tile, sm.stg, sm.stg + cap, cap, acc);
     } else if (ROLE != 1 && mode == kModeBitmap) {
       // ---- S decoded into a bitvector this batch: R blocks [b0, b0+nb) (or
       // intermediate chunks) looked up in O(1), hits compacted, then scored ----
@@ -2373,6 +2389,76 @@ __device__ uint64_t cta_radix_select(KeyF key, uint32_t n, uint32_t kk, SelectSm
     }
   }
   return ss.prefix;
+}
+
+// Top-k threshold of a 2-term word-AND query (round 1 is its last round): the
+// k-th largest key among a SUBSET of its survivors — strided 32-word steps of
+// the AND over R's docID range, up to kTauKeys keys — is at most its k-th
+// largest key overall (the subset's k largest are survivors), so every key of
+// its top-k is >= it and bitand_unit may drop the survivors below it (exact;
+// keys are unique).  tau = 0 (no dropping) when the subset holds
+// fewer than k keys, for other queries, and when k > kTauKeys / 2.
+constexpr uint32_t kTauKeys = 8192;
+__host__ __device__ inline size_t tau_smem_bytes() { return (size_t)kTauKeys * 8; }
+__global__ void __launch_bounds__(1024) bitand_tau_kernel(DevIndex ix, RoundArgs a, uint32_t k,
+                                                         uint64_t *tau) {
+  extern __shared__ uint64_t tkeys[];
+  __shared__ SelectSmem ss;
+  __shared__ uint32_t nk;
+  const uint32_t lane = lane_id(), warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+  for (uint32_t q = blockIdx.x; q < a.nq; q += gridDim.x) {
+    const uint32_t *pt = a.plan_terms + (size_t)q * kMaxTerms;
+    if (a.qmode[q] != kModeBitAnd || a.plan_m[q] != 2 || k == 0 || k > kTauKeys / 2) {
+      if (threadIdx.x == 0) tau[q] = 0;
+      continue;
+    }
+    const TermInfo tR = ix.terms[pt[0]], tS = ix.terms[pt[1]];
+    const uint2 *bR = a.bm + (size_t)a.bm_slot[pt[0]] * a.bm_words;
+    const uint2 *bS = a.bm + (size_t)a.bm_slot[pt[1]] * a.bm_words;
+    const uint32_t w0 = __ldg(ix.first + tR.block0) >> 5;
+    const uint32_t nch = (a.bm_words - w0 + 31u) / 32u;
+    // stride over 32-word steps so the sample holds about kTauKeys keys
+    // (an estimate: a subset of any size is exact, a larger one is tighter)
+    const double est = (double)tR.df_local * (double)tS.df_local / (double)max(1u, ix.n_docs);
+    const uint32_t stride = max(1u, (uint32_t)(est / kTauKeys));
+    if (threadIdx.x == 0) nk = 0;
+    __syncthreads();
+    // four 32-word steps per warp in flight
+    for (uint32_t c0 = warp * stride * 4u; c0 < nch; c0 += nwarps * stride * 4u) {
+      if (*(volatile uint32_t *)&nk >= kTauKeys) break;
+      uint2 ra[4], sa[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t c = c0 + (uint32_t)j * stride;
+        const uint32_t w = w0 + c * 32u + lane;
+        const bool in = c < nch && w < a.bm_words;
+        ra[j] = in ? __ldg(bR + w) : make_uint2(0, 0);
+        sa[j] = in ? __ldg(bS + w) : make_uint2(0, 0);
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t w = w0 + (c0 + (uint32_t)j * stride) * 32u + lane;
+        uint32_t m = ra[j].x & sa[j].x;
+        while (m) {
+          const uint32_t bit = __ffs(m) - 1u;
+          m &= m - 1u;
+          const uint32_t below = (1u << bit) - 1u, doc = (w << 5) | bit;
+          const float nrm = __ldg(ix.norm + doc);
+          const float wS = bm25_w(tS.idf, tf_lookup(ix, tS, ~sa[j].y + __popc(sa[j].x & below)), nrm, ix.k1p1);
+          const float wR = bm25_w(tR.idf, tf_lookup(ix, tR, ~ra[j].y + __popc(ra[j].x & below)), nrm, ix.k1p1);
+          const uint32_t slot = atomicAdd(&nk, 1u);
+          if (slot < kTauKeys)
+            tkeys[slot] = make_key(make_uint2(doc, __float_as_uint(__fadd_rn(wR, wS))), ix.doc_base);
+        }
+      }
+    }
+    __syncthreads();
+    const uint32_t n = min(nk, kTauKeys);
+    uint64_t thr = 0;
+    if (n >= k) thr = cta_radix_select([&](uint32_t i) { return tkeys[i]; }, n, k, ss);
+    if (threadIdx.x == 0) tau[q] = thr;
+    __syncthreads();
+  }
 }
 
 constexpr int kTopkMaxLevels = 5;
@@ -3259,6 +3345,20 @@ griffin_status run_batch(griffin_index *ix, Workspace &w, uint32_t nq, const uin
       GRIFFIN_CUDA_TRY(exclusive_scan<uint32_t>(qunits, w.unit_base.as<uint64_t>(), nq, scan_tmp, st,
                                                 &ix->launch_count));
       ix->launch_count += 1;  // plan_round (the scan counts itself)
+    }
+    ra.qtau = nullptr;
+    if (r == 1 && final_topk && ra.bm && k <= kTauKeys / 2 && nq >= 8) {
+      // 2-term word-AND queries: their top-k key threshold from a subset of
+      // their survivors (a top-k selection step: timed with the top-k stage)
+      StageTimer tt(ix, st, 3);
+      GRIFFIN_CUDA_TRY(w.qtau.reserve(((size_t)nq + 1) * 8));
+      GRIFFIN_CUDA_TRY(launch_config((const void *)bitand_tau_kernel, ix->device, tau_smem_bytes(),
+                                     1024, nullptr));
+      bitand_tau_kernel<<<std::min<uint32_t>(nq, num_sms(ix->device) * 2), 1024, tau_smem_bytes(),
+                          st>>>(di, ra, k, w.qtau.as<uint64_t>());
+      GRIFFIN_CUDA_TRY(cudaGetLastError());
+      ix->launch_count += 1;
+      ra.qtau = w.qtau.as<uint64_t>();
     }
     {
       StageTimer t(ix, st, 1);
