@@ -2303,7 +2303,8 @@ __device__ void bitonic_desc(uint64_t *s, uint32_t n) {
   for (uint32_t size = 2; size <= n; size <<= 1) {
     for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
       for (uint32_t t = threadIdx.x; t < (n >> 1); t += blockDim.x) {
-        const uint32_t lo = 2 * stride * (t / stride) + (t % stride);
+        // stride is a power of two: 2*stride*(t/stride) + t%stride without division
+        const uint32_t lo = ((t & ~(stride - 1u)) << 1) | (t & (stride - 1u));
         const uint32_t hi = lo + stride;
         const bool desc = (lo & size) == 0;
         const uint64_t x = s[lo], y = s[hi];
