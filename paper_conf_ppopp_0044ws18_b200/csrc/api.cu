@@ -212,6 +212,7 @@ static griffin_status build_shard(const griffin_corpus *c, const griffin_build_o
   if (const char *e = std::getenv("GRIFFIN_TOPK_FILTER")) ix->topk_filter = std::atoi(e);  // A/B
   if (const char *e = std::getenv("GRIFFIN_TDEC")) ix->Tdec = std::max(1, std::atoi(e));  // A/B
   if (const char *e = std::getenv("GRIFFIN_T")) ix->T = std::max(1, std::atoi(e));        // A/B
+  if (const char *e = std::getenv("GRIFFIN_TAU_MIN_QUERIES")) ix->tau_min_queries = (uint32_t)std::atoi(e);  // tests / A/B
   if (const char *e = std::getenv("GRIFFIN_SORDER")) {   // A/B probes: 0 = off, else 1 + shift
     const int v = std::atoi(e);
     ix->sorder = v > 0;

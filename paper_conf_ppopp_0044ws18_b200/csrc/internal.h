@@ -214,6 +214,8 @@ struct griffin_index {
   // Slots are per eligible term (host-assigned when the knob changes).
   uint32_t bm_inv = 32, bm_slots_inv = 0, bm_nslots = 0;
   uint32_t *d_bm_slot = nullptr, *d_bm_term = nullptr;
+  // batches of at least this many queries get the R7 subset top-k threshold
+  uint32_t tau_min_queries = 4096;
   uint64_t entry_budget = 0;   // griffin_set_entry_budget: intermediate entries per workspace (0 = exact bound)
   int profiling = 0;   // bit 0: per-stage CUDA events, bit 1: algorithmic-byte counters
   griffin_profile prof{};

@@ -512,8 +512,9 @@ def test_bitmap_decode_once_bit_exact(tiny, inv):
     gx.close()
 
 
+@pytest.mark.parametrize("tau", [True, False])
 @pytest.mark.parametrize("B", [64, 96, 128, 256, 512])
-def test_bitmap_dense_runs_and_edges(B):
+def test_bitmap_dense_runs_and_edges(B, tau, monkeypatch):
     """Bitvector construction and word-AND edge cases: lists of consecutive docIDs (whole
     words owned by one lane: plain stores), near-complete lists, docID 0 and
     N-1, word boundaries shared by lanes and blocks, multi-term queries (probe
@@ -534,6 +535,9 @@ def test_bitmap_dense_runs_and_edges(B):
     dl = rng.integers(1, 3000, size=N).astype(np.uint32)
     c = corpus_from_lists(N, lists, tfs, dl)
     ox = oracle.OracleIndex(c, block_size=B)
+    # tau: the subset top-k threshold of 2-term word-AND queries (DESIGN R7)
+    # at this small batch size too (the library applies it from 4096 queries)
+    monkeypatch.setenv("GRIFFIN_TAU_MIN_QUERIES", "8" if tau else "1000000")
     gx = g.GriffinIndex(c, block_size=B)
     gx.griffin_set_reuse(1)
     gx.griffin_set_bitmap(1 << 24)

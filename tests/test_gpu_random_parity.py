@@ -67,7 +67,12 @@ def workloads(draw):
 @given(workloads())
 def test_random_workloads_bit_exact(w):
     c, ql, B, k, mode, reuse, bitmap = w
-    gx = g.GriffinIndex(c, block_size=B)
+    import os
+    os.environ["GRIFFIN_TAU_MIN_QUERIES"] = "8"   # the R7 threshold at these small batches too
+    try:
+        gx = g.GriffinIndex(c, block_size=B)
+    finally:
+        del os.environ["GRIFFIN_TAU_MIN_QUERIES"]
     gx.griffin_set_mode(mode)
     gx.griffin_set_reuse(reuse)
     gx.griffin_set_bitmap(bitmap)
