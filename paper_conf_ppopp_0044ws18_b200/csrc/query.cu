@@ -1487,10 +1487,15 @@ __device__ __forceinline__ void bitand_unit(const DevIndex &ix, const RoundArgs 
 
 // Round-1 unit kinds run as two kernels, back to back (ROLE): 1 = the merge
 // units (the processing order puts them first: tickets [0, #merge)), 2 = the
-// gallop and single-term units (tickets [#merge, total)) with a smaller shared
-// layout (no merge tiles) and 4 CTAs/SM — they are global-latency bound
-// (skip searches, arena probes).  ROLE 0 = every unit kind in one kernel (the SvS
-// rounds without the probe pass).
+// gallop, bitvector, word-AND and single-term units (tickets [#merge, total))
+// with a smaller shared layout (no merge tiles).  It ran at 4 CTAs/SM (64
+// registers) while it held only gallop units; with the bitvector kinds it
+// spilled there, and 3 CTAs/SM without spills is faster (C5 intersect 7.58 ->
+// 7.27 ms).  ROLE 0 = every unit kind in one kernel (the SvS rounds without
+// the probe pass).
+#ifndef GRIFFIN_IK2_MINB
+#define GRIFFIN_IK2_MINB 3
+#endif
 #ifndef GRIFFIN_INTERSECT_MINB
 #define GRIFFIN_INTERSECT_MINB 3
 #endif
@@ -1502,7 +1507,7 @@ __host__ __device__ inline uint32_t other_warp_smem_words(uint32_t B, uint32_t D
   return kWarpHdr + 64 + (B + 32) + other_stage_words(B, D) + kStgSlack + other_tile_words(B, D, nextgeq);
 }
 template <int ROLE>
-struct IkMinBlocks { static constexpr int v = ROLE == 2 ? 4 : GRIFFIN_INTERSECT_MINB; };
+struct IkMinBlocks { static constexpr int v = ROLE == 2 ? GRIFFIN_IK2_MINB : GRIFFIN_INTERSECT_MINB; };
 
 template <bool RC, int ROLE>
 __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) intersect_kernel(DevIndex ix, RoundArgs a) {
