@@ -2115,9 +2115,14 @@ __global__ void __launch_bounds__(kIntersectThreads, IkMinBlocks<ROLE>::v) inter
 
 // SvS rounds 2..m-1 as one multi-list probe pass: its own kernel,
 // so it carries only the probe unit's code and shared memory (no merge tiles)
-// and runs 4 CTAs of 8 warps per SM — the pass is global-latency bound
-// (skip-pointer searches and arena probes), so more resident warps hide more.
-__global__ void __launch_bounds__(kIntersectThreads, 4) probe_kernel(DevIndex ix, RoundArgs a) {
+// at GRIFFIN_PROBE_MINB CTAs of 8 warps per SM.  The pass is global-latency
+// bound (skip-pointer searches, arena probes, bitvector lookups); 4 CTAs (64
+// registers) hid more of it until the bitvector lookups and lazy norm gathers
+// made 3 CTAs with 80 registers faster (C5 intersect 7.26 -> 7.11 ms).
+#ifndef GRIFFIN_PROBE_MINB
+#define GRIFFIN_PROBE_MINB 3
+#endif
+__global__ void __launch_bounds__(kIntersectThreads, GRIFFIN_PROBE_MINB) probe_kernel(DevIndex ix, RoundArgs a) {
   extern __shared__ uint4 smem4[];
   const uint32_t lane = lane_id();
   const uint32_t B = ix.B, D = a.D;
@@ -2404,7 +2409,10 @@ __device__ uint64_t cta_radix_select(KeyF key, uint32_t n, uint32_t kk, SelectSm
 // its top-k is >= it and bitand_unit may drop the survivors below it (exact;
 // keys are unique).  tau = 0 (no dropping) when the subset holds
 // fewer than k keys, for other queries, and when k > kTauKeys / 2.
-constexpr uint32_t kTauKeys = 8192;
+#ifndef GRIFFIN_TAU_KEYS
+#define GRIFFIN_TAU_KEYS 8192
+#endif
+constexpr uint32_t kTauKeys = GRIFFIN_TAU_KEYS;
 __host__ __device__ inline size_t tau_smem_bytes() { return (size_t)kTauKeys * 8; }
 __global__ void __launch_bounds__(1024) bitand_tau_kernel(DevIndex ix, RoundArgs a, uint32_t k,
                                                          uint64_t *tau) {
