@@ -378,6 +378,21 @@ def test_large_batch_s_locality_order(inv):
         assert prof["bitmap_units"] > 0
 
 
+def test_large_host_batch_bit_exact():
+    """A host-buffer griffin_query_batch of 9000 queries (word-AND units, the
+    S-locality order and the subset top-k threshold all engaged) equals the
+    oracle, with bitvectors on and off."""
+    c, ql, cfg = make_workload("small", num_queries=9000)
+    ox = oracle.OracleIndex(c, block_size=128)
+    od, os_, oc = ox.query_batch(ql, 10, nthreads=4)
+    for inv in (32, 0):
+        gx = g.GriffinIndex(c, block_size=128)
+        gx.griffin_set_bitmap(inv)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 10)
+        assert_topk_equal(gd, gs, gc, od, os_, oc)
+        gx.close()
+
+
 @pytest.mark.slow
 def test_c5_full_size_timed_config():
     """BASELINE configs[4] at full size (50M docs, ~1.9 B postings, 10K queries
