@@ -577,6 +577,7 @@ def run_gpu(args):
                          "gbs": sw["bytes"] / (sw["ms"] / 1e3) / 1e9,
                          "postings_per_s": sw["postings"] / (sw["ms"] / 1e3),
                          "frac_of_hbm_peak": sw["bytes"] / (sw["ms"] / 1e3) / 1e9 / peak,
+                         "alu_roofline": _sweep_alu(sw["postings"] / (sw["ms"] / 1e3)),
                          "note": "every block of the shard decoded once per launch; the index "
                                  "(> L2) is streamed from HBM"},
     }
@@ -600,6 +601,35 @@ def run_gpu(args):
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+# Warp instructions the run decoder issues per posting: ncu --set full of the
+# decode-only sweep (C2 index, B = 128): 1.48e8 warp instructions for 192,979,545
+# postings (profiles/r02s11_decode_sweep_ncu_kernels.txt).
+SWEEP_WARP_INST_PER_POSTING = 1.48e8 / 192979545
+
+
+def _sweep_alu(postings_per_s):
+    """The decode sweep against its issue roofline (it is integer-ALU / issue
+    bound, not HBM bound): achieved warp-instruction rate = postings/s x the
+    ncu-measured instructions per posting; peak = SMs x 4 schedulers x the max
+    SM clock (one warp instruction per scheduler per cycle)."""
+    try:
+        import torch
+        sms = torch.cuda.get_device_properties(0).multi_processor_count
+    except Exception:   # no device visible: the B200's count
+        sms = 148
+    mhz = 1965.0
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            mhz = float(json.load(f).get("sm_max_mhz", mhz))
+    except (OSError, ValueError):
+        pass
+    peak = sms * 4 * mhz * 1e6
+    ach = postings_per_s * SWEEP_WARP_INST_PER_POSTING
+    return {"bound": "alu", "unit": "warp instructions/s", "achieved": ach, "peak": peak,
+            "frac": ach / peak, "warp_inst_per_posting": SWEEP_WARP_INST_PER_POSTING,
+            "peak_how": f"{sms} SMs x 4 schedulers x {mhz:.0f} MHz"}
 
 
 def _ncu_traffic(config, kernel):
