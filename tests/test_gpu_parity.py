@@ -384,11 +384,12 @@ def test_large_host_batch_bit_exact():
     oracle, with bitvectors on and off."""
     c, ql, cfg = make_workload("small", num_queries=9000)
     ox = oracle.OracleIndex(c, block_size=128)
-    od, os_, oc = ox.query_batch(ql, 10, nthreads=4)
-    for inv in (32, 0):
+    # k = 1000: 72 MB of results through the pinned staging
+    for inv, k in ((32, 10), (0, 10), (32, 1000)):
+        od, os_, oc = ox.query_batch(ql, k, nthreads=4)
         gx = g.GriffinIndex(c, block_size=128)
         gx.griffin_set_bitmap(inv)
-        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, 10)
+        gd, gs, gc = gx.griffin_query_batch(ql.offsets, ql.terms, k)
         assert_topk_equal(gd, gs, gc, od, os_, oc)
         gx.close()
 
